@@ -1,0 +1,174 @@
+/*
+ * spp.h — C ABI of libspp: scientific-sample preprocessing for B200 (sm_100a).
+ *
+ * The library implements the data-parallel hot path of Ibrahim & Oliker,
+ * "Preprocessing Pipeline Optimization for Scientific Deep Learning Workloads"
+ * (IPDPS'22; /root/reference/PAPER.md, cited as P:<line>):
+ *   b.1  encode each sample once on the host            (Fig. 1 b.1)
+ *   b.4  move the compressed bytes host -> HBM           (b.4)
+ *   b.5  decode on the GPU, fused with the application's preprocessing, into
+ *        an FP16 training tensor
+ * for CosmoFlow (LUT format + ln(1+c) on the unique values)
+ * and DeepCAM (differential line format + per-channel normalisation,
+ * P:72-92).  Byte layouts and arithmetic: FORMAT.md.
+ *
+ * Conventions (all entry points):
+ *  - extern "C", little-endian, sizes in bytes.  No torch types.
+ *  - Ownership: every buffer is caller-owned.  The library never allocates or
+ *    frees caller memory; scratch comes from opts->workspace.  Only
+ *    spp_pipeline_create allocates (its own staging ring and events), freed by
+ *    spp_pipeline_destroy.
+ *  - Host-checkable argument errors return immediately and enqueue nothing.
+ *    Stream corruption is detected on the device and reported through
+ *    opts->status (the first error wins); the affected sample's output is
+ *    unspecified, no out-of-bounds access happens.
+ *  - Device calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
+ *    default stream), on the current CUDA device, never synchronise the host
+ *    and never allocate.
+ *  - There is no CPU fallback: a device call without a usable sm_100 GPU
+ *    returns SPP_ERR_CUDA.
+ */
+#ifndef SPP_H
+#define SPP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *spp_stream_t; /* identical to cudaStream_t */
+
+typedef enum {
+    SPP_OK = 0,
+    SPP_ERR_INVALID_ARG = 1,      /* null pointer, bad dims, bad enum, misalignment */
+    SPP_ERR_BUFFER_TOO_SMALL = 2, /* dst / workspace / staging too small; *encoded_size = required */
+    SPP_ERR_CORRUPT = 3,          /* malformed stream (device status, or host-side parse) */
+    SPP_ERR_UNSUPPORTED = 4,      /* legal by FORMAT.md but outside the GPU path's limits */
+    SPP_ERR_CUDA = 5              /* CUDA runtime error (no device, launch failure, ...) */
+} spp_status;
+
+typedef enum { SPP_FMT_COSMO = 1, SPP_FMT_DEEPCAM = 2 } spp_format;
+
+typedef enum {
+    SPP_OUT_F16 = 1, /* IEEE binary16, RNE from the fp32 value ("FP16 samples") */
+    SPP_OUT_F32 = 2, /* IEEE binary32 */
+    SPP_OUT_I16 = 3  /* CosmoFlow with transform = 0 only: the decoded int16 counts */
+} spp_out;
+
+/* ------------------------------------------------------------------------ */
+/* Host encoders (b.1).  Reentrant and thread-safe, no global state, no
+ * CUDA.  On SPP_ERR_BUFFER_TOO_SMALL, *encoded_size holds the required size. */
+
+/* Upper bound of spp_encode_cosmo's output for a C x D x H x W volume. */
+size_t spp_cosmo_max_encoded_size(int C, int D, int H, int W);
+
+/* CosmoFlow LUT encoder (FORMAT.md 1.3; P:98-100 unique values and 4-groups,
+ * P:106 1/2-byte keys with 8-byte lookup values).
+ *   counts : host int16 [C][D][H][W] (CDHW), every value >= 0 (P:96 particle
+ *            counts; negative -> SPP_ERR_INVALID_ARG)
+ *   C      : must be 4 (four redshifts)
+ *   dst    : host buffer of dst_capacity bytes, 16-B aligned not required
+ * Output is deterministic: same input -> same bytes. */
+spp_status spp_encode_cosmo(const int16_t *counts, int C, int D, int H, int W,
+                            void *dst, size_t dst_capacity, size_t *encoded_size);
+
+/* Upper bound of spp_encode_deepcam's output for C x H x W. */
+size_t spp_deepcam_max_encoded_size(int C, int H, int W);
+
+/* DeepCAM differential line encoder (FORMAT.md 2.4; Fig. 4).
+ *   x : host fp32 [C][H][W] (CHW); lines are rows of W values along x.
+ *       Non-finite values are legal and force a RAW (uncompressed) line.
+ * Lossy within the bound of DESIGN.md reading S19; deterministic. */
+spp_status spp_encode_deepcam(const float *x, int C, int H, int W,
+                              void *dst, size_t dst_capacity, size_t *encoded_size);
+
+/* Host-side parse of one encoded sample's header (no CUDA).  For CosmoFlow
+ * info[0..3] = nU, nslab, G of slab 0, kw of slab 0; for DeepCAM info[0..3] =
+ * number of RAW lines, SEG lines, total segments, total delta bytes.
+ * Returns SPP_ERR_CORRUPT on a malformed stream. */
+spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, int64_t info[4]);
+
+/* ------------------------------------------------------------------------ */
+/* Device decode (b.5). */
+
+typedef struct {
+    int out;                 /* spp_out: SPP_OUT_F16 (default) | SPP_OUT_F32 | SPP_OUT_I16 */
+    int transform;           /* CosmoFlow: 1 = ln(1+c) (default), 0 = identity */
+    const float *shift;      /* DeepCAM: device fp32[C] or NULL (= 0)   y = (x - shift) * scale */
+    const float *scale;      /* DeepCAM: device fp32[C] or NULL (= 1)   (reading S18) */
+    uint32_t *status;        /* optional device word; 0 = ok, else (spp_status | sample << 8) of
+                                the first corrupt sample.  The caller zeroes it. */
+    const uint64_t *src_bytes; /* optional device u64[n]: size of each source buffer; when given,
+                                  every read is bounds-checked against it as well */
+    void *workspace;         /* device scratch >= spp_decode_workspace_size(), 256-B aligned */
+    size_t workspace_size;
+    int C, D, H, W;          /* expected dims (CosmoFlow C=4,D,H,W; DeepCAM C,H,W with D ignored);
+                                every sample header must match (else CORRUPT in status) */
+} spp_decode_opts;
+
+/* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */
+void spp_decode_opts_init(spp_decode_opts *opts, spp_format fmt, int C, int D, int H, int W);
+
+/* Bytes of device workspace spp_decode_batch needs for n samples. */
+size_t spp_decode_workspace_size(spp_format fmt, int n, const spp_decode_opts *opts);
+
+/* Bytes of one decoded sample (C*D*H*W or C*H*W elements times the out size). */
+size_t spp_decoded_sample_bytes(spp_format fmt, const spp_decode_opts *opts);
+
+/* Decode + preprocess a batch of n encoded samples resident in HBM.
+ *   d_src : DEVICE array of n DEVICE pointers, each to a 16-B aligned stream
+ *   d_dst : device output, n samples back to back, [n][C][D][H][W] (CosmoFlow,
+ *           CDHW: the transpose is fused) or [n][C][H][W] (DeepCAM),
+ *           16-B aligned
+ * Launches the sm_100a kernels (CosmoFlow: transform of the unique values then
+ * the fused LUT expansion; DeepCAM: header/directory parse then the warp-per-line
+ * differential decode) on `stream`.  Returns after enqueueing. */
+spp_status spp_decode_batch(spp_format fmt, const void *const *d_src, int n, void *d_dst,
+                            const spp_decode_opts *opts, spp_stream_t stream);
+
+/* Number of kernel launches one spp_decode_batch call enqueues (for accounting). */
+int spp_decode_launches(spp_format fmt);
+
+/* ------------------------------------------------------------------------ */
+/* Streamed decode from host memory (b.4 + b.5): the compressed bytes are
+ * copied host -> device in chunks on a copy stream, overlapped with the
+ * decode of the previous chunk on `stream` (double/triple buffered staging
+ * ring owned by the pipeline).  Host sources should be pinned
+ * (cudaHostAlloc / cudaHostRegister) for the copies to be asynchronous. */
+typedef struct spp_pipeline spp_pipeline;
+
+/*   slot_bytes : capacity of one staging slot (>= the largest chunk of samples)
+ *   nslots     : ring depth (2..8)
+ *   max_chunk  : maximum samples per chunk (decode launch)
+ * Allocates device staging (nslots * slot_bytes), a pinned descriptor area,
+ * a device workspace, events and a copy stream on the current device. */
+spp_status spp_pipeline_create(spp_pipeline **out, spp_format fmt, const spp_decode_opts *opts,
+                               size_t slot_bytes, int nslots, int max_chunk);
+void spp_pipeline_destroy(spp_pipeline *p);
+
+/* Decode n host-resident samples into d_dst (layout as spp_decode_batch).
+ *   h_src     : HOST array of n HOST pointers (pinned for async copies)
+ *   src_bytes : HOST array of n sizes (multiples of 16)
+ *   opts      : as spp_decode_batch; opts->workspace/src_bytes are ignored
+ *               (the pipeline owns its workspace)
+ * All work is enqueued on `stream` (decode) and the pipeline's copy stream; the
+ * call returns when everything is enqueued (it may block only while the
+ * staging ring is full). */
+spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size_t *src_bytes,
+                           int n, void *d_dst, const spp_decode_opts *opts, spp_stream_t stream);
+
+/* Number of decode launches and copies the last spp_decode_host call enqueued. */
+int spp_pipeline_last_launches(const spp_pipeline *p);
+
+const char *spp_status_string(spp_status s);
+
+/* Library build identification: "spp <version> sm_100a". */
+const char *spp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SPP_H */

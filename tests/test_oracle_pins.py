@@ -1,0 +1,429 @@
+"""Pins of the CPU oracle to things other than itself (no GPU needed).
+
+Each test names what fixes the expected value: IEEE-754 exact arithmetic
+(Fractions), a library routine (numpy float16 conversion, mpmath), brute force
+over sets on tiny inputs, closed forms from the paper, or special cases.
+PAPER.md lines are cited as P:<n>; readings S<n> are listed in DESIGN.md.
+"""
+import json
+import struct
+from fractions import Fraction
+from pathlib import Path
+
+import mpmath
+import numpy as np
+import pytest
+
+from tests import exact, fmt
+
+GOLDEN = Path(__file__).parent / "golden"
+
+
+# --------------------------------------------------------------------------
+# binary32 -> binary16 RNE (FORMAT.md 1.2 / 2.3 emission; P:110 FP16 samples)
+# pinned against numpy's conversion (library routine)
+
+def test_f16_conversion_matches_numpy(orc):
+    rng = np.random.default_rng(7)
+    bits = rng.integers(0, 2**32, size=400_000, dtype=np.uint64).astype(np.uint32)
+    # every half value, its neighbours' midpoints and +-1 binary32 ulp around them
+    h = np.arange(0, 0x7C00, dtype=np.uint16).view(np.float16).astype(np.float32)
+    mids = ((h[:-1].astype(np.float64) + h[1:].astype(np.float64)) / 2).astype(np.float32)
+    extra = np.concatenate([h, mids, np.nextafter(mids, np.float32(np.inf)),
+                            np.nextafter(mids, np.float32(0)), np.float32([65504, 65519.99, 65520, 7e4, 1e-8,
+                                                                           2**-25, 2**-24, 3 * 2**-26, np.inf])])
+    x = np.concatenate([bits.view(np.float32), extra, -extra])
+    got = orc.f32_to_f16(x)
+    with np.errstate(over="ignore"):
+        ref = x.astype(np.float16).view(np.uint16)
+    nan = np.isnan(x)
+    assert np.array_equal(got[~nan], ref[~nan])
+    assert np.all(np.isnan(got[nan].view(np.float16)))
+
+
+# --------------------------------------------------------------------------
+# CosmoFlow transform: RN_f32(ln(1+c)) (readings S1/S2), exhaustive vs mpmath
+
+def _mp_f32_log1p(c: int) -> np.float32:
+    with mpmath.workprec(200):
+        v = mpmath.log1p(c)
+        m, e = mpmath.mpf(v).man_exp
+        q = Fraction(int(m)) * (Fraction(2) ** int(e)) if e >= 0 else Fraction(int(m), 2 ** (-int(e)))
+    return exact.to_f32(q), q
+
+
+def test_cosmo_transform_exhaustive_mpmath(orc):
+    table = orc.cosmo_transform_table()
+    bad = []
+    for c in range(32768):
+        ref, _ = _mp_f32_log1p(c)
+        if table[c].view(np.uint32) != ref.view(np.uint32):
+            bad.append(c)
+    assert bad == []
+    # fp16 = RNE_f16(the fp32 value) ("casting to FP16")
+    f16 = orc.f32_to_f16(table).view(np.float16)
+    for c in (0, 1, 2, 100, 558, 10363, 15316, 32767):
+        assert f16[c] == exact.to_f16(Fraction(float(table[c])))
+
+
+def test_cosmo_fp16_double_rounding_cases(orc):
+    """Reading S2: fp16 is rounded from the fp32 value.  At these counts that
+    differs from rounding the exact logarithm directly (documented cases)."""
+    found = []
+    table = orc.cosmo_transform_table()
+    f16 = orc.f32_to_f16(table).view(np.float16)
+    for c in range(32768):
+        _, q = _mp_f32_log1p(c)
+        if exact.to_f16(q) != f16[c]:
+            found.append(c)
+    golden = json.loads((GOLDEN / "cosmo_fp16_double_rounding.json").read_text())
+    assert found == golden["counts"]
+
+
+def test_cosmo_direct_special_values(orc):
+    x = np.array([0, 1, 2, 3, 32767], dtype=np.int16)
+    f32 = orc.cosmo_direct(x, 1, "f32")
+    assert f32[0] == 0.0 and f32.view(np.uint32)[0] == 0          # ln(1) = +0 exactly
+    assert f32[1] == np.float32(np.log(2.0))                      # RN(ln 2)
+    assert orc.cosmo_direct(x, 0, "i16").tolist() == x.tolist()   # identity
+    assert orc.cosmo_direct(x, 0, "f32").tolist() == [0, 1, 2, 3, 32767]
+    with pytest.raises(orc.OracleError):
+        orc.cosmo_direct(np.array([-1], dtype=np.int16), 1, "f32")   # reading S7
+
+
+# --------------------------------------------------------------------------
+# CosmoFlow LUT format: brute force over sets on tiny volumes
+
+def _tiny_volumes():
+    rng = np.random.default_rng(11)
+    vols = []
+    for n in (1, 2, 3, 4, 8):
+        vols.append(rng.integers(0, 5, size=(4, n, n, n)).astype(np.int16))      # few values
+        vols.append((rng.pareto(1.5, size=(4, n, n, n)) * 3).astype(np.int16))  # power-law
+    vols.append(np.zeros((4, 5, 3, 2), dtype=np.int16))                         # all equal -> kw 0
+    vols.append(np.full((4, 6, 4, 4), 7, dtype=np.int16))
+    v = rng.integers(0, 3, size=(1, 6, 5, 7)).astype(np.int16)
+    vols.append(np.concatenate([v, v + 1, v * 2, v], axis=0))                   # fully coupled
+    vols.append(np.arange(4 * 4 * 4 * 4, dtype=np.int16).reshape(4, 4, 4, 4))   # all distinct
+    return vols
+
+
+@pytest.mark.parametrize("vi", range(14))
+def test_cosmo_encoder_bruteforce_tiny(orc, vi):
+    x = _tiny_volumes()[vi]
+    b = orc.cosmo_encode(x)
+    h = fmt.cosmo_header(b)
+    _, D, H, W = x.shape
+    N = D * H * W
+    assert h["magic"] == 0x43505053 and h["ver"] == 1 and (h["C"], h["D"], h["H"], h["W"]) == (4, D, H, W)
+    assert h["total"] == b.size and b.size % 16 == 0
+    # |U| = |set of values|, U ascending
+    assert h["U"].tolist() == sorted(set(x.ravel().tolist()))
+    Uidx = {v: i for i, v in enumerate(h["U"].tolist())}
+    flat = x.reshape(4, N)
+    assert h["T"] == 1  # tiny volumes never need a split
+    s = h["slabs"][0]
+    tuples = [tuple(Uidx[int(flat[c, v])] for c in range(4)) for v in range(N)]
+    G = len(set(tuples))
+    if s["kw"] == 8:
+        assert 8 * G + (0 if G == 1 else (1 if G <= 256 else 2)) * N >= 8 * N
+        raw = fmt.cosmo_keys(b, s, N)
+        assert [tuple(int(raw[c, v]) for c in range(4)) for v in range(N)] == tuples
+    else:
+        assert s["G"] == G
+        assert s["kw"] == (0 if G == 1 else (1 if G <= 256 else 2))
+        lut = [tuple(int(t) for t in row) for row in fmt.cosmo_lut(b, s)]
+        assert sorted(lut) == sorted(set(tuples))
+        freq = {t: tuples.count(t) for t in set(tuples)}
+        assert lut == sorted(set(tuples), key=lambda t: (-freq[t], t))   # FORMAT.md 1.3 step 4
+        keys = fmt.cosmo_keys(b, s, N)
+        assert [lut[int(k)] for k in keys] == tuples
+    # lossless round trip against the plain definition
+    for out in ("f32", "f16"):
+        dec = orc.cosmo_decode(b, x.shape, 1, out)
+        ref = orc.cosmo_direct(x, 1, out)
+        assert dec.tobytes() == ref.tobytes()
+    assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
+
+
+def test_cosmo_slab_split_and_raw_escape(orc):
+    rng = np.random.default_rng(5)
+    # ~2 x 65536 distinct groups over 8 planes of 128x128, coupled enough that a
+    # half-volume fits 16-bit keys: split into slabs, each kw = 2
+    D, H, W = 8, 128, 128
+    N = D * H * W
+    base = rng.integers(0, 150000, size=N)  # group id per voxel
+    g = np.array([base % 7, (base // 7) % 11, (base // 77) % 13, (base // 1001) % 151], dtype=np.int16)
+    # confine ids per half so each half has <= 65536 groups
+    half = N // 2
+    ids = np.concatenate([rng.integers(0, 60000, size=half), rng.integers(60000, 120000, size=half)])
+    g = np.array([ids % 7, (ids // 7) % 11, (ids // 77) % 13, (ids // 1001) % 151], dtype=np.int16).reshape(4, D, H, W)
+    b = orc.cosmo_encode(g)
+    h = fmt.cosmo_header(b)
+    assert h["T"] >= 2
+    assert [(s["z0"], s["z1"]) for s in h["slabs"]][0][0] == 0 and h["slabs"][-1]["z1"] == D
+    for s in h["slabs"]:
+        assert s["kw"] in (2, 8) and s["G"] <= 65536
+    assert np.array_equal(orc.cosmo_decode(b, g.shape, 0, "i16"), g)
+    # dense independent volume: LUT would not save space -> RAW escape (kw 8)
+    y = rng.integers(0, 200, size=(4, 2, 64, 64)).astype(np.int16)
+    hb = orc.cosmo_encode(y)
+    hh = fmt.cosmo_header(hb)
+    assert all(s["kw"] == 8 and s["G"] == 0 for s in hh["slabs"])
+    assert orc.cosmo_decode(hb, y.shape, 1, "f32").tobytes() == orc.cosmo_direct(y, 1, "f32").tobytes()
+
+
+def test_cosmo_size_closed_form_and_paper_ratio(orc):
+    """P:98 'compression factor of roughly 4x' vs gzip 5x; P:219 gzip files are
+    'roughly 75%' of ours.  Layout size = 64 + up16(2|U|) + 32 + up16(8G) + 2N."""
+    paper = json.loads((GOLDEN / "paper_numbers.json").read_text())
+    up16 = lambda v: (v + 15) // 16 * 16
+    N = 128 ** 3
+    G, nU = paper["cosmo_example_groups"]["value"], paper["cosmo_example_unique_values"]["value"]
+    size = 64 + up16(2 * nU) + 32 + up16(8 * G) + 2 * N
+    ratio = 4 * N * 2 / size
+    assert 3.6 < ratio < 4.0                                   # "roughly 4x"
+    assert 0.70 < ratio / paper["gzip_ratio"]["value"] < 0.80   # "roughly 75%"
+    # the oracle's encoder produces exactly the closed-form size
+    rng = np.random.default_rng(3)
+    D = H = W = 16
+    n = D * H * W
+    gid = rng.integers(0, 300, size=n)
+    gid[:300] = np.arange(300)          # every group present: G = 300 -> kw = 2
+    vol = np.array([gid % 5, gid % 7, gid // 5, gid // 7], dtype=np.int16).reshape(4, D, H, W)
+    b = orc.cosmo_encode(vol)
+    h = fmt.cosmo_header(b)
+    nU2 = len(set(vol.ravel().tolist()))
+    assert h["slabs"][0]["G"] == 300 and h["slabs"][0]["kw"] == 2
+    assert b.size == 64 + up16(2 * nU2) + 32 + up16(8 * 300) + up16(2 * n)
+
+
+def test_cosmo_paper_shaped_sample(orc):
+    """Generator 'paper' preset lands near the paper's example (Fig. 5):
+    hundreds of unique values, tens of thousands of 4-groups, 2-byte keys."""
+    from synth import gen_cosmo
+    x = gen_cosmo(1001)
+    b = orc.cosmo_encode(x)
+    h = fmt.cosmo_header(b)
+    assert 300 <= h["nU"] <= 1500
+    assert h["T"] == 1 and 10_000 <= h["slabs"][0]["G"] <= 65_536 and h["slabs"][0]["kw"] == 2
+    assert 3.4 < x.nbytes / b.size < 4.2
+    assert orc.cosmo_decode(b, x.shape, 1, "f16").tobytes() == orc.cosmo_direct(x, 1, "f16").tobytes()
+
+
+def test_cosmo_decoder_rejects_corruption(orc):
+    x = _tiny_volumes()[6]
+    b = orc.cosmo_encode(x)
+    for off, val in ((0, 0x00), (4, 0x02), (20, 0x00), (8, 0x03)):
+        c = b.copy(); c[off] = val
+        with pytest.raises(orc.OracleError):
+            orc.cosmo_decode(c, x.shape, 1, "f32")
+    with pytest.raises(orc.OracleError):
+        orc.cosmo_decode(b[:48], x.shape, 1, "f32")
+
+
+# --------------------------------------------------------------------------
+# DeepCAM 8-bit delta code (1 sign bit, 3 exponent bits, 4 mantissa bits)
+
+def test_delta_code_table_characterisation(orc):
+    codes = [orc.deepcam_code(b) for b in range(256)]
+    mags = codes[:128]
+    # sign bit: b and b^0x80 decode to opposite values
+    assert all(codes[b] == -codes[b ^ 0x80] for b in range(256))
+    # magnitudes strictly increase with the 7-bit exponent|mantissa field
+    assert all(mags[i] < mags[i + 1] for i in range(127))
+    # a float with 4 stored mantissa bits (5 significant with the hidden bit):
+    # the magnitude set is exactly the integers <= 31*64 with <= 5 significant bits
+    def five_bits(n):
+        if n < 32:
+            return True
+        s = n >> (n.bit_length() - 5)
+        return n == s << (n.bit_length() - 5)
+    assert set(mags) == {n for n in range(0, 31 * 64 + 1) if five_bits(n)}
+    assert len(set(mags)) == 128 and max(mags) == 1984 and mags[0] == 0
+    # 3-bit exponent field groups magnitudes into 8 classes (E=0 is the linear range)
+    for E in range(8):
+        grp = mags[16 * E:16 * E + 16]
+        steps = {grp[i + 1] - grp[i] for i in range(15)}
+        assert steps == {1 if E <= 1 else 2 ** (E - 1)}
+
+
+# --------------------------------------------------------------------------
+# DeepCAM reconstruction: exact rational arithmetic on hand-built lines
+
+def _expected_line(W, segs, deltas, code):
+    """Exact value of FORMAT.md 2.3 using Fractions, rounded RNE to fp32."""
+    out, pos, dp = [], 0, 0
+    for ln, kind, eb, h in segs:
+        h = np.float32(h)
+        if kind == 0:
+            out += [h] * ln
+        else:
+            S = 0
+            out.append(h)
+            for j in range(1, ln):
+                S += code[deltas[dp]]
+                dp += 1
+                if S == 0:
+                    out.append(h)
+                else:
+                    out.append(exact.to_f32(exact.frac(h) + S * Fraction(2) ** (eb - 150)))
+        pos += ln
+    assert pos == W
+    return np.array(out, dtype=np.float32)
+
+
+def _random_segs(rng, W, code):
+    segs, deltas, pos = [], [], 0
+    while pos < W:
+        ln = int(min(W - pos, rng.integers(1, 24)))
+        kind = int(rng.random() < 0.8)
+        eb = int(rng.choice([1, 2, 20, 100, 130, 140, 147, 148, 150, 160, 200, 246]))
+        hk = rng.integers(0, 6)
+        h = [0.0, -0.0, 1.0, float(rng.standard_normal() * 10.0 ** rng.integers(-40, 38)),
+             float(np.float32(2.0 ** -140)), float(rng.standard_normal())][hk]
+        segs.append((ln, kind, eb, np.float32(h)))
+        if kind == 1:
+            deltas += [int(v) for v in rng.integers(0, 256, size=ln - 1)]
+        pos += ln
+    return segs, deltas
+
+
+def test_deepcam_reconstruction_exact_rational(orc):
+    rng = np.random.default_rng(1234)
+    code = [orc.deepcam_code(b) for b in range(256)]
+    n_sub = 0
+    for trial in range(300):
+        W = int(rng.integers(1, 40))
+        segs, deltas = _random_segs(rng, W, code)
+        line = fmt.build_seg_line(W, segs, deltas)
+        stream = fmt.build_deepcam_stream(1, 1, W, [line])
+        got = orc.deepcam_decode_line(stream, 0, W)
+        with np.errstate(over="ignore"):
+            want = _expected_line(W, segs, deltas, code)
+        same = (got.view(np.uint32) == want.view(np.uint32))
+        assert same.all(), (trial, np.nonzero(~same))
+        n_sub += int(np.sum((np.abs(want) < np.float32(2.0 ** -126)) & (want != 0)))
+    assert n_sub > 0   # subnormal reconstructions were exercised (no FTZ)
+
+
+def test_deepcam_raw_and_repeat_lines(orc):
+    W = 20
+    x = np.array([np.nan, np.inf, -np.inf, -0.0, 1e-45, 3.4e38] + [1.5] * 14, dtype=np.float32)
+    raw = fmt.build_raw_line(x)
+    rep = fmt.build_seg_line(W, [(W, 0, 0, np.float32(-0.0))], [])
+    s = fmt.build_deepcam_stream(1, 2, W, [raw, rep])
+    a = orc.deepcam_decode_line(s, 0, W)
+    assert np.array_equal(a.view(np.uint32), x.view(np.uint32))        # RAW is verbatim
+    r = orc.deepcam_decode_line(s, 1, W)
+    assert np.all(r.view(np.uint32) == np.float32(-0.0).view(np.uint32))  # REPEAT keeps -0.0
+
+
+def test_deepcam_normalisation_all_raw_matches_numpy(orc):
+    """P8: with every line RAW the output is numpy's two-rounding fp32 formula
+    then the library fp16 cast (reading S18)."""
+    rng = np.random.default_rng(9)
+    C, H, W = 3, 4, 24
+    x = (rng.standard_normal((C, H, W)) * 1e3).astype(np.float32)
+    x[0, 0, 0] = np.nan
+    lines = [fmt.build_raw_line(x[c, y]) for c in range(C) for y in range(H)]
+    s = fmt.build_deepcam_stream(C, H, W, lines)
+    shift = np.float32([1.5, -250.0, 3e3])
+    scale = np.float32([0.5, 1.0 / 3.0, 1e-3])
+    ref32 = ((x - shift[:, None, None]).astype(np.float32) * scale[:, None, None]).astype(np.float32)
+    got32 = orc.deepcam_decode(s, (C, H, W), shift, scale, "f32")
+    nan = np.isnan(ref32)
+    assert np.array_equal(got32[~nan].view(np.uint32), ref32[~nan].view(np.uint32)) and np.isnan(got32[nan]).all()
+    got16 = orc.deepcam_decode(s, (C, H, W), shift, scale, "f16")
+    ref16 = ref32.astype(np.float16)
+    assert np.array_equal(got16[~nan].view(np.uint16), ref16[~nan].view(np.uint16))
+    # no shift/scale: fp32 output is x-hat itself
+    assert np.array_equal(orc.deepcam_decode(s, (C, H, W), out="f32")[~nan].view(np.uint32), x[~nan].view(np.uint32))
+
+
+# --------------------------------------------------------------------------
+# DeepCAM encoder: per-value error bound (reading S19) and the paper statistic
+
+def _check_bound(x_line, xh_line, seg_info):
+    """|x̂_j - x_j| <= ½ulp(x̂_j) + ½ulp(x̂_{j-1}) + max(1/2, |t|/32)·2^emin (exact)."""
+    pos = 0
+    for s in seg_info:
+        ln = s["len"]
+        if s["kind"] == 0:
+            assert all(xh_line[pos + j].view(np.uint32) == x_line[pos + j].view(np.uint32) for j in range(ln))
+        else:
+            assert xh_line[pos].view(np.uint32) == x_line[pos].view(np.uint32)  # head exact
+            u = Fraction(2) ** s["emin"]
+            for j in range(1, ln):
+                p = pos + j
+                t = (exact.frac(x_line[p]) - exact.frac(xh_line[p - 1])) / u
+                bound = exact.ulp32(xh_line[p]) / 2 + exact.ulp32(xh_line[p - 1]) / 2 + max(Fraction(1, 2), abs(t) / 32) * u
+                assert abs(exact.frac(xh_line[p]) - exact.frac(x_line[p])) <= bound, (p, t)
+        pos += ln
+
+
+def test_deepcam_encoder_error_bound_and_roundtrip(orc):
+    rng = np.random.default_rng(21)
+    C, H, W = 2, 6, 300
+    x = np.cumsum(rng.standard_normal((C, H, W)) * 0.01, axis=2).astype(np.float32) + 250.0
+    x[1] = np.where(rng.random((H, W)) < 0.9, 0.0, rng.random((H, W)) * 1e-6).astype(np.float32)  # sparse
+    x[0, 3, 100:140] = 7.0                              # a repeat run
+    x[0, 5, 200] = np.inf                               # forces RAW
+    b = orc.deepcam_encode(x)
+    h = fmt.deepcam_header(b)
+    assert h["L"] == C * H and b.size == h["total"]
+    for c in range(C):
+        for y in range(H):
+            l = c * H + y
+            xh = orc.deepcam_decode_line(b, l, W)
+            info = fmt.deepcam_line(b, h, l)
+            if info["mode"] == 0:
+                assert np.array_equal(xh.view(np.uint32), x[c, y].view(np.uint32))
+            else:
+                assert sum(s["len"] for s in info["segs"]) == W
+                _check_bound(x[c, y], xh, info["segs"])
+    assert fmt.deepcam_line(b, h, 5)["mode"] == 0
+    assert any(s["kind"] == 0 for s in fmt.deepcam_line(b, h, 3)["segs"])
+
+
+def test_deepcam_paper_statistic(orc):
+    """roughly 3% of values with more than 10% error, mostly near
+    zero.  Soft acceptance on the paper-shaped generator (reading S19)."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2001, H=192)
+    b = orc.deepcam_encode(x)
+    xh = orc.deepcam_decode(b, x.shape, out="f32")
+    rel = np.abs(xh.astype(np.float64) - x) / np.maximum(np.abs(x.astype(np.float64)), 1e-300)
+    rel[(x == 0) & (xh == 0)] = 0.0
+    frac_bad = float((rel > 0.1).mean())
+    assert frac_bad <= 0.035
+    # large errors are near zero: their |x| is far below each channel's scale
+    bad = rel > 0.1
+    scale = np.abs(x).reshape(x.shape[0], -1).max(axis=1)[:, None, None]
+    assert np.median((np.abs(x) / scale)[bad]) < 0.05
+    assert x.nbytes / b.size > 3.0                     # it compresses
+
+
+def test_deepcam_special_shapes(orc):
+    for (C, H, W) in ((1, 1, 1), (1, 3, 2), (2, 2, 17), (1, 1, 16)):
+        x = np.random.default_rng(C * 100 + W).standard_normal((C, H, W)).astype(np.float32)
+        b = orc.deepcam_encode(x)
+        xh = orc.deepcam_decode(b, (C, H, W), out="f32")
+        assert xh.shape == (C, H, W) and np.isfinite(xh).all()
+    x = np.full((1, 2, 64), 3.25, dtype=np.float32)          # constant lines -> REPEAT, exact
+    b = orc.deepcam_encode(x)
+    info = fmt.deepcam_line(b, fmt.deepcam_header(b), 0)
+    assert info["mode"] == 1 and info["nseg"] == 1 and info["segs"][0]["kind"] == 0
+    assert np.array_equal(orc.deepcam_decode(b, x.shape, out="f32"), x)
+
+
+def test_deepcam_decoder_rejects_corruption(orc):
+    W = 8
+    good = fmt.build_seg_line(W, [(4, 1, 140, 1.0), (4, 0, 0, 2.0)], [1, 2, 3])
+    bad_len = fmt.build_seg_line(W, [(4, 1, 140, 1.0), (5, 0, 0, 2.0)], [1, 2, 3])
+    bad_kind = fmt.build_seg_line(W, [(4, 3, 140, 1.0), (4, 0, 0, 2.0)], [1, 2, 3])
+    bad_emin = fmt.build_seg_line(W, [(4, 1, 0, 1.0), (4, 0, 0, 2.0)], [1, 2, 3])
+    orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [good]), 0, W)
+    for ln in (bad_len, bad_kind, bad_emin):
+        with pytest.raises(orc.OracleError):
+            orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [ln]), 0, W)
