@@ -369,8 +369,7 @@ int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat)
             xhat[pos] = h;
             for (int j = 1; j < len; j++) {
                 S += orc_deepcam_code(p[dpos + (uint64_t)(j - 1)]);
-                if (S == 0) xhat[pos + j] = h;
-                else xhat[pos + j] = h + (float)S * unit;  /* fp32: exact product, one rounding */
+                xhat[pos + j] = h + (float)S * unit;     /* fp32: exact product, one rounding */
             }
             dpos += (uint64_t)(len - 1);
         } else {
@@ -475,7 +474,7 @@ static int64_t encode_line(const float *x, int W, seg_t *segs, int *nseg_out, ui
             int k = orc_deepcam_code(b);
             if (llabs(S + k) > 1983LL * 1984LL) break;
             S += k;
-            float xh = (S == 0) ? h : h + (float)S * unit;
+            float xh = h + (float)S * unit;
             if (deltas) deltas[nd] = (uint8_t)b;
             nd++;
             prev = xh;

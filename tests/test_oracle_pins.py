@@ -264,10 +264,10 @@ def _expected_line(W, segs, deltas, code):
             for j in range(1, ln):
                 S += code[deltas[dp]]
                 dp += 1
-                if S == 0:
-                    out.append(h)
-                else:
-                    out.append(exact.to_f32(exact.frac(h) + S * Fraction(2) ** (eb - 150)))
+                v = exact.to_f32(exact.frac(h) + S * Fraction(2) ** (eb - 150))
+                if v == 0:
+                    v = np.float32(0.0)      # exact sum zero: RN gives +0 (h = -0 with S = 0 too)
+                out.append(v)
         pos += ln
     assert pos == W
     return np.array(out, dtype=np.float32)
