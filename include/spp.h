@@ -106,6 +106,9 @@ typedef struct {
     size_t workspace_size;
     int C, D, H, W;          /* expected dims (CosmoFlow C=4,D,H,W; DeepCAM C,H,W with D ignored);
                                 every sample header must match (else CORRUPT in status) */
+    void *const *timing_events; /* optional host array of 3 cudaEvent_t, recorded on `stream`
+                                   before the prologue kernel, between the prologue and the main
+                                   kernel, and after the main kernel (live per-kernel timing) */
 } spp_decode_opts;
 
 /* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */

@@ -1,0 +1,438 @@
+// cosmo.cu — CosmoFlow decode + log-preprocess on sm_100a (FORMAT.md 1.2).
+//
+// PAPER.md §V.B and §VI: a sample is a per-sample lookup
+// table of 4-groups (8-byte values of four 16-bit indices into the unique
+// count set U) plus one 1- or 2-byte key per voxel.  The log transform is
+// applied to U only, before expansion, and the four redshift planes
+// are written directly in the training layout (fused transpose).
+//
+// Two kernels per batch:
+//   KC0  kc0_prologue   one CTA per sample: validate header + slab table,
+//                        fU[i] = RN_fp32(log1p(U[i])) (or the identity) into
+//                        the workspace.  |U| is hundreds, so this is ~10^3
+//                        transcendental evaluations per 8M outputs.
+//   KC   kc_expand      persistent CTAs over (sample, voxel chunk) items,
+//                        contiguous per CTA.  Each CTA stages the hottest
+//                        groups of the current slab (keys are frequency-ordered
+//                        by the encoder) as ready-to-store output tuples
+//                        T[g] = (f(U[e0]),..,f(U[e3])) in shared memory; cold
+//                        keys rebuild the tuple from the L1/L2-resident LUT.
+//                        Each thread handles 8 consecutive voxels: one 16-B key
+//                        load, 8 smem gathers, four 16-B (fp16) streaming
+//                        stores, one per redshift plane.
+// HBM traffic per sample = keys + LUT + U + outputs; everything else is
+// on-chip or L2.
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "spp_format.h"
+#include "spp_internal.h"
+
+namespace spp {
+namespace {
+
+using namespace spp::cosmo;
+
+struct CosmoMeta {  // written by KC0, read by KC
+    uint32_t valid;
+    uint32_t nU;
+    uint32_t nslab;
+    uint32_t pad;
+};
+
+constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
+constexpr int kThreads = 256;
+constexpr int kHotBytes = 64 * 1024;  // shared-memory hot prefix of T per CTA
+
+size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
+
+// --------------------------------------------------------------------------
+// KC0: header/slab validation and the unique-value transform
+__global__ void __launch_bounds__(kThreads) kc0_prologue(const void *const *__restrict__ src,
+                                                         const uint64_t *__restrict__ src_bytes, int transform,
+                                                         int D, int H, int W, float *__restrict__ fU_ws,
+                                                         CosmoMeta *__restrict__ meta,
+                                                         uint32_t *__restrict__ status) {
+    const int s = blockIdx.x;
+    const uint8_t *b = static_cast<const uint8_t *>(src[s]);
+    __shared__ uint32_t sh_ok, sh_nU, sh_T;
+    __shared__ uint64_t sh_Uoff;
+    if (threadIdx.x == 0) {
+        uint32_t ok = b != nullptr && (reinterpret_cast<uintptr_t>(b) & 15) == 0;
+        uint64_t limit = src_bytes ? src_bytes[s] : ~0ull;
+        uint32_t nU = 0, T = 0;
+        uint64_t U_off = 0;
+        if (ok && limit < (uint64_t)kHeaderBytes) ok = 0;
+        if (ok) {
+            ok = ld_le32(b) == kCosmoMagic && ld_le16(b + 4) == kVersion && ld_le16(b + kC) == 4 &&
+                 ld_le16(b + kD) == D && ld_le16(b + kH) == H && ld_le16(b + kW) == W;
+        }
+        if (ok) {
+            nU = ld_le32(b + kNU);
+            T = ld_le32(b + kNSlab);
+            U_off = ld_le64(b + kUOff);
+            const uint64_t slab_off = ld_le64(b + kSlabOff), total = ld_le64(b + kTotal);
+            ok = total <= limit && nU >= 1 && nU <= (uint32_t)kMaxU && T >= 1 && T <= (uint32_t)D &&
+                 U_off + 2ull * nU <= total && slab_off + (uint64_t)kSlabBytes * T <= total &&
+                 (slab_off & 15) == 0 && (U_off & 1) == 0;
+            const uint64_t plane = (uint64_t)H * W;
+            uint32_t zexp = 0;
+            for (uint32_t t = 0; ok && t < T; t++) {
+                const uint8_t *sl = b + slab_off + (uint64_t)kSlabBytes * t;
+                const uint32_t z0 = ld_le32(sl), z1 = ld_le32(sl + 4), G = ld_le32(sl + 8);
+                const int kw = sl[12];
+                const uint64_t lut_off = ld_le64(sl + 16), keys_off = ld_le64(sl + 24);
+                ok = z0 == zexp && z1 > z0 && z1 <= (uint32_t)D;
+                const uint64_t Nt = (uint64_t)(z1 - z0) * plane;
+                if (kw == 0) ok = ok && G == 1;
+                else if (kw == 1) ok = ok && G >= 1 && G <= (uint32_t)kMaxG1;
+                else if (kw == 2) ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
+                else if (kw == kRawSlab) ok = ok && G == 0;
+                else ok = 0;
+                if (kw != kRawSlab) ok = ok && (lut_off & 15) == 0 && lut_off + 8ull * G <= total;
+                if (kw != 0) ok = ok && (keys_off & 15) == 0 && keys_off + (uint64_t)(kw == kRawSlab ? 8 : kw) * Nt <= total;
+                zexp = z1;
+            }
+            ok = ok && zexp == (uint32_t)D;
+        }
+        if (!ok) report(status, SPP_ERR_CORRUPT, s);
+        sh_ok = ok;
+        sh_nU = nU;
+        sh_T = T;
+        sh_Uoff = U_off;
+        meta[s] = CosmoMeta{ok, nU, T, 0};
+    }
+    __syncthreads();
+    if (!sh_ok) return;
+    const uint8_t *U = b + sh_Uoff;
+    float *fU = fU_ws + (size_t)s * kFuStride;
+    for (uint32_t i = threadIdx.x; i < sh_nU; i += blockDim.x) {
+        const int c = (int16_t)ld_le16(U + 2 * i);
+        // fp64 log1p rounded once to fp32 (FORMAT.md 1.2, reading S2)
+        fU[i] = transform ? (float)log1p((double)c) : (float)c;
+    }
+}
+
+// --------------------------------------------------------------------------
+// KC: fused LUT expansion + transpose
+template <int OUT>
+struct Entry;
+template <>
+struct Entry<SPP_OUT_F16> { using T = uint2; };
+template <>
+struct Entry<SPP_OUT_I16> { using T = uint2; };
+template <>
+struct Entry<SPP_OUT_F32> { using T = uint4; };
+
+template <int OUT>
+__device__ __forceinline__ uint32_t cvt_lane(float f);
+template <>
+__device__ __forceinline__ uint32_t cvt_lane<SPP_OUT_F16>(float f) {
+    return (uint32_t)__half_as_ushort(__float2half_rn(f));
+}
+template <>
+__device__ __forceinline__ uint32_t cvt_lane<SPP_OUT_I16>(float f) {
+    return (uint32_t)(uint16_t)(int16_t)__float2int_rn(f);
+}
+
+// output 4-tuple for LUT entry `e` (four 16-bit U indices)
+template <int OUT>
+__device__ __forceinline__ typename Entry<OUT>::T make_entry(uint2 e, const float *__restrict__ fU, uint32_t nU,
+                                                             uint32_t *status, int s) {
+    uint32_t idx[4] = {e.x & 0xFFFFu, e.x >> 16, e.y & 0xFFFFu, e.y >> 16};
+    float f[4];
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+        if (idx[c] >= nU) {
+            report(status, SPP_ERR_CORRUPT, s);
+            idx[c] = 0;
+        }
+        f[c] = ld_ro_f32(fU + idx[c]);
+    }
+    if constexpr (OUT == SPP_OUT_F32) {
+        return make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]), __float_as_uint(f[3]));
+    } else {
+        return make_uint2(cvt_lane<OUT>(f[0]) | (cvt_lane<OUT>(f[1]) << 16),
+                          cvt_lane<OUT>(f[2]) | (cvt_lane<OUT>(f[3]) << 16));
+    }
+}
+
+struct SlabView {
+    uint32_t z0, z1, G;
+    int kw;
+    const uint8_t *lut;
+    const uint8_t *keys;
+};
+
+__device__ __forceinline__ SlabView read_slab(const uint8_t *b, int t) {
+    const uint8_t *sl = b + ld_le64(b + kSlabOff) + (uint64_t)kSlabBytes * t;
+    SlabView v;
+    v.z0 = ld_le32(sl);
+    v.z1 = ld_le32(sl + 4);
+    v.G = ld_le32(sl + 8);
+    v.kw = sl[12];
+    v.lut = b + ld_le64(sl + 16);
+    v.keys = b + ld_le64(sl + 24);
+    return v;
+}
+
+// store the 4 planes of 8 consecutive voxels (vector path)
+template <int OUT>
+__device__ __forceinline__ void store8(uint8_t *out_s, uint64_t N, uint64_t v, const typename Entry<OUT>::T *e) {
+    if constexpr (OUT == SPP_OUT_F32) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+            float f[8];
+#pragma unroll
+            for (int j = 0; j < 8; j++) f[j] = __uint_as_float(c == 0 ? e[j].x : c == 1 ? e[j].y : c == 2 ? e[j].z : e[j].w);
+            st_stream_f8(out_s + ((uint64_t)c * N + v) * 4, f);
+        }
+    } else {
+        // entry = (c0 | c1 << 16, c2 | c3 << 16): plane c takes 16-bit lane c of each entry
+        uint4 p0, p1, p2, p3;
+        p0.x = __byte_perm(e[0].x, e[1].x, 0x5410); p1.x = __byte_perm(e[0].x, e[1].x, 0x7632);
+        p2.x = __byte_perm(e[0].y, e[1].y, 0x5410); p3.x = __byte_perm(e[0].y, e[1].y, 0x7632);
+        p0.y = __byte_perm(e[2].x, e[3].x, 0x5410); p1.y = __byte_perm(e[2].x, e[3].x, 0x7632);
+        p2.y = __byte_perm(e[2].y, e[3].y, 0x5410); p3.y = __byte_perm(e[2].y, e[3].y, 0x7632);
+        p0.z = __byte_perm(e[4].x, e[5].x, 0x5410); p1.z = __byte_perm(e[4].x, e[5].x, 0x7632);
+        p2.z = __byte_perm(e[4].y, e[5].y, 0x5410); p3.z = __byte_perm(e[4].y, e[5].y, 0x7632);
+        p0.w = __byte_perm(e[6].x, e[7].x, 0x5410); p1.w = __byte_perm(e[6].x, e[7].x, 0x7632);
+        p2.w = __byte_perm(e[6].y, e[7].y, 0x5410); p3.w = __byte_perm(e[6].y, e[7].y, 0x7632);
+        st_stream_u4(out_s + (0 * N + v) * 2, p0);
+        st_stream_u4(out_s + (1 * N + v) * 2, p1);
+        st_stream_u4(out_s + (2 * N + v) * 2, p2);
+        st_stream_u4(out_s + (3 * N + v) * 2, p3);
+    }
+}
+
+template <int OUT>
+__device__ __forceinline__ void store1(uint8_t *out_s, uint64_t N, uint64_t v, typename Entry<OUT>::T e) {
+    if constexpr (OUT == SPP_OUT_F32) {
+        float *o = reinterpret_cast<float *>(out_s);
+        o[v] = __uint_as_float(e.x); o[N + v] = __uint_as_float(e.y);
+        o[2 * N + v] = __uint_as_float(e.z); o[3 * N + v] = __uint_as_float(e.w);
+    } else {
+        uint16_t *o = reinterpret_cast<uint16_t *>(out_s);
+        o[v] = (uint16_t)(e.x & 0xFFFF); o[N + v] = (uint16_t)(e.x >> 16);
+        o[2 * N + v] = (uint16_t)(e.y & 0xFFFF); o[3 * N + v] = (uint16_t)(e.y >> 16);
+    }
+}
+
+template <int OUT, int KW>
+__device__ __forceinline__ uint32_t key8(const uint8_t *keys, uint64_t rel, uint32_t (&g)[8]) {
+    if constexpr (KW == 2) {
+        uint4 k = ld_stream_u4(keys + 2 * rel);
+        g[0] = k.x & 0xFFFF; g[1] = k.x >> 16; g[2] = k.y & 0xFFFF; g[3] = k.y >> 16;
+        g[4] = k.z & 0xFFFF; g[5] = k.z >> 16; g[6] = k.w & 0xFFFF; g[7] = k.w >> 16;
+    } else {
+        uint2 k = ld_stream_u2(keys + rel);
+#pragma unroll
+        for (int j = 0; j < 4; j++) { g[j] = (k.x >> (8 * j)) & 0xFF; g[4 + j] = (k.y >> (8 * j)) & 0xFF; }
+    }
+    return 0;
+}
+
+// expansion of voxels [a, b) of one slab (relative voxel indices within the slab)
+template <int OUT, int KW>
+__device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
+                                                const typename Entry<OUT>::T *__restrict__ hot, uint32_t n_hot,
+                                                const float *__restrict__ fU, uint32_t nU, uint8_t *out_s,
+                                                uint64_t N, uint32_t *status, int s) {
+    using E = typename Entry<OUT>::T;
+    const uint64_t step = (uint64_t)blockDim.x * 8;
+    for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < b; q += 2 * step) {
+        uint32_t g0[8], g1[8];
+        const bool two = q + step < b;
+        key8<OUT, KW>(sv.keys, q, g0);
+        if (two) key8<OUT, KW>(sv.keys, q + step, g1);
+        E e[8];
+#pragma unroll
+        for (int j = 0; j < 8; j++) {
+            uint32_t g = g0[j];
+            if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
+            e[j] = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, nU, status, s);
+        }
+        store8<OUT>(out_s, N, slab_v0 + q, e);
+        if (two) {
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                uint32_t g = g1[j];
+                if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
+                e[j] = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, nU, status, s);
+            }
+            store8<OUT>(out_s, N, slab_v0 + q + step, e);
+        }
+    }
+}
+
+template <int OUT, bool VEC>
+__global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restrict__ src, int n,
+                                                      const float *__restrict__ fU_ws,
+                                                      const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
+                                                      int H, int W, uint64_t N, uint64_t chunk,
+                                                      uint32_t items_per_sample, uint32_t hot_cap,
+                                                      uint32_t *__restrict__ status) {
+    using E = typename Entry<OUT>::T;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    E *hot = reinterpret_cast<E *>(smem_raw);
+    const uint64_t plane = (uint64_t)H * W;
+    const uint64_t total_items = (uint64_t)n * items_per_sample;
+    const uint64_t per = (total_items + gridDim.x - 1) / gridDim.x;
+    const uint64_t i0 = (uint64_t)blockIdx.x * per;
+    const uint64_t i1 = min(total_items, i0 + per);
+    const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
+    int cached_s = -1, cached_t = -1;
+    uint32_t n_hot = 0;
+    for (uint64_t it = i0; it < i1; it++) {
+        const int s = (int)(it / items_per_sample);
+        const uint64_t v0 = (it % items_per_sample) * chunk;
+        const uint64_t v1 = min(N, v0 + chunk);
+        const CosmoMeta m = meta[s];
+        if (!m.valid) continue;
+        const uint8_t *b = static_cast<const uint8_t *>(src[s]);
+        const float *fU = fU_ws + (size_t)s * kFuStride;
+        uint8_t *out_s = dst + (uint64_t)s * 4 * N * ob;
+        for (uint32_t t = 0; t < m.nslab; t++) {
+            const SlabView sv = read_slab(b, t);
+            const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
+            const uint64_t a = max(v0, sa), e = min(v1, sb);
+            if (a >= e) continue;
+            if (sv.kw == 1 || sv.kw == 2) {
+                if (cached_s != s || cached_t != (int)t) {
+                    // stage the hottest groups (frequency-ordered keys) as output tuples
+                    __syncthreads();
+                    n_hot = min(sv.G, hot_cap);
+                    for (uint32_t g = threadIdx.x; g < n_hot; g += blockDim.x)
+                        hot[g] = make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, m.nU, status, s);
+                    __syncthreads();
+                    cached_s = s;
+                    cached_t = (int)t;
+                }
+                if constexpr (VEC) {
+                    if (sv.kw == 2)
+                        expand_keys_vec<OUT, 2>(sv, sa, a - sa, e - sa, hot, n_hot, fU, m.nU, out_s, N, status, s);
+                    else
+                        expand_keys_vec<OUT, 1>(sv, sa, a - sa, e - sa, hot, n_hot, fU, m.nU, out_s, N, status, s);
+                } else {
+                    for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
+                        const uint64_t rel = v - sa;
+                        uint32_t g = sv.kw == 2 ? ld_le16(sv.keys + 2 * rel) : sv.keys[rel];
+                        if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
+                        const E en = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, m.nU, status, s);
+                        store1<OUT>(out_s, N, v, en);
+                    }
+                }
+            } else if (sv.kw == 0) {
+                // broadcast of a constant 4-group
+                const E en = make_entry<OUT>(ld_ro_u2(sv.lut), fU, m.nU, status, s);
+                if constexpr (VEC) {
+                    E e8[8];
+#pragma unroll
+                    for (int j = 0; j < 8; j++) e8[j] = en;
+                    for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)blockDim.x * 8)
+                        store8<OUT>(out_s, N, q, e8);
+                } else {
+                    for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) store1<OUT>(out_s, N, v, en);
+                }
+            } else {
+                // RAW escape slab: four planes of U indices (FORMAT.md 1.1, kw = 8)
+                const uint64_t Nt = sb - sa;
+                for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
+                    const uint64_t rel = v - sa;
+                    uint2 ent;
+                    ent.x = (uint32_t)ld_le16(sv.keys + 2 * rel) | ((uint32_t)ld_le16(sv.keys + 2 * (Nt + rel)) << 16);
+                    ent.y = (uint32_t)ld_le16(sv.keys + 2 * (2 * Nt + rel)) |
+                            ((uint32_t)ld_le16(sv.keys + 2 * (3 * Nt + rel)) << 16);
+                    store1<OUT>(out_s, N, v, make_entry<OUT>(ent, fU, m.nU, status, s));
+                }
+            }
+        }
+    }
+}
+
+template <int OUT, bool VEC>
+spp_status launch_expand(const void *const *d_src, int n, const float *fU, const CosmoMeta *meta, uint8_t *dst,
+                         const spp_decode_opts &o, uint64_t N, cudaStream_t stream, const DeviceProps &dp) {
+    auto kern = kc_expand<OUT, VEC>;
+    const int entry_bytes = OUT == SPP_OUT_F32 ? 16 : 8;
+    const int smem = kHotBytes;
+    static int attr_done[8] = {0};  // per template instance (device-agnostic attribute)
+    const int key = (OUT - 1) * 2 + (VEC ? 1 : 0);
+    if (!attr_done[key]) {
+        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+            return SPP_ERR_CUDA;
+        attr_done[key] = 1;
+    }
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, smem) != cudaSuccess || occ < 1)
+        return SPP_ERR_CUDA;
+    const int ctas = dp.sms * occ;
+    // chunk: multiple of 2*8*kThreads voxels, at least ~8 items per CTA slot
+    uint64_t chunk = 4096;
+    const uint64_t want_items = (uint64_t)ctas * 8;
+    while (chunk < (1u << 18) && (uint64_t)n * ((N + chunk * 2 - 1) / (chunk * 2)) >= want_items) chunk *= 2;
+    if (!VEC) chunk = std::max<uint64_t>(1, std::min<uint64_t>(chunk, N));
+    const uint32_t ips = (uint32_t)((N + chunk - 1) / chunk);
+    const uint64_t items = (uint64_t)n * ips;
+    const int grid = (int)std::min<uint64_t>(items, (uint64_t)ctas);
+    kern<<<grid, kThreads, smem, stream>>>(d_src, n, fU, meta, dst, o.H, o.W, N, chunk, ips,
+                                           (uint32_t)(smem / entry_bytes), o.status);
+    return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
+}
+
+}  // namespace
+
+static spp_status cosmo_expand(const void *const *d_src, int n, void *d_dst, const spp_decode_opts &o,
+                               cudaStream_t stream, const DeviceProps &dp, float *fU, CosmoMeta *meta);
+
+size_t cosmo_workspace_bytes(int n) {
+    if (n <= 0) return 0;
+    return meta_offset(n) + round_up16((size_t)n * sizeof(CosmoMeta));
+}
+
+spp_status cosmo_decode(const void *const *d_src, int n, void *d_dst, const spp_decode_opts &o,
+                        cudaStream_t stream) {
+    DeviceProps dp;
+    spp_status st = current_device_props(&dp);
+    if (st != SPP_OK) return st;
+    uint8_t *ws = static_cast<uint8_t *>(o.workspace);
+    float *fU = reinterpret_cast<float *>(ws);
+    CosmoMeta *meta = reinterpret_cast<CosmoMeta *>(ws + meta_offset(n));
+    cudaEvent_t const *ev = reinterpret_cast<cudaEvent_t const *>(o.timing_events);
+    if (ev && cudaEventRecord(ev[0], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    kc0_prologue<<<n, kThreads, 0, stream>>>(d_src, o.src_bytes, o.transform, o.D, o.H, o.W, fU, meta, o.status);
+    if (cudaGetLastError() != cudaSuccess) return SPP_ERR_CUDA;
+    if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    spp_status r = cosmo_expand(d_src, n, d_dst, o, stream, dp, fU, meta);
+    if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    return r;
+}
+
+static spp_status cosmo_expand(const void *const *d_src, int n, void *d_dst, const spp_decode_opts &o,
+                               cudaStream_t stream, const DeviceProps &dp, float *fU, CosmoMeta *meta) {
+    const uint64_t N = (uint64_t)o.D * o.H * o.W;
+    const uint64_t plane = (uint64_t)o.H * o.W;
+    const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
+    const bool vec = plane % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
+    uint8_t *dst = static_cast<uint8_t *>(d_dst);
+    switch (o.out) {
+        case SPP_OUT_F16:
+            return vec ? launch_expand<SPP_OUT_F16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                       : launch_expand<SPP_OUT_F16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+        case SPP_OUT_F32:
+            return vec ? launch_expand<SPP_OUT_F32, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                       : launch_expand<SPP_OUT_F32, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+        case SPP_OUT_I16:
+            return vec ? launch_expand<SPP_OUT_I16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                       : launch_expand<SPP_OUT_I16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+        default:
+            return SPP_ERR_INVALID_ARG;
+    }
+}
+
+}  // namespace spp

@@ -1,0 +1,501 @@
+// deepcam.cu — DeepCAM decode + per-channel normalisation on sm_100a
+// (FORMAT.md 2.3).
+//
+// PAPER.md §V.A: lines along x are split into segments with a head
+// value and 8-bit minifloat differences relative to a per-segment minimum
+// exponent; abrupt lines are stored raw; constant runs are broadcast; per-line
+// metadata makes every line independently decodable.  §VI: the
+// loop-carried dependency is handled with hierarchical parallelism — here one
+// warp per line, lanes cooperating on the inner loop.
+//
+//   KD0  kd0_parse   one thread per sample: validate header, publish the line
+//                    directory / payload pointers.
+//   KD   kd_decode   persistent warps, each over a contiguous range of lines.
+//                    Lane 0 prefetches the directory two lines ahead and
+//                    issues a 1-D TMA bulk copy (cp.async.bulk + mbarrier) of
+//                    the next line into the warp's second smem buffer while
+//                    the warp decodes the current one (double buffering).
+//                    Decode of a SEG line:
+//                      1. warp scans of segment lengths / delta-byte counts ->
+//                         start bitmap + per-segment byte base (in place);
+//                      2. per 256-position chunk, lane l owns positions
+//                         [8l, 8l+8): 8 delta bytes -> 8 exact codes (as fp32
+//                         multiples of 2^-130: every partial sum is exact),
+//                         lane-serial prefix, warp segmented scan (reset at
+//                         segment heads) -> S_j, x̂ = fma(S_j, 2^emin, h)
+//                         (one rounding; FORMAT.md 2.3 reading S13);
+//                      3. y = (x̂ - shift) * scale (two roundings), RNE to fp16,
+//                         one 16-B streaming store per lane (512 B per warp).
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "spp_format.h"
+#include "spp_internal.h"
+
+namespace spp {
+namespace {
+
+using namespace spp::deepcam;
+
+struct DcMeta {  // written by KD0, read by KD (32 B)
+    const uint8_t *dir;
+    const uint8_t *payload;
+    uint64_t limit;  // bytes available from payload
+    uint32_t valid;
+    uint32_t pad;
+};
+
+constexpr int kMaxWarpsPerCta = 8;
+constexpr int kMaxW = 16383;  // GPU path: per-segment byte base packed in 16 bits
+
+__global__ void kd0_parse(const void *const *__restrict__ src, const uint64_t *__restrict__ src_bytes, int n, int C,
+                          int H, int W, DcMeta *__restrict__ meta, uint32_t *__restrict__ status) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    const uint8_t *b = static_cast<const uint8_t *>(src[s]);
+    const uint64_t limit = src_bytes ? src_bytes[s] : ~0ull;
+    bool ok = b != nullptr && (reinterpret_cast<uintptr_t>(b) & 15) == 0 && limit >= (uint64_t)kHeaderBytes;
+    DcMeta m{nullptr, nullptr, 0, 0, 0};
+    if (ok) {
+        const uint64_t L = (uint64_t)C * H;
+        ok = ld_le32(b) == kDeepcamMagic && ld_le16(b + 4) == kVersion && ld_le16(b + kC) == C &&
+             ld_le16(b + kH) == H && ld_le16(b + kW) == W && ld_le32(b + kL) == L;
+        const uint64_t dir_off = ld_le64(b + kDirOff), pay = ld_le64(b + kPayloadOff), total = ld_le64(b + kTotal);
+        ok = ok && total <= limit && (dir_off & 3) == 0 && dir_off + 4 * (L + 1) <= total && (pay & 15) == 0 &&
+             pay <= total;
+        if (ok) m = DcMeta{b + dir_off, b + pay, total - pay, 1u, 0u};
+    }
+    if (!ok) report(status, SPP_ERR_CORRUPT, s);
+    meta[s] = m;
+}
+
+// delta byte -> code value as an fp32 multiple of 2^-130 (exact; FORMAT.md 2.2):
+// sign bit -> bit 31, the 7 exponent|mantissa bits -> bits 19..25, so that
+// E = 0 lands on fp32 subnormals (M * 2^-130) and E >= 1 on (16+M) * 2^(E-131).
+template <int K>
+__device__ __forceinline__ float code_f(uint32_t w) {
+    uint32_t r;
+    if constexpr (K == 0) r = ((w << 24) & 0x80000000u) | ((w << 19) & 0x03F80000u);
+    else if constexpr (K == 1) r = ((w << 16) & 0x80000000u) | ((w << 11) & 0x03F80000u);
+    else if constexpr (K == 2) r = ((w << 8) & 0x80000000u) | ((w << 3) & 0x03F80000u);
+    else r = (w & 0x80000000u) | ((w >> 5) & 0x03F80000u);
+    return __uint_as_float(r);
+}
+__device__ __forceinline__ float code_f_byte(uint32_t b) {
+    return __uint_as_float(((b & 0x80u) << 24) | ((b & 0x7Fu) << 19));
+}
+
+// per-segment packed info written in place of the descriptor:
+//   bits 0..15  byte base a + 16384 (delta byte of position p is dl[a + p])
+//   bits 16..23 kind, bits 24..31 emin_b
+struct SegInfo {
+    float h;
+    float sc;      // 2^(emin+130) (emin <= -3) or 2^(emin+30) (big)
+    int a;
+    uint32_t kind;
+    uint32_t big;
+};
+__device__ __forceinline__ SegInfo seg_info(const uint32_t *desc, const float *heads, int s) {
+    const uint32_t d = desc[s];
+    SegInfo si;
+    si.h = heads[s];
+    si.a = (int)(d & 0xFFFFu) - 16384;
+    si.kind = (d >> 16) & 0xFFu;
+    const uint32_t eb = d >> 24;
+    si.big = eb >= 148u;
+    si.sc = __uint_as_float((si.big ? (eb + 7u) : (eb + 107u)) << 23);
+    return si;
+}
+
+template <int OUT>
+__device__ __forceinline__ void emit8(uint8_t *row, uint32_t p0, uint32_t W, const float (&y)[8]) {
+    if constexpr (OUT == SPP_OUT_F32) {
+        st_stream_f8(row + 4ull * p0, y);
+    } else {
+        uint4 u;
+        __half2 h0 = __floats2half2_rn(y[0], y[1]), h1 = __floats2half2_rn(y[2], y[3]);
+        __half2 h2 = __floats2half2_rn(y[4], y[5]), h3 = __floats2half2_rn(y[6], y[7]);
+        u.x = *reinterpret_cast<uint32_t *>(&h0);
+        u.y = *reinterpret_cast<uint32_t *>(&h1);
+        u.z = *reinterpret_cast<uint32_t *>(&h2);
+        u.w = *reinterpret_cast<uint32_t *>(&h3);
+        st_stream_u4(row + 2ull * p0, u);
+    }
+}
+template <int OUT>
+__device__ __forceinline__ void emit_scalar(uint8_t *row, uint32_t p0, uint32_t W, const float (&y)[8]) {
+#pragma unroll
+    for (int j = 0; j < 8; j++) {
+        if (p0 + j < W) {
+            if constexpr (OUT == SPP_OUT_F32) reinterpret_cast<float *>(row)[p0 + j] = y[j];
+            else reinterpret_cast<__half *>(row)[p0 + j] = __float2half_rn(y[j]);
+        }
+    }
+}
+
+// Decode one staged line (warp-cooperative).  Returns false if malformed.
+template <int OUT, bool VEC>
+__device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *sbits,
+                                            uint32_t nwords, float shv, float scv, uint8_t *row, int lane) {
+    const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
+    const uint32_t mode = hdr & 0xFFu;
+    if (mode == kModeRaw) {
+        if (16u + 4u * W > bytes) return false;
+        const float *x = reinterpret_cast<const float *>(buf + 16);
+        for (uint32_t c0 = 0; c0 < W; c0 += 256) {
+            const uint32_t p0 = c0 + 8 * lane;
+            if (p0 >= W) continue;
+            float y[8];
+            if constexpr (VEC) {
+                const float4 a = *reinterpret_cast<const float4 *>(x + p0);
+                const float4 b = *reinterpret_cast<const float4 *>(x + p0 + 4);
+                const float xv[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+#pragma unroll
+                for (int j = 0; j < 8; j++) y[j] = __fmul_rn(__fsub_rn(xv[j], shv), scv);
+                emit8<OUT>(row, p0, W, y);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 8; j++) y[j] = p0 + j < W ? __fmul_rn(__fsub_rn(x[p0 + j], shv), scv) : 0.f;
+                emit_scalar<OUT>(row, p0, W, y);
+            }
+        }
+        return true;
+    }
+    if (mode != kModeSeg) return false;
+    const uint32_t nseg = hdr >> 16;
+    if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;
+    uint32_t *desc = reinterpret_cast<uint32_t *>(buf + 4);
+    const float *heads = reinterpret_cast<const float *>(buf + 4 + 4 * nseg);
+    const uint8_t *dl = buf + 4 + 8 * nseg;
+
+    // 1. segment table: starts (bitmap), byte bases (in place), validation
+    for (uint32_t w = lane; w < nwords; w += kWarp) sbits[w] = 0;
+    __syncwarp();
+    uint32_t cl = 0, cd = 0;
+    bool bad = false;
+    for (uint32_t b0 = 0; b0 < nseg; b0 += kWarp) {
+        const uint32_t s = b0 + lane;
+        uint32_t len = 0, kind = 0, eb = 0;
+        if (s < nseg) {
+            const uint32_t d = desc[s];
+            len = d & 0xFFFFu;
+            kind = (d >> 16) & 0xFFu;
+            eb = d >> 24;
+        }
+        const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
+        const uint32_t il = warp_incl_scan(len, lane), id = warp_incl_scan(dlen, lane);
+        const uint32_t st = cl + il - len, db = cd + id - dlen;
+        if (s < nseg) {
+            bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
+                   st + len > W;
+            if (st < W) atomicOr(&sbits[st >> 5], 1u << (st & 31));
+            const int a = (int)db - (int)st - 1;
+            desc[s] = (uint32_t)(a + 16384) | (kind << 16) | (eb << 24);
+        }
+        cl += __shfl_sync(0xffffffffu, il, 31);
+        cd += __shfl_sync(0xffffffffu, id, 31);
+    }
+    bad = __any_sync(0xffffffffu, bad) || cl != W || 4u + 8u * nseg + cd > bytes;
+    if (bad) return false;
+    __syncwarp();
+
+    // 2. chunks of 256 positions, 8 per lane
+    float carry = 0.f;
+    uint32_t segc = 0;
+    for (uint32_t c0 = 0; c0 < W; c0 += 256) {
+        const uint32_t p0 = c0 + 8 * lane;
+        const bool act = p0 < W;
+        uint32_t sb = 0, valid = 0;
+        if (act) {
+            sb = (sbits[p0 >> 5] >> (p0 & 31)) & 0xFFu;
+            valid = W - p0 >= 8 ? 0xFFu : ((1u << (W - p0)) - 1u);
+            sb &= valid;
+        }
+        const uint32_t cnt = __popc(sb);
+        const uint32_t icnt = warp_incl_scan(cnt, lane);
+        const int s_prev = (int)(segc + icnt - cnt) - 1;
+        segc += __shfl_sync(0xffffffffu, icnt, 31);
+
+        float v[8], hj[8], scj[8];
+        uint32_t keep = 0, reset = 0, bigm = 0;
+        if ((sb >> 1) == 0) {
+            // fast path: all 8 positions in one segment (a head may sit at position 0)
+            const int s = act ? s_prev + (int)(sb & 1u) : 0;
+            const SegInfo si = seg_info(desc, heads, s);
+            float f[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+            if (act && si.kind == kDiff) {
+                const uint32_t addr = smem_u32(dl) + (uint32_t)(si.a + (int)p0);
+                const uint32_t al = addr & ~3u, shb = (addr & 3u) * 8u;
+                uint32_t w0, w1, w2;
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w0) : "r"(al));
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w1) : "r"(al + 4));
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w2) : "r"(al + 8));
+                uint32_t lo = __funnelshift_r(w0, w1, shb), hi = __funnelshift_r(w1, w2, shb);
+                if (sb & 1u) lo &= 0xFFFFFF00u;  // the head has no delta byte
+                if (valid != 0xFFu) {           // positions past the line end
+                    const uint64_t m = (1ull << (8 * __popc(valid))) - 1ull;
+                    lo &= (uint32_t)m;
+                    hi &= (uint32_t)(m >> 32);
+                }
+                f[0] = code_f<0>(lo); f[1] = code_f<1>(lo); f[2] = code_f<2>(lo); f[3] = code_f<3>(lo);
+                f[4] = code_f<0>(hi); f[5] = code_f<1>(hi); f[6] = code_f<2>(hi); f[7] = code_f<3>(hi);
+            }
+            v[0] = f[0];
+#pragma unroll
+            for (int j = 1; j < 8; j++) v[j] = v[j - 1] + f[j];
+#pragma unroll
+            for (int j = 0; j < 8; j++) { hj[j] = si.h; scj[j] = si.sc; }
+            keep = si.kind == kRepeat ? 0xFFu : (sb & 1u);
+            reset = (sb & 1u) ? 0xFFu : 0u;
+            bigm = si.big ? 0xFFu : 0u;
+        } else {
+            // general path: segment boundaries inside the lane's 8 positions
+            int s = s_prev;
+            SegInfo si = seg_info(desc, heads, s < 0 ? 0 : s);
+            float run = 0.f;
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                const uint32_t p = p0 + j;
+                if ((sb >> j) & 1u) {
+                    s++;
+                    si = seg_info(desc, heads, s);
+                    run = 0.f;
+                    reset |= 0xFFu << j;
+                    keep |= 1u << j;
+                } else if ((valid >> j) & 1u) {
+                    if (si.kind == kRepeat) keep |= 1u << j;
+                    else run += code_f_byte(dl[si.a + (int)p]);
+                }
+                v[j] = run;
+                hj[j] = si.h;
+                scj[j] = si.sc;
+                if (si.big) bigm |= 1u << j;
+            }
+        }
+        // warp segmented inclusive scan of the lane totals (reset at heads)
+        float x = v[7];
+        uint32_t fl = sb != 0;
+#pragma unroll
+        for (int d = 1; d < kWarp; d <<= 1) {
+            const float y = __shfl_up_sync(0xffffffffu, x, d);
+            const uint32_t fy = __shfl_up_sync(0xffffffffu, fl, d);
+            if (lane >= d) {
+                if (!fl) x += y;
+                fl |= fy;
+            }
+        }
+        const float xe = __shfl_up_sync(0xffffffffu, x, 1);
+        const uint32_t fe = __shfl_up_sync(0xffffffffu, fl, 1);
+        const float excl = lane == 0 ? carry : (fe ? xe : xe + carry);
+        const float xl = __shfl_sync(0xffffffffu, x, 31);
+        const uint32_t fll = __shfl_sync(0xffffffffu, fl, 31);
+        carry = fll ? xl : xl + carry;
+        if (!act) continue;
+        float y[8];
+#pragma unroll
+        for (int j = 0; j < 8; j++) {
+            float S = ((reset >> j) & 1u) ? v[j] : v[j] + excl;  // exact: multiples of 2^-130 below 2^-106
+            if ((bigm >> j) & 1u) S *= 0x1p100f;                  // keep the scale representable
+            const float xh = ((keep >> j) & 1u) ? hj[j] : __fmaf_rn(S, scj[j], hj[j]);
+            y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+        }
+        if constexpr (VEC) emit8<OUT>(row, p0, W, y);
+        else emit_scalar<OUT>(row, p0, W, y);
+    }
+    return true;
+}
+
+template <int OUT, bool VEC>
+__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
+    const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
+    const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
+    uint32_t *__restrict__ status) {
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int wpc = blockDim.x >> 5;
+    uint8_t *base = smem_raw + (size_t)warp * warp_bytes;
+    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + 2 * cap);
+    uint64_t *mbar = reinterpret_cast<uint64_t *>(base + 2 * cap + 4 * nwords);
+    const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
+    const uint32_t cap_data = cap - 16;       // one slot; the last 16 B are read slack
+    const uint32_t big_cap = 2 * cap - 16;    // both slots (any legal SEG line fits, FORMAT.md 2.1)
+
+    const uint64_t T = (uint64_t)n * L;
+    const uint64_t NW = (uint64_t)gridDim.x * wpc;
+    const uint64_t gw = (uint64_t)blockIdx.x * wpc + warp;
+    const uint64_t g_begin = gw * T / NW, g_end = (gw + 1) * T / NW;
+
+    if (lane == 0) {
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+
+    // lane-0 pipeline state: directory entries are loaded one line ahead of the
+    // line whose copy is being issued, so their latency hides behind a decode.
+    int64_t cs = -1;
+    DcMeta cm{nullptr, nullptr, 0, 0, 0};
+    uint32_t da = 0, db = 0;
+    const uint8_t *dpay = nullptr;
+    uint64_t dlim = 0;
+    uint32_t dvalid = 0;
+    int64_t dsample = 0;
+    auto load_dir = [&](uint64_t g) {
+        const int64_t s = (int64_t)(g / L);
+        const uint32_t l = (uint32_t)(g - (uint64_t)s * L);
+        if (s != cs) {
+            cm = meta[s];
+            cs = s;
+        }
+        dvalid = cm.valid;
+        dpay = cm.payload;
+        dlim = cm.limit;
+        dsample = s;
+        if (dvalid) {
+            const uint32_t *dir = reinterpret_cast<const uint32_t *>(cm.dir);
+            da = __ldg(dir + l);
+            db = __ldg(dir + l + 1);
+        }
+    };
+    // validate the loaded entry: bytes (0 = skip), big = needs both slots
+    auto prepare = [&](const uint8_t *&src, uint32_t &big) -> uint32_t {
+        big = 0;
+        if (!dvalid) return 0;
+        const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= dlim && db - da >= 16;
+        if (!ok) {
+            report(status, SPP_ERR_CORRUPT, dsample);
+            return 0;
+        }
+        const uint32_t bytes = db - da;
+        if (bytes > big_cap) {
+            report(status, SPP_ERR_UNSUPPORTED, dsample);
+            return 0;
+        }
+        big = bytes > cap_data;
+        src = dpay + da;
+        return bytes;
+    };
+    auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&mbar[slot], bytes);
+        bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
+    };
+
+    uint32_t cur_bytes = 0, cur_big = 0, phase0 = 0, phase1 = 0;
+    const uint8_t *cur_src = nullptr;
+    int slot = 0;
+    if (lane == 0 && g_begin < g_end) {
+        load_dir(g_begin);
+        cur_bytes = prepare(cur_src, cur_big);
+        if (cur_bytes && !cur_big) issue(0, cur_src, cur_bytes);
+        if (g_begin + 1 < g_end) load_dir(g_begin + 1);
+    }
+    for (uint64_t g = g_begin; g < g_end; g++) {
+        uint32_t nxt_bytes = 0, nxt_big = 0, nxt_issued = 0;
+        const uint8_t *nxt_src = nullptr;
+        if (lane == 0) {
+            if (g + 1 < g_end) {
+                nxt_bytes = prepare(nxt_src, nxt_big);
+                // an oversize current line occupies both slots: issue the next later
+                if (nxt_bytes && !nxt_big && !cur_big) {
+                    issue(slot ^ 1, nxt_src, nxt_bytes);
+                    nxt_issued = 1;
+                }
+            }
+            if (g + 2 < g_end) load_dir(g + 2);
+        }
+        const uint32_t bytes = __shfl_sync(0xffffffffu, cur_bytes, 0);
+        const uint32_t big = __shfl_sync(0xffffffffu, cur_big, 0);
+        if (bytes) {
+            uint8_t *buf = base + slot * cap;
+            if (big) {
+                // stage across both slots with plain 16-B loads (rare: SEG line larger than RAW)
+                const uint64_t sp = __shfl_sync(0xffffffffu, reinterpret_cast<uint64_t>(cur_src), 0);
+                const uint4 *src4 = reinterpret_cast<const uint4 *>(sp);
+                for (uint32_t k = lane; k < bytes / 16; k += kWarp) reinterpret_cast<uint4 *>(base)[k] = src4[k];
+                __syncwarp();
+                buf = base;
+            } else if (slot == 0) {
+                mbar_wait(&mbar[0], phase0);
+                phase0 ^= 1;
+            } else {
+                mbar_wait(&mbar[1], phase1);
+                phase1 ^= 1;
+            }
+            const uint32_t l = (uint32_t)(g % L);
+            const uint32_t c = l / H;
+            const float shv = shift ? __ldg(shift + c) : 0.f;
+            const float scv = scale ? __ldg(scale + c) : 1.f;
+            uint8_t *row = dst + g * (uint64_t)W * ob;
+            const bool ok = decode_line<OUT, VEC>(buf, bytes, W, sbits, nwords, shv, scv, row, lane);
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
+        }
+        __syncwarp();
+        if (lane == 0 && nxt_bytes && !nxt_big && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
+        slot ^= 1;
+        cur_bytes = nxt_bytes;
+        cur_big = nxt_big;
+        cur_src = nxt_src;
+    }
+}
+
+template <int OUT, bool VEC>
+spp_status launch_kd(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
+                     const DeviceProps &dp) {
+    const uint32_t W = (uint32_t)o.W;
+    const uint32_t cap = (uint32_t)round_up16(16 + 4ull * W) + 16;
+    const uint32_t nwords = (((W + 31) / 32 + 1) + 3) & ~3u;
+    const uint32_t warp_bytes = 2 * cap + 4 * nwords + 16;
+    int wpc = kMaxWarpsPerCta;
+    while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
+    if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
+    const int smem = wpc * (int)warp_bytes;
+    auto kern = kd_decode<OUT, VEC>;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+        return SPP_ERR_CUDA;
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, wpc * kWarp, smem) != cudaSuccess || occ < 1)
+        return SPP_ERR_CUDA;
+    const uint64_t lines = (uint64_t)n * o.C * o.H;
+    const uint64_t max_ctas = (uint64_t)dp.sms * occ;
+    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
+    kern<<<grid, wpc * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift, o.scale,
+                                               static_cast<uint8_t *>(d_dst), cap, nwords, warp_bytes, o.status);
+    return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
+}
+
+}  // namespace
+
+size_t deepcam_workspace_bytes(int n) { return n <= 0 ? 0 : round_up16((size_t)n * sizeof(DcMeta)); }
+
+spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const spp_decode_opts &o,
+                          cudaStream_t stream) {
+    if (o.W > kMaxW) return SPP_ERR_UNSUPPORTED;
+    DeviceProps dp;
+    spp_status st = current_device_props(&dp);
+    if (st != SPP_OK) return st;
+    DcMeta *meta = static_cast<DcMeta *>(o.workspace);
+    cudaEvent_t const *ev = reinterpret_cast<cudaEvent_t const *>(o.timing_events);
+    if (ev && cudaEventRecord(ev[0], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    kd0_parse<<<(n + 127) / 128, 128, 0, stream>>>(d_src, o.src_bytes, n, o.C, o.H, o.W, meta, o.status);
+    if (cudaGetLastError() != cudaSuccess) return SPP_ERR_CUDA;
+    if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
+    const bool vec = o.W % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
+    spp_status r = SPP_ERR_INVALID_ARG;
+    if (o.out == SPP_OUT_F32)
+        r = vec ? launch_kd<SPP_OUT_F32, true>(meta, n, d_dst, o, stream, dp)
+                : launch_kd<SPP_OUT_F32, false>(meta, n, d_dst, o, stream, dp);
+    else if (o.out == SPP_OUT_F16)
+        r = vec ? launch_kd<SPP_OUT_F16, true>(meta, n, d_dst, o, stream, dp)
+                : launch_kd<SPP_OUT_F16, false>(meta, n, d_dst, o, stream, dp);
+    if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;
+    return r;
+}
+
+}  // namespace spp

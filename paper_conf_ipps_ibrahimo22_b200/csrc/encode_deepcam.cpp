@@ -1,0 +1,198 @@
+// encode_deepcam.cpp — host DeepCAM differential line encoder (step b.1,
+// PAPER.md P:32), FORMAT.md 2.4.
+//
+// PAPER.md §V.A (Fig. 4): each line along x is split into
+// segments; a segment has a pivot/head value and 8-bit differences (1 sign, 3
+// exponent bits relative to the segment's minimum exponent, 4 mantissa bits).
+// Lines with abrupt transitions or too many segments stay uncompressed (RAW);
+// runs of identical values use a special encoding (REPEAT); the encoder picks
+// whichever is smaller ("best space-saving").  Closed-loop: each difference is
+// taken against the value the decoder will reconstruct, so errors do not
+// accumulate along the line.
+#include <math.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <vector>
+
+#include "spp.h"
+#include "spp_format.h"
+
+namespace {
+
+using namespace spp::deepcam;
+using spp::round_up16;
+
+// magnitude of the 7-bit exponent|mantissa field (FORMAT.md 2.2), ascending in b
+struct CodeTable {
+    int mag[128];
+    CodeTable() {
+        for (int b = 0; b < 128; b++) {
+            int E = b >> 4, M = b & 15;
+            mag[b] = E == 0 ? M : (16 + M) << (E - 1);
+        }
+    }
+    // byte whose value is nearest to t; ties toward the smaller magnitude
+    inline int quantise(double t, int *value) const {
+        double a = fabs(t);
+        int lo = 0, hi = 127;  // largest b with mag[b] <= a
+        while (lo < hi) {
+            int mid = (lo + hi + 1) >> 1;
+            if (mag[mid] <= a) lo = mid; else hi = mid - 1;
+        }
+        int b = lo;
+        if (b < 127 && (mag[b + 1] - a) < (a - mag[b])) b++;
+        if (mag[b] == 0) { *value = 0; return 0; }
+        *value = t < 0 ? -mag[b] : mag[b];
+        return t < 0 ? (b | 0x80) : b;
+    }
+};
+const CodeTable kCodes;
+
+inline uint32_t fbits(float f) { uint32_t u; memcpy(&u, &f, 4); return u; }
+
+// exact ceil(log2(q)), q > 0
+inline int ceil_log2(double q) {
+    int e;
+    double f = frexp(q, &e);
+    return f == 0.5 ? e - 1 : e;
+}
+
+struct Seg { uint16_t len; uint8_t kind, emin_b; float head; };
+
+struct LineEncoder {
+    int W;
+    std::vector<int> run;
+    std::vector<Seg> segs;
+    std::vector<uint8_t> deltas;
+    explicit LineEncoder(int w) : W(w), run(w), segs(), deltas() { segs.reserve(w); deltas.reserve(w); }
+
+    // returns the SEG payload size; fills segs/deltas
+    uint64_t encode(const float *x) {
+        segs.clear();
+        deltas.clear();
+        run[W - 1] = 1;
+        for (int i = W - 2; i >= 0; i--) run[i] = fbits(x[i]) == fbits(x[i + 1]) ? run[i + 1] + 1 : 1;
+        int i = 0;
+        while (i < W) {
+            if (run[i] >= kRepeatMin) {
+                segs.push_back(Seg{(uint16_t)run[i], kRepeat, 0, x[i]});
+                i += run[i];
+                continue;
+            }
+            const float h = x[i];
+            double m = 0.0;
+            const int jend = (i + kLookahead < W) ? i + kLookahead : W;
+            for (int j = i + 1; j < jend; j++) {
+                double d = fabs((double)x[j] - (double)x[j - 1]);
+                if (d > m) m = d;
+            }
+            int emin = -149;
+            if (m > 0.0) {
+                emin = ceil_log2(m / (double)kMaxCode);
+                emin = emin < -149 ? -149 : (emin > 96 ? 96 : emin);
+            }
+            const float unit = ldexpf(1.0f, emin);
+            int64_t S = 0;
+            float prev = h;
+            int j = i + 1;
+            for (; j < W; j++) {
+                if (run[j] >= kRepeatMin) break;
+                double t = ldexp((double)x[j] - (double)prev, -emin);
+                if (fabs(t) > kMaxCode + 0.5) break;
+                int k;
+                int b = kCodes.quantise(t, &k);
+                if (llabs(S + k) > kMaxAbsS) break;
+                S += k;
+                prev = h + (float)S * unit;                // decoder's x̂_j (fp32, one rounding)
+                deltas.push_back((uint8_t)b);
+            }
+            segs.push_back(Seg{(uint16_t)(j - i), kDiff, (uint8_t)(emin + kEminBias), h});
+            i = j;
+        }
+        return round_up16(4 + 8 * (uint64_t)segs.size() + deltas.size());
+    }
+};
+
+inline bool all_finite(const float *x, int W) {
+    for (int k = 0; k < W; k++)
+        if (!isfinite(x[k])) return false;
+    return true;
+}
+
+}  // namespace
+
+extern "C" size_t spp_deepcam_max_encoded_size(int C, int H, int W) {
+    if (C < 1 || H < 1 || W < 1) return 0;
+    uint64_t L = (uint64_t)C * H;
+    return (size_t)(spp::kHeaderBytes + round_up16(4 * (L + 1)) + L * round_up16(16 + 4 * (uint64_t)W));
+}
+
+extern "C" spp_status spp_encode_deepcam(const float *x, int C, int H, int W, void *dst,
+                                         size_t dst_capacity, size_t *encoded_size) {
+    if (!x || !encoded_size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535)
+        return SPP_ERR_INVALID_ARG;
+    const uint64_t L = (uint64_t)C * H;
+    const uint64_t dir_off = spp::kHeaderBytes;
+    const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
+    const uint64_t raw_size = round_up16(16 + 4 * (uint64_t)W);
+    LineEncoder enc(W);
+    // pass 1: per-line size (SEG vs RAW)
+    std::vector<uint8_t> is_seg(L);
+    std::vector<uint32_t> dir(L + 1);
+    uint64_t cur = 0;
+    for (uint64_t l = 0; l < L; l++) {
+        const float *xl = x + l * (uint64_t)W;
+        uint64_t sz = raw_size;
+        is_seg[l] = 0;
+        if (all_finite(xl, W)) {
+            uint64_t seg = enc.encode(xl);
+            if (seg < raw_size) { sz = seg; is_seg[l] = 1; }
+        }
+        if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;
+        dir[l] = (uint32_t)cur;
+        cur += sz;
+    }
+    if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;
+    dir[L] = (uint32_t)cur;
+    const uint64_t total = payload_off + cur;
+    *encoded_size = (size_t)total;
+    if (!dst || dst_capacity < total) return SPP_ERR_BUFFER_TOO_SMALL;
+    uint8_t *out = (uint8_t *)dst;
+    memset(out, 0, (size_t)total);
+    uint32_t u32;
+    uint16_t u16;
+    u32 = spp::kDeepcamMagic; memcpy(out, &u32, 4);
+    u16 = spp::kVersion; memcpy(out + 4, &u16, 2);
+    u16 = (uint16_t)C; memcpy(out + kC, &u16, 2);
+    u16 = (uint16_t)H; memcpy(out + kH, &u16, 2);
+    u16 = (uint16_t)W; memcpy(out + kW, &u16, 2);
+    u32 = (uint32_t)L; memcpy(out + kL, &u32, 4);
+    memcpy(out + kDirOff, &dir_off, 8);
+    memcpy(out + kPayloadOff, &payload_off, 8);
+    memcpy(out + kTotal, &total, 8);
+    memcpy(out + dir_off, dir.data(), 4 * (L + 1));
+    // pass 2: payloads
+    for (uint64_t l = 0; l < L; l++) {
+        const float *xl = x + l * (uint64_t)W;
+        uint8_t *p = out + payload_off + dir[l];
+        if (!is_seg[l]) {
+            p[0] = kModeRaw;
+            memcpy(p + 16, xl, 4 * (size_t)W);
+            continue;
+        }
+        enc.encode(xl);
+        const uint16_t nseg = (uint16_t)enc.segs.size();
+        p[0] = kModeSeg;
+        memcpy(p + 2, &nseg, 2);
+        for (int s = 0; s < nseg; s++) {
+            const Seg &g = enc.segs[s];
+            memcpy(p + 4 + 4 * s, &g.len, 2);
+            p[4 + 4 * s + 2] = g.kind;
+            p[4 + 4 * s + 3] = g.emin_b;
+            memcpy(p + 4 + 4 * (size_t)nseg + 4 * s, &g.head, 4);
+        }
+        memcpy(p + 4 + 8 * (size_t)nseg, enc.deltas.data(), enc.deltas.size());
+    }
+    return SPP_OK;
+}

@@ -1,0 +1,191 @@
+"""ctypes binding of libspp (include/spp.h) — argument marshalling only.
+
+Every step of the hot path runs in libspp's sm_100a kernels; PyTorch supplies
+device memory, streams and process groups.  There is no CPU fallback: if
+``libspp.so`` is missing or the device is not an sm_100 GPU, calls raise.
+Function names mirror the C ABI.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from pathlib import Path
+from typing import Sequence
+
+import numpy as np
+
+_PKG = Path(__file__).resolve().parent
+LIB_PATH = _PKG / "libspp.so"
+
+SPP_OK, SPP_ERR_INVALID_ARG, SPP_ERR_BUFFER_TOO_SMALL, SPP_ERR_CORRUPT, SPP_ERR_UNSUPPORTED, SPP_ERR_CUDA = range(6)
+SPP_FMT_COSMO, SPP_FMT_DEEPCAM = 1, 2
+SPP_OUT_F16, SPP_OUT_F32, SPP_OUT_I16 = 1, 2, 3
+FMT = {"cosmo": SPP_FMT_COSMO, "deepcam": SPP_FMT_DEEPCAM}
+OUT = {"f16": SPP_OUT_F16, "f32": SPP_OUT_F32, "i16": SPP_OUT_I16}
+
+# every symbol include/spp.h declares (checked by tests/test_host.py)
+EXPORTS = (
+    "spp_cosmo_max_encoded_size", "spp_encode_cosmo", "spp_deepcam_max_encoded_size", "spp_encode_deepcam",
+    "spp_stream_info", "spp_decode_opts_init", "spp_decode_workspace_size", "spp_decoded_sample_bytes",
+    "spp_decode_batch", "spp_decode_launches", "spp_pipeline_create", "spp_pipeline_destroy", "spp_decode_host",
+    "spp_pipeline_last_launches", "spp_status_string", "spp_version",
+)
+
+
+class SppError(RuntimeError):
+    def __init__(self, code: int, what: str):
+        super().__init__(f"{what}: {spp_status_string(code)} ({code})")
+        self.code = code
+
+
+class spp_decode_opts(C.Structure):
+    _fields_ = [("out", C.c_int), ("transform", C.c_int), ("shift", C.c_void_p), ("scale", C.c_void_p),
+                ("status", C.c_void_p), ("src_bytes", C.c_void_p), ("workspace", C.c_void_p),
+                ("workspace_size", C.c_size_t), ("C", C.c_int), ("D", C.c_int), ("H", C.c_int), ("W", C.c_int),
+                ("timing_events", C.c_void_p)]
+
+
+_lib = None
+
+
+def load() -> C.CDLL:
+    """Load the in-tree libspp.so (built by __graft_entry__.build()); fail loudly."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not LIB_PATH.exists():
+        raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                          "(there is no CPU fallback)")
+    L = C.CDLL(str(LIB_PATH))
+    P, I, SZ, I64 = C.c_void_p, C.c_int, C.c_size_t, C.c_int64
+    sig = {
+        "spp_cosmo_max_encoded_size": ([I, I, I, I], SZ),
+        "spp_encode_cosmo": ([P, I, I, I, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_deepcam_max_encoded_size": ([I, I, I], SZ),
+        "spp_encode_deepcam": ([P, I, I, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_stream_info": ([I, P, SZ, C.POINTER(I64)], I),
+        "spp_decode_opts_init": ([C.POINTER(spp_decode_opts), I, I, I, I, I], None),
+        "spp_decode_workspace_size": ([I, I, C.POINTER(spp_decode_opts)], SZ),
+        "spp_decoded_sample_bytes": ([I, C.POINTER(spp_decode_opts)], SZ),
+        "spp_decode_batch": ([I, P, I, P, C.POINTER(spp_decode_opts), P], I),
+        "spp_decode_launches": ([I], I),
+        "spp_pipeline_create": ([C.POINTER(P), I, C.POINTER(spp_decode_opts), SZ, I, I], I),
+        "spp_pipeline_destroy": ([P], None),
+        "spp_decode_host": ([P, P, P, I, P, C.POINTER(spp_decode_opts), P], I),
+        "spp_pipeline_last_launches": ([P], I),
+        "spp_status_string": ([I], C.c_char_p),
+        "spp_version": ([], C.c_char_p),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+    _lib = L
+    return L
+
+
+def _check(rc: int, what: str):
+    if rc != SPP_OK:
+        raise SppError(rc, what)
+
+
+def spp_status_string(code: int) -> str:
+    return load().spp_status_string(int(code)).decode()
+
+
+def spp_version() -> str:
+    return load().spp_version().decode()
+
+
+# ---------------------------------------------------------------- host encoders
+def spp_cosmo_max_encoded_size(Cc: int, D: int, H: int, W: int) -> int:
+    return int(load().spp_cosmo_max_encoded_size(Cc, D, H, W))
+
+
+def spp_encode_cosmo(counts: np.ndarray) -> np.ndarray:
+    """int16 [4, D, H, W] counts -> encoded uint8 stream (FORMAT.md 1)."""
+    a = np.ascontiguousarray(counts, dtype=np.int16)
+    if a.ndim != 4:
+        raise ValueError("counts must be [4, D, H, W]")
+    Cc, D, H, W = a.shape
+    cap = spp_cosmo_max_encoded_size(Cc, D, H, W)
+    dst = np.empty(max(cap, 64), dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(load().spp_encode_cosmo(a.ctypes.data, Cc, D, H, W, dst.ctypes.data, dst.size, C.byref(size)),
+           "spp_encode_cosmo")
+    return dst[: size.value].copy()
+
+
+def spp_deepcam_max_encoded_size(Cc: int, H: int, W: int) -> int:
+    return int(load().spp_deepcam_max_encoded_size(Cc, H, W))
+
+
+def spp_encode_deepcam(x: np.ndarray) -> np.ndarray:
+    """fp32 [C, H, W] -> encoded uint8 stream (FORMAT.md 2)."""
+    a = np.ascontiguousarray(x, dtype=np.float32)
+    if a.ndim != 3:
+        raise ValueError("x must be [C, H, W]")
+    Cc, H, W = a.shape
+    cap = spp_deepcam_max_encoded_size(Cc, H, W)
+    dst = np.empty(max(cap, 64), dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(load().spp_encode_deepcam(a.ctypes.data, Cc, H, W, dst.ctypes.data, dst.size, C.byref(size)),
+           "spp_encode_deepcam")
+    return dst[: size.value].copy()
+
+
+def spp_stream_info(fmt: str, buf: np.ndarray):
+    b = np.ascontiguousarray(buf, dtype=np.uint8)
+    info = (C.c_int64 * 4)()
+    _check(load().spp_stream_info(FMT[fmt], b.ctypes.data, b.size, info), "spp_stream_info")
+    return tuple(int(v) for v in info)
+
+
+# ---------------------------------------------------------------- device decode
+def spp_decode_opts_init(fmt: str, Cc: int, D: int, H: int, W: int, out: str = "f16",
+                         transform: int | None = None) -> spp_decode_opts:
+    o = spp_decode_opts()
+    load().spp_decode_opts_init(C.byref(o), FMT[fmt], Cc, D, H, W)
+    o.out = OUT[out]
+    if transform is not None:
+        o.transform = int(transform)
+    return o
+
+
+def spp_decode_workspace_size(fmt: str, n: int, opts: spp_decode_opts) -> int:
+    return int(load().spp_decode_workspace_size(FMT[fmt], n, C.byref(opts)))
+
+
+def spp_decoded_sample_bytes(fmt: str, opts: spp_decode_opts) -> int:
+    return int(load().spp_decoded_sample_bytes(FMT[fmt], C.byref(opts)))
+
+
+def spp_decode_launches(fmt: str) -> int:
+    return int(load().spp_decode_launches(FMT[fmt]))
+
+
+def spp_decode_batch(fmt: str, d_src_ptrs: int, n: int, d_dst: int, opts: spp_decode_opts, stream: int = 0):
+    """Raw call: d_src_ptrs = device address of n device pointers; d_dst = device address."""
+    _check(load().spp_decode_batch(FMT[fmt], d_src_ptrs, n, d_dst, C.byref(opts), stream), "spp_decode_batch")
+
+
+def spp_pipeline_create(fmt: str, opts: spp_decode_opts, slot_bytes: int, nslots: int, max_chunk: int) -> int:
+    h = C.c_void_p()
+    _check(load().spp_pipeline_create(C.byref(h), FMT[fmt], C.byref(opts), slot_bytes, nslots, max_chunk),
+           "spp_pipeline_create")
+    return h.value
+
+
+def spp_pipeline_destroy(handle: int):
+    load().spp_pipeline_destroy(handle)
+
+
+def spp_decode_host(handle: int, h_ptrs: Sequence[int], sizes: Sequence[int], d_dst: int, opts: spp_decode_opts,
+                    stream: int = 0):
+    n = len(h_ptrs)
+    ptrs = (C.c_void_p * n)(*h_ptrs)
+    sz = (C.c_size_t * n)(*sizes)
+    _check(load().spp_decode_host(handle, ptrs, sz, n, d_dst, C.byref(opts), stream), "spp_decode_host")
+
+
+def spp_pipeline_last_launches(handle: int) -> int:
+    return int(load().spp_pipeline_last_launches(handle))

@@ -1,0 +1,318 @@
+"""GPU parity: libspp's sm_100a kernels vs the CPU oracle, element by element.
+
+Tolerances (BASELINE.json north_star): decoded integer data bit-exact; fp32
+within 2 ulp; fp16 within 1 ulp.  By construction (readings S2, S13,
+S18) the expected difference is 0 ulp, so these tests demand bit equality
+(NaN positions must match; NaN payloads are not compared).
+"""
+import numpy as np
+import pytest
+
+from tests import fmt
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_ibrahimo22_b200 import build
+    build.build()
+    return torch.device("cuda:0")
+
+
+def _to_dev(buf: np.ndarray):
+    t = torch.empty(int(buf.size) + 15, dtype=torch.uint8, device="cuda")
+    t = t[: buf.size]  # torch allocations are 512-B aligned; slicing from 0 keeps alignment
+    t.copy_(torch.from_numpy(np.ascontiguousarray(buf)))
+    return t
+
+
+def _same_bits(got: np.ndarray, want: np.ndarray):
+    assert got.shape == want.shape and got.dtype == want.dtype
+    if got.dtype.kind == "f":
+        gn, wn = np.isnan(got), np.isnan(want)
+        assert np.array_equal(gn, wn)
+        iv = got.view(np.uint16 if got.itemsize == 2 else np.uint32)
+        jv = want.view(np.uint16 if got.itemsize == 2 else np.uint32)
+        bad = (iv != jv) & ~gn
+        assert not bad.any(), f"{int(bad.sum())} mismatches, first at {np.argwhere(bad)[:3].tolist()}"
+    else:
+        assert np.array_equal(got, want)
+
+
+def _decode(fmt_name, bufs, dims, out="f16", transform=None, shift=None, scale=None):
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder
+    dec = Decoder(fmt_name, dims, out=out, transform=transform)
+    if shift is not None or scale is not None:
+        dec.set_normalisation(shift, scale)
+    srcs = [_to_dev(b) for b in bufs]
+    res = dec.decode(srcs)
+    torch.cuda.synchronize()
+    status = int(dec.status.item())
+    return res.cpu().numpy(), status
+
+
+# ------------------------------------------------------------------ CosmoFlow
+def test_cosmo_c1_paper_sample_all_outputs(dev, orc):
+    """C1: one paper-shaped 4x128^3 sample; fp16 / fp32 / identity int16."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_cosmo(1001)
+    b = spp.spp_encode_cosmo(x)
+    for out, tr in (("f16", 1), ("f32", 1), ("i16", 0), ("f32", 0), ("f16", 0)):
+        got, st = _decode("cosmo", [b], x.shape, out=out, transform=tr)
+        assert st == 0
+        _same_bits(got[0], orc.cosmo_direct(x, tr, out))
+
+
+def test_cosmo_transform_table_exhaustive(dev, orc):
+    """Every count 0..32767 through the GPU's fp64 log1p -> fp32 (and fp16)."""
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    vals = np.arange(32768, dtype=np.int16)
+    x = np.stack([vals, vals[::-1], np.roll(vals, 7), vals]).reshape(4, 32, 32, 32).copy()
+    b = spp.spp_encode_cosmo(x)
+    for out in ("f32", "f16"):
+        got, st = _decode("cosmo", [b], x.shape, out=out)
+        assert st == 0
+        _same_bits(got[0], orc.cosmo_direct(x, 1, out))
+
+
+@pytest.mark.parametrize("preset,n", [("sparse", 64), ("verysparse", 64), ("dense", 64), ("unit", 48),
+                                      ("independent", 32), ("coupled", 40)])
+def test_cosmo_presets_key_widths_and_slabs(dev, orc, preset, n):
+    """C5 sweep shapes: kw = 1 / 2, z-slab split and the RAW escape."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_cosmo(3001, preset, n=n)
+    b = spp.spp_encode_cosmo(x)
+    got, st = _decode("cosmo", [b], x.shape, out="f16")
+    assert st == 0
+    _same_bits(got[0], orc.cosmo_direct(x, 1, "f16"))
+
+
+def test_cosmo_edge_shapes_and_broadcast(dev, orc):
+    """Degenerate cases: all-zero volume (kw = 0 broadcast), 1-voxel volume,
+    odd shapes (scalar path), a slab split on a tiny volume."""
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(3)
+    cases = [np.zeros((4, 16, 16, 16), dtype=np.int16), np.full((4, 1, 1, 1), 5, dtype=np.int16),
+             rng.integers(0, 30, size=(4, 5, 7, 3)).astype(np.int16),
+             rng.integers(0, 4, size=(4, 3, 3, 3)).astype(np.int16),
+             rng.integers(0, 2000, size=(4, 4, 64, 64)).astype(np.int16)]   # G > 0.75 N -> RAW escape
+    for x in cases:
+        b = spp.spp_encode_cosmo(x)
+        for out in ("f32", "f16"):
+            got, st = _decode("cosmo", [b], x.shape, out=out)
+            assert st == 0
+            _same_bits(got[0], orc.cosmo_direct(x, 1, out))
+        got, st = _decode("cosmo", [b], x.shape, out="i16", transform=0)
+        assert st == 0 and np.array_equal(got[0], x)
+
+
+def test_cosmo_oracle_encoded_stream(dev, orc):
+    """The GPU decodes a stream written by the oracle's own encoder."""
+    from synth import gen_cosmo
+    x = gen_cosmo(1002, n=64)
+    b = orc.cosmo_encode(x)
+    got, st = _decode("cosmo", [b], x.shape, out="f32")
+    assert st == 0
+    _same_bits(got[0], orc.cosmo_decode(b, x.shape, 1, "f32"))
+
+
+def test_cosmo_c2_launch_configuration(dev, orc):
+    """C2 at full size (n = 512, the bench's launch configuration): every
+    output sample equals the oracle's plain definition of its source."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, spp
+    pool = [gen_cosmo(1001 + i) for i in range(3)]
+    bufs = [_to_dev(spp.spp_encode_cosmo(x)) for x in pool]
+    want = [torch.from_numpy(orc.cosmo_direct(x, 1, "f16").view(np.int16)).to(dev) for x in pool]
+    n = 512
+    dec = Decoder("cosmo", (4, 128, 128, 128))
+    out = dec.decode([bufs[i % 3] for i in range(n)])
+    torch.cuda.synchronize()
+    assert int(dec.status.item()) == 0
+    o16 = out.view(torch.int16)
+    for i in range(n):
+        assert torch.equal(o16[i], want[i % 3]), i
+
+
+def test_cosmo_corruption_detected(dev):
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_cosmo(1005, n=32)
+    b = spp.spp_encode_cosmo(x)
+    h = fmt.cosmo_header(b)
+    bad_magic = b.copy(); bad_magic[0] ^= 0xFF
+    bad_key = b.copy()
+    s0 = h["slabs"][0]
+    if s0["kw"] == 2:
+        bad_key[s0["keys_off"]:s0["keys_off"] + 2] = 0xFF   # key 65535 >= G
+    bad_lut = b.copy(); bad_lut[s0["lut_off"]:s0["lut_off"] + 2] = 0xFF  # U index >= nU
+    for i, bb in enumerate((bad_magic, bad_key, bad_lut)):
+        _, st = _decode("cosmo", [b, bb], x.shape, out="f16")
+        assert st & 0xFF == 3 and st >> 8 == 1, (i, st)
+
+
+# ------------------------------------------------------------------ DeepCAM
+def _dc_ref(orc, b, shape, shift, scale, out):
+    return orc.deepcam_decode(b, shape, shift, scale, out)
+
+
+def test_deepcam_c3_paper_sample(dev, orc):
+    """C3: one 16x768x1152 sample, per-channel normalisation, fp16 and fp32."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2001)
+    mean, rstd = deepcam_stats(x)
+    b = spp.spp_encode_deepcam(x)
+    for out in ("f16", "f32"):
+        got, st = _decode("deepcam", [b], x.shape, out=out, shift=mean, scale=rstd)
+        assert st == 0
+        _same_bits(got[0], _dc_ref(orc, b, x.shape, mean, rstd, out))
+    got, st = _decode("deepcam", [b], x.shape, out="f32")     # x-hat itself
+    assert st == 0
+    _same_bits(got[0], _dc_ref(orc, b, x.shape, None, None, "f32"))
+
+
+def test_deepcam_oracle_encoded_stream(dev, orc):
+    from synth import gen_deepcam
+    x = gen_deepcam(2002, H=64)
+    b = orc.deepcam_encode(x)
+    got, st = _decode("deepcam", [b], x.shape, out="f32")
+    assert st == 0
+    _same_bits(got[0], _dc_ref(orc, b, x.shape, None, None, "f32"))
+
+
+def _random_line(rng, W, kinds=(0, 1), seglen=(1, 40)):
+    segs, deltas, pos = [], [], 0
+    while pos < W:
+        ln = int(min(W - pos, rng.integers(*seglen)))
+        kind = int(rng.choice(kinds))
+        eb = int(rng.choice([1, 2, 60, 120, 140, 147, 148, 149, 170, 246]))
+        h = np.float32(rng.choice([0.0, -0.0, 1.0, rng.standard_normal() * 10.0 ** rng.integers(-40, 30),
+                                   2.0 ** -140]))
+        segs.append((ln, kind, eb, h))
+        if kind == 1:
+            deltas += [int(v) for v in rng.integers(0, 256, size=ln - 1)]
+        pos += ln
+    return fmt.build_seg_line(W, segs, deltas)
+
+
+@pytest.mark.parametrize("W", [1, 7, 8, 17, 64, 256, 264, 1152])
+def test_deepcam_handbuilt_lines(dev, orc, W):
+    """Hand-built SEG/RAW lines: short segments (several per lane: general
+    path), REPEAT of -0.0, subnormal and large-exponent scales, heads at every
+    lane offset, NaN/Inf RAW lines, W not a multiple of 8 (scalar path)."""
+    rng = np.random.default_rng(W)
+    C, H = 2, 24
+    lines = []
+    for l in range(C * H):
+        r = l % 6
+        if r == 0:
+            v = rng.standard_normal(W).astype(np.float32)
+            v[rng.integers(0, W)] = np.nan
+            v[rng.integers(0, W)] = -np.inf
+            lines.append(fmt.build_raw_line(v))
+        elif r == 1:
+            lines.append(fmt.build_seg_line(W, [(W, 0, 0, np.float32(-0.0))], []))
+        elif r == 2:
+            lines.append(_random_line(rng, W, seglen=(1, 4)))
+        elif r == 3:
+            lines.append(_random_line(rng, W, kinds=(1,), seglen=(W, W + 1)))
+        else:
+            lines.append(_random_line(rng, W))
+    b = fmt.build_deepcam_stream(C, H, W, lines)
+    shift = np.float32([0.5, -3.0])
+    scale = np.float32([2.0, 1e-3])
+    for out in ("f32", "f16"):
+        got, st = _decode("deepcam", [b], (C, H, W), out=out, shift=shift, scale=scale)
+        assert st == 0
+        _same_bits(got[0], _dc_ref(orc, b, (C, H, W), shift, scale, out))
+    got, st = _decode("deepcam", [b], (C, H, W), out="f32")
+    _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, "f32"))
+
+
+def test_deepcam_batch_order_independence(dev, orc):
+    """P13: decoding samples alone, in a batch, or in another order gives the
+    same bytes per sample."""
+    from synth import gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    xs = [gen_deepcam(2010 + i, H=96) for i in range(3)]
+    bs = [spp.spp_encode_deepcam(x) for x in xs]
+    batch, st = _decode("deepcam", bs, xs[0].shape, out="f16")
+    assert st == 0
+    rev, _ = _decode("deepcam", bs[::-1], xs[0].shape, out="f16")
+    for i in range(3):
+        alone, _ = _decode("deepcam", [bs[i]], xs[0].shape, out="f16")
+        assert np.array_equal(alone[0].view(np.uint16), batch[i].view(np.uint16))
+        assert np.array_equal(rev[2 - i].view(np.uint16), batch[i].view(np.uint16))
+        _same_bits(batch[i], _dc_ref(orc, bs[i], xs[0].shape, None, None, "f16"))
+
+
+def test_deepcam_c4_launch_configuration(dev, orc):
+    """C4 at full size (n = 2048 samples -> fp16, the bench's launch
+    configuration): every output sample equals the oracle decode of its
+    source."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, spp
+    pool = [gen_deepcam(2001 + i) for i in range(2)]
+    mean, rstd = deepcam_stats(pool[0])
+    bufs = [_to_dev(spp.spp_encode_deepcam(x)) for x in pool]
+    want = [torch.from_numpy(orc.deepcam_decode(spp.spp_encode_deepcam(x), x.shape, mean, rstd, "f16")
+                             .view(np.int16)).to(dev) for x in pool]
+    n = 2048
+    dec = Decoder("deepcam", (16, 768, 1152))
+    dec.set_normalisation(mean, rstd)
+    out = dec.decode([bufs[i % 2] for i in range(n)])
+    torch.cuda.synchronize()
+    assert int(dec.status.item()) == 0
+    o16 = out.view(torch.int16)
+    for i in range(n):
+        assert torch.equal(o16[i], want[i % 2]), i
+    del out, o16
+
+
+def test_deepcam_corruption_detected(dev):
+    W = 64
+    good = fmt.build_seg_line(W, [(W, 1, 140, 1.0)], [1] * (W - 1))
+    bad_sum = fmt.build_seg_line(W, [(W - 1, 1, 140, 1.0)], [1] * (W - 2))
+    bad_kind = fmt.build_seg_line(W, [(W, 5, 140, 1.0)], [1] * (W - 1))
+    for bad in (bad_sum, bad_kind):
+        b = fmt.build_deepcam_stream(1, 2, W, [good, bad])
+        _, st = _decode("deepcam", [b, b], (1, 2, W), out="f16")
+        assert st & 0xFF == 3
+    b = fmt.build_deepcam_stream(1, 2, W, [good, good])
+    c = b.copy(); c[0] = 0
+    _, st = _decode("deepcam", [b, c], (1, 2, W), out="f16")
+    assert st == (3 | (1 << 8))
+
+
+# ------------------------------------------------------------------ streamed (b.4 + b.5)
+@pytest.mark.parametrize("fmt_name", ["cosmo", "deepcam"])
+def test_host_pipeline_matches_device_decode(dev, fmt_name):
+    from synth import gen_cosmo, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, HostPipeline, spp
+    if fmt_name == "cosmo":
+        xs = [gen_cosmo(1001 + i, n=64) for i in range(5)]
+        bs = [spp.spp_encode_cosmo(x) for x in xs]
+    else:
+        xs = [gen_deepcam(2001 + i, H=64) for i in range(5)]
+        bs = [spp.spp_encode_deepcam(x) for x in xs]
+    dims = xs[0].shape
+    host = [torch.from_numpy(b).pin_memory() for b in bs] * 3
+    dec = Decoder(fmt_name, dims)
+    ref = dec.decode([_to_dev(b) for b in bs])
+    pipe = HostPipeline(dec, slot_bytes=2 * max(b.size for b in bs) + 64, nslots=3, max_chunk=2)
+    out = dec.alloc_out(len(host))
+    pipe.decode(host, out)
+    torch.cuda.synchronize()
+    assert int(dec.status.item()) == 0
+    for i in range(len(host)):
+        assert torch.equal(out[i].view(torch.int16), ref[i % 5].view(torch.int16))
+    assert pipe.launches() == 2 * ((len(host) + 1) // 2)
+    pipe.close()

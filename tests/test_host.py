@@ -1,0 +1,125 @@
+"""Host-side tests of the product library (no GPU): the C ABI loads and exports
+every symbol include/spp.h declares, the host encoders, argument validation
+and the host-side stream parser.  The CUDA kernels are exercised only in the
+-m gpu suite."""
+import ctypes
+import re
+from pathlib import Path
+
+import numpy as np
+import pytest
+
+from tests import fmt
+
+ROOT = Path(__file__).resolve().parent.parent
+
+
+@pytest.fixture(scope="module")
+def spp():
+    from paper_conf_ipps_ibrahimo22_b200 import build, spp as s
+    build.build()
+    s.load()
+    return s
+
+
+def test_header_symbols_exported(spp):
+    header = (ROOT / "include" / "spp.h").read_text()
+    declared = set(re.findall(r"\b(spp_[a-z0-9_]+)\s*\(", header))
+    declared -= {"spp_status", "spp_format", "spp_out"}
+    lib = ctypes.CDLL(str(spp.LIB_PATH))
+    missing = [name for name in sorted(declared) if not hasattr(lib, name)]
+    assert missing == []
+    assert declared == set(spp.EXPORTS)
+    assert spp.spp_version().endswith("sm_100a")
+
+
+def test_library_is_sm100a_only(spp):
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", str(spp.LIB_PATH)],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out and "sm_90" not in out and "sm_80" not in out
+
+
+def test_cosmo_encoder_matches_oracle_bytes(spp, orc):
+    from synth import gen_cosmo
+    rng = np.random.default_rng(2)
+    vols = [gen_cosmo(1001), gen_cosmo(3001, "verysparse", n=32), gen_cosmo(3002, "dense", n=64),
+            np.zeros((4, 3, 5, 7), dtype=np.int16), rng.integers(0, 9, size=(4, 2, 3, 5)).astype(np.int16)]
+    for x in vols:
+        a = spp.spp_encode_cosmo(x)
+        b = orc.cosmo_encode(x)
+        assert a.size == b.size and np.array_equal(a, b)
+        assert np.array_equal(orc.cosmo_decode(a, x.shape, 0, "i16"), x)
+
+
+def test_deepcam_encoder_matches_oracle_bytes(spp, orc):
+    from synth import gen_deepcam
+    rng = np.random.default_rng(4)
+    xs = [gen_deepcam(2001, H=48), rng.standard_normal((2, 3, 37)).astype(np.float32),
+          np.full((1, 2, 40), -0.0, dtype=np.float32)]
+    x = rng.standard_normal((1, 4, 64)).astype(np.float32)
+    x[0, 1, 5] = np.nan
+    x[0, 2, :] = np.float32(1e-40) * np.arange(64, dtype=np.float32)  # subnormal ramp
+    xs.append(x)
+    for x in xs:
+        a = spp.spp_encode_deepcam(x)
+        b = orc.deepcam_encode(x)
+        assert a.size == b.size and np.array_equal(a, b)
+
+
+def test_encoder_argument_errors(spp):
+    with pytest.raises(spp.SppError) as e:
+        spp.spp_encode_cosmo(-np.ones((4, 2, 2, 2), dtype=np.int16))
+    assert e.value.code == spp.SPP_ERR_INVALID_ARG
+    with pytest.raises(spp.SppError):
+        spp.spp_encode_cosmo(np.zeros((3, 2, 2, 2), dtype=np.int16))      # C must be 4
+    lib = spp.load()
+    size = ctypes.c_size_t(0)
+    x = np.zeros((4, 4, 4, 4), dtype=np.int16)
+    rc = lib.spp_encode_cosmo(x.ctypes.data, 4, 4, 4, 4, None, 0, ctypes.byref(size))
+    assert rc == spp.SPP_ERR_BUFFER_TOO_SMALL and size.value > 0 and size.value % 16 == 0
+
+
+def test_stream_info(spp):
+    from synth import gen_cosmo
+    x = gen_cosmo(1001)
+    nU, T, G, kw = spp.spp_stream_info("cosmo", spp.spp_encode_cosmo(x))
+    assert nU == len(np.unique(x)) and T == 1 and kw == 2
+    v = x.reshape(4, -1).astype(np.int64)
+    assert G == len(np.unique((v[0] << 48) | (v[1] << 32) | (v[2] << 16) | v[3]))
+    y = np.zeros((1, 2, 32), dtype=np.float32)
+    y[0, 1] = np.inf
+    raw, seg, segs, dbytes = spp.spp_stream_info("deepcam", spp.spp_encode_deepcam(y))
+    assert (raw, seg, segs, dbytes) == (1, 1, 1, 0)
+
+
+def test_decode_argument_validation_without_gpu(spp):
+    """Host-checkable argument errors return before any CUDA call."""
+    lib = spp.load()
+    o = spp.spp_decode_opts_init("cosmo", 4, 8, 8, 8)
+    assert lib.spp_decode_batch(1, None, -1, None, ctypes.byref(o), None) == spp.SPP_ERR_INVALID_ARG
+    assert lib.spp_decode_batch(7, None, 1, None, ctypes.byref(o), None) == spp.SPP_ERR_INVALID_ARG
+    assert lib.spp_decode_batch(1, None, 0, None, ctypes.byref(o), None) == spp.SPP_OK   # empty batch
+    o.out = spp.SPP_OUT_I16                                                            # i16 needs transform 0
+    assert lib.spp_decode_batch(1, 16, 1, 256, ctypes.byref(o), None) == spp.SPP_ERR_INVALID_ARG
+    bad = spp.spp_decode_opts_init("cosmo", 3, 8, 8, 8)
+    assert lib.spp_decode_batch(1, 16, 1, 256, ctypes.byref(bad), None) == spp.SPP_ERR_INVALID_ARG
+    o = spp.spp_decode_opts_init("deepcam", 16, 1, 768, 1152)
+    assert lib.spp_decode_batch(2, 16, 1, 256, ctypes.byref(o), None) == spp.SPP_ERR_BUFFER_TOO_SMALL  # no ws
+    assert spp.spp_decode_workspace_size("deepcam", 4, o) > 0
+    assert spp.spp_decoded_sample_bytes("deepcam", o) == 16 * 768 * 1152 * 2
+    assert spp.spp_decode_launches("cosmo") == 2 and spp.spp_decode_launches("deepcam") == 2
+
+
+def test_deepcam_encoder_bound_on_product_streams(spp, orc):
+    """The product encoder's streams decode (oracle) within the per-value bound."""
+    from tests.test_oracle_pins import _check_bound
+    rng = np.random.default_rng(8)
+    x = np.cumsum(rng.standard_normal((1, 4, 200)) * 0.05, axis=2).astype(np.float32)
+    b = spp.spp_encode_deepcam(x)
+    h = fmt.deepcam_header(b)
+    for l in range(4):
+        info = fmt.deepcam_line(b, h, l)
+        xh = orc.deepcam_decode_line(b, l, 200)
+        if info["mode"] == 1:
+            _check_bound(x[0, l], xh, info["segs"])
