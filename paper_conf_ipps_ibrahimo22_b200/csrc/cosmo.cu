@@ -47,7 +47,8 @@ struct CosmoMeta {  // written by KC0, read by KC
 
 constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 constexpr int kThreads = 256;
-constexpr int kHotBytes = 64 * 1024;  // shared-memory hot prefix of T per CTA
+constexpr int kHotBytes = 48 * 1024;  // shared-memory hot prefix of T per CTA
+constexpr int kUCap = 4096;           // unique values staged in shared memory (16 KB)
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
 
@@ -60,7 +61,7 @@ __global__ void __launch_bounds__(kThreads) kc0_prologue(const void *const *__re
                                                          uint32_t *__restrict__ status) {
     const int s = blockIdx.x;
     const uint8_t *b = static_cast<const uint8_t *>(src[s]);
-    __shared__ uint32_t sh_ok, sh_nU, sh_T;
+    __shared__ uint32_t sh_ok, sh_nU;
     __shared__ uint64_t sh_Uoff;
     if (threadIdx.x == 0) {
         uint32_t ok = b != nullptr && (reinterpret_cast<uintptr_t>(b) & 15) == 0;
@@ -103,7 +104,6 @@ __global__ void __launch_bounds__(kThreads) kc0_prologue(const void *const *__re
         if (!ok) report(status, SPP_ERR_CORRUPT, s);
         sh_ok = ok;
         sh_nU = nU;
-        sh_T = T;
         sh_Uoff = U_off;
         meta[s] = CosmoMeta{ok, nU, T, 0};
     }
@@ -140,26 +140,50 @@ __device__ __forceinline__ uint32_t cvt_lane<SPP_OUT_I16>(float f) {
     return (uint32_t)(uint16_t)(int16_t)__float2int_rn(f);
 }
 
-// output 4-tuple for LUT entry `e` (four 16-bit U indices)
 template <int OUT>
-__device__ __forceinline__ typename Entry<OUT>::T make_entry(uint2 e, const float *__restrict__ fU, uint32_t nU,
-                                                             uint32_t *status, int s) {
-    uint32_t idx[4] = {e.x & 0xFFFFu, e.x >> 16, e.y & 0xFFFFu, e.y >> 16};
-    float f[4];
-#pragma unroll
-    for (int c = 0; c < 4; c++) {
-        if (idx[c] >= nU) {
-            report(status, SPP_ERR_CORRUPT, s);
-            idx[c] = 0;
-        }
-        f[c] = ld_ro_f32(fU + idx[c]);
-    }
+__device__ __forceinline__ typename Entry<OUT>::T pack_entry(const float (&f)[4]) {
     if constexpr (OUT == SPP_OUT_F32) {
         return make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]), __float_as_uint(f[3]));
     } else {
         return make_uint2(cvt_lane<OUT>(f[0]) | (cvt_lane<OUT>(f[1]) << 16),
                           cvt_lane<OUT>(f[2]) | (cvt_lane<OUT>(f[3]) << 16));
     }
+}
+
+// Where f(U) lives for the current sample: shared memory (|U| <= kUCap, the
+// normal case: hundreds of values) or the global workspace.
+struct FuView {
+    uint32_t smem;        // shared address of fU_s
+    const float *global;  // workspace copy
+    uint32_t nU;
+    bool in_smem;
+};
+
+// output 4-tuple of LUT entry `e` (four 16-bit U indices); an index >= nU
+// (corrupt stream) is clamped and flagged in `bad` (reported once per item)
+template <int OUT, bool SMEM>
+__device__ __forceinline__ typename Entry<OUT>::T make_entry(uint2 e, const FuView &fu, uint32_t &bad) {
+    uint32_t idx[4] = {e.x & 0xFFFFu, e.x >> 16, e.y & 0xFFFFu, e.y >> 16};
+    float f[4];
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+        bad |= idx[c] >= fu.nU;
+        const uint32_t i = min(idx[c], fu.nU - 1);
+        if constexpr (SMEM) f[c] = lds_f32(fu.smem + 4 * i);
+        else f[c] = ld_ro_f32(fu.global + i);
+    }
+    return pack_entry<OUT>(f);
+}
+
+template <int OUT>
+__device__ __forceinline__ typename Entry<OUT>::T lds_entry(uint32_t addr) {
+    if constexpr (OUT == SPP_OUT_F32) return lds_u4(addr);
+    else return lds_u2(addr);
+}
+template <int OUT>
+__device__ __forceinline__ void sts_entry(uint32_t addr, typename Entry<OUT>::T v) {
+    if constexpr (OUT == SPP_OUT_F32) sts_u4(addr, v);
+    else sts_u2(addr, v);
 }
 
 struct SlabView {
@@ -181,9 +205,10 @@ __device__ __forceinline__ SlabView read_slab(const uint8_t *b, int t) {
     return v;
 }
 
-// store the 4 planes of 8 consecutive voxels (vector path)
+// store the 4 planes of 8 consecutive voxels (vector path): plane c of voxel v
+// is out_s[(c*N + v)]; one 16-B (fp16/int16) or 32-B (fp32) store per plane
 template <int OUT>
-__device__ __forceinline__ void store8(uint8_t *out_s, uint64_t N, uint64_t v, const typename Entry<OUT>::T *e) {
+__device__ __forceinline__ void store8(uint8_t *out_s, uint64_t N, uint64_t v, const typename Entry<OUT>::T (&e)[8]) {
     if constexpr (OUT == SPP_OUT_F32) {
 #pragma unroll
         for (int c = 0; c < 4; c++) {
@@ -203,10 +228,11 @@ __device__ __forceinline__ void store8(uint8_t *out_s, uint64_t N, uint64_t v, c
         p2.z = __byte_perm(e[4].y, e[5].y, 0x5410); p3.z = __byte_perm(e[4].y, e[5].y, 0x7632);
         p0.w = __byte_perm(e[6].x, e[7].x, 0x5410); p1.w = __byte_perm(e[6].x, e[7].x, 0x7632);
         p2.w = __byte_perm(e[6].y, e[7].y, 0x5410); p3.w = __byte_perm(e[6].y, e[7].y, 0x7632);
-        st_stream_u4(out_s + (0 * N + v) * 2, p0);
-        st_stream_u4(out_s + (1 * N + v) * 2, p1);
-        st_stream_u4(out_s + (2 * N + v) * 2, p2);
-        st_stream_u4(out_s + (3 * N + v) * 2, p3);
+        uint8_t *o = out_s + v * 2;
+        st_stream_u4(o, p0);
+        st_stream_u4(o + N * 2, p1);
+        st_stream_u4(o + N * 4, p2);
+        st_stream_u4(o + N * 6, p3);
     }
 }
 
@@ -223,63 +249,88 @@ __device__ __forceinline__ void store1(uint8_t *out_s, uint64_t N, uint64_t v, t
     }
 }
 
-template <int OUT, int KW>
-__device__ __forceinline__ uint32_t key8(const uint8_t *keys, uint64_t rel, uint32_t (&g)[8]) {
-    if constexpr (KW == 2) {
-        uint4 k = ld_stream_u4(keys + 2 * rel);
-        g[0] = k.x & 0xFFFF; g[1] = k.x >> 16; g[2] = k.y & 0xFFFF; g[3] = k.y >> 16;
-        g[4] = k.z & 0xFFFF; g[5] = k.z >> 16; g[6] = k.w & 0xFFFF; g[7] = k.w >> 16;
-    } else {
-        uint2 k = ld_stream_u2(keys + rel);
-#pragma unroll
-        for (int j = 0; j < 4; j++) { g[j] = (k.x >> (8 * j)) & 0xFF; g[4 + j] = (k.y >> (8 * j)) & 0xFF; }
+template <int KW>
+struct KeyVec;
+template <>
+struct KeyVec<2> {
+    uint4 v;
+    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel) { v = ld_stream_u4(keys + 2 * rel); }
+    __device__ __forceinline__ uint32_t get(int j) const {
+        const uint32_t w = j < 2 ? v.x : j < 4 ? v.y : j < 6 ? v.z : v.w;
+        return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
     }
-    return 0;
+};
+template <>
+struct KeyVec<1> {
+    uint2 v;
+    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel) { v = ld_stream_u2(keys + rel); }
+    __device__ __forceinline__ uint32_t get(int j) const { return ((j < 4 ? v.x : v.y) >> (8 * (j & 3))) & 0xFFu; }
+};
+
+// 8 consecutive voxels: hot tuples from smem; the rare cold keys (beyond the
+// staged prefix) are fetched together in one warp-uniform branch
+template <int OUT, int KW>
+__device__ __forceinline__ void expand8(const KeyVec<KW> &k, const SlabView &sv, uint32_t hot_base, uint32_t n_hot,
+                                        const FuView &fu, uint8_t *out_s, uint64_t N, uint64_t v0, uint32_t &bad) {
+    using E = typename Entry<OUT>::T;
+    constexpr uint32_t EB = sizeof(E);
+    uint32_t g[8];
+    E e[8];
+    uint32_t cold = 0;
+#pragma unroll
+    for (int j = 0; j < 8; j++) {
+        uint32_t gj = k.get(j);
+        bad |= gj >= sv.G;
+        gj = gj < sv.G ? gj : 0u;
+        g[j] = gj;
+        if (gj < n_hot) e[j] = lds_entry<OUT>(hot_base + gj * EB);
+        else cold |= 1u << j;
+    }
+    if (__any_sync(0xffffffffu, cold != 0)) {
+        uint2 lv[8];
+#pragma unroll
+        for (int j = 0; j < 8; j++)
+            if ((cold >> j) & 1u) lv[j] = ld_ro_u2(sv.lut + 8ull * g[j]);
+#pragma unroll
+        for (int j = 0; j < 8; j++)
+            if ((cold >> j) & 1u) e[j] = make_entry<OUT, true>(lv[j], fu, bad);
+    }
+    store8<OUT>(out_s, N, v0, e);
 }
 
-// expansion of voxels [a, b) of one slab (relative voxel indices within the slab)
+// voxels [a, b) of one slab (relative indices), 8 per thread per group; the
+// keys of the next two groups are in flight while a group is expanded
 template <int OUT, int KW>
 __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
-                                                const typename Entry<OUT>::T *__restrict__ hot, uint32_t n_hot,
-                                                const float *__restrict__ fU, uint32_t nU, uint8_t *out_s,
-                                                uint64_t N, uint32_t *status, int s) {
-    using E = typename Entry<OUT>::T;
+                                                uint32_t hot_base, uint32_t n_hot, const FuView &fu, uint8_t *out_s,
+                                                uint64_t N, uint32_t &bad) {
     const uint64_t step = (uint64_t)blockDim.x * 8;
-    for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < b; q += 2 * step) {
-        uint32_t g0[8], g1[8];
-        const bool two = q + step < b;
-        key8<OUT, KW>(sv.keys, q, g0);
-        if (two) key8<OUT, KW>(sv.keys, q + step, g1);
-        E e[8];
-#pragma unroll
-        for (int j = 0; j < 8; j++) {
-            uint32_t g = g0[j];
-            if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
-            e[j] = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, nU, status, s);
-        }
-        store8<OUT>(out_s, N, slab_v0 + q, e);
-        if (two) {
-#pragma unroll
-            for (int j = 0; j < 8; j++) {
-                uint32_t g = g1[j];
-                if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
-                e[j] = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, nU, status, s);
-            }
-            store8<OUT>(out_s, N, slab_v0 + q + step, e);
-        }
+    uint64_t q = a + (uint64_t)threadIdx.x * 8;
+    KeyVec<KW> k0, k1;
+    if (q < b) k0.load(sv.keys, q);
+    if (q + step < b) k1.load(sv.keys, q + step);
+#pragma unroll 1
+    for (; q < b; q += step) {
+        KeyVec<KW> k2;
+        if (q + 2 * step < b) k2.load(sv.keys, q + 2 * step);
+        expand8<OUT, KW>(k0, sv, hot_base, n_hot, fu, out_s, N, slab_v0 + q, bad);
+        k0 = k1;
+        k1 = k2;
     }
 }
 
 template <int OUT, bool VEC>
-__global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restrict__ src, int n,
-                                                      const float *__restrict__ fU_ws,
-                                                      const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
-                                                      int H, int W, uint64_t N, uint64_t chunk,
-                                                      uint32_t items_per_sample, uint32_t hot_cap,
-                                                      uint32_t *__restrict__ status) {
+__global__ void __launch_bounds__(kThreads, 2) kc_expand(const void *const *__restrict__ src, int n,
+                                                         const float *__restrict__ fU_ws,
+                                                         const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
+                                                         int H, int W, uint64_t N, uint64_t chunk,
+                                                         uint32_t items_per_sample, uint32_t hot_cap,
+                                                         uint32_t *__restrict__ status) {
     using E = typename Entry<OUT>::T;
+    constexpr uint32_t EB = sizeof(E);
     extern __shared__ __align__(16) uint8_t smem_raw[];
-    E *hot = reinterpret_cast<E *>(smem_raw);
+    const uint32_t hot_base = smem_u32(smem_raw);
+    const uint32_t fu_base = hot_base + kHotBytes;
     const uint64_t plane = (uint64_t)H * W;
     const uint64_t total_items = (uint64_t)n * items_per_sample;
     const uint64_t per = (total_items + gridDim.x - 1) / gridDim.x;
@@ -288,6 +339,7 @@ __global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restr
     const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
     int cached_s = -1, cached_t = -1;
     uint32_t n_hot = 0;
+#pragma unroll 1
     for (uint64_t it = i0; it < i1; it++) {
         const int s = (int)(it / items_per_sample);
         const uint64_t v0 = (it % items_per_sample) * chunk;
@@ -295,8 +347,11 @@ __global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restr
         const CosmoMeta m = meta[s];
         if (!m.valid) continue;
         const uint8_t *b = static_cast<const uint8_t *>(src[s]);
-        const float *fU = fU_ws + (size_t)s * kFuStride;
+        const FuView fu{fu_base, fU_ws + (size_t)s * kFuStride, m.nU, m.nU <= (uint32_t)kUCap};
+        const FuView fu_g{fu_base, fu.global, m.nU, false};
         uint8_t *out_s = dst + (uint64_t)s * 4 * N * ob;
+        uint32_t bad = 0;  // corrupt key / index seen by this thread in this item
+#pragma unroll 1
         for (uint32_t t = 0; t < m.nslab; t++) {
             const SlabView sv = read_slab(b, t);
             const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
@@ -304,32 +359,51 @@ __global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restr
             if (a >= e) continue;
             if (sv.kw == 1 || sv.kw == 2) {
                 if (cached_s != s || cached_t != (int)t) {
-                    // stage the hottest groups (frequency-ordered keys) as output tuples
+                    // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples
+                    __syncthreads();
+                    if (cached_s != s && fu.in_smem)
+                        for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
                     __syncthreads();
                     n_hot = min(sv.G, hot_cap);
-                    for (uint32_t g = threadIdx.x; g < n_hot; g += blockDim.x)
-                        hot[g] = make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, m.nU, status, s);
+#pragma unroll 1
+                    for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * blockDim.x) {
+                        uint2 lv[4];
+#pragma unroll
+                        for (int u = 0; u < 4; u++) {
+                            const uint32_t g = g0 + u * blockDim.x;
+                            if (g < n_hot) lv[u] = ld_ro_u2(sv.lut + 8ull * g);
+                        }
+#pragma unroll
+                        for (int u = 0; u < 4; u++) {
+                            const uint32_t g = g0 + u * blockDim.x;
+                            if (g < n_hot)
+                                sts_entry<OUT>(hot_base + g * EB, fu.in_smem ? make_entry<OUT, true>(lv[u], fu, bad)
+                                                                             : make_entry<OUT, false>(lv[u], fu, bad));
+                        }
+                    }
                     __syncthreads();
                     cached_s = s;
                     cached_t = (int)t;
                 }
-                if constexpr (VEC) {
-                    if (sv.kw == 2)
-                        expand_keys_vec<OUT, 2>(sv, sa, a - sa, e - sa, hot, n_hot, fU, m.nU, out_s, N, status, s);
-                    else
-                        expand_keys_vec<OUT, 1>(sv, sa, a - sa, e - sa, hot, n_hot, fU, m.nU, out_s, N, status, s);
-                } else {
+                if (VEC && fu.in_smem) {
+                    if constexpr (VEC) {
+                    if (sv.kw == 2) expand_keys_vec<OUT, 2>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
+                    else expand_keys_vec<OUT, 1>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
+                    }
+                } else {  // scalar path: odd shapes, or |U| too large for shared memory
                     for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
                         const uint64_t rel = v - sa;
                         uint32_t g = sv.kw == 2 ? ld_le16(sv.keys + 2 * rel) : sv.keys[rel];
-                        if (g >= sv.G) { report(status, SPP_ERR_CORRUPT, s); g = 0; }
-                        const E en = g < n_hot ? hot[g] : make_entry<OUT>(ld_ro_u2(sv.lut + 8ull * g), fU, m.nU, status, s);
+                        bad |= g >= sv.G;
+                        g = g < sv.G ? g : 0u;
+                        const E en = g < n_hot ? lds_entry<OUT>(hot_base + g * EB)
+                                               : make_entry<OUT, false>(ld_ro_u2(sv.lut + 8ull * g), fu_g, bad);
                         store1<OUT>(out_s, N, v, en);
                     }
                 }
             } else if (sv.kw == 0) {
                 // broadcast of a constant 4-group
-                const E en = make_entry<OUT>(ld_ro_u2(sv.lut), fU, m.nU, status, s);
+                const E en = make_entry<OUT, false>(ld_ro_u2(sv.lut), fu_g, bad);
                 if constexpr (VEC) {
                     E e8[8];
 #pragma unroll
@@ -348,10 +422,11 @@ __global__ void __launch_bounds__(kThreads) kc_expand(const void *const *__restr
                     ent.x = (uint32_t)ld_le16(sv.keys + 2 * rel) | ((uint32_t)ld_le16(sv.keys + 2 * (Nt + rel)) << 16);
                     ent.y = (uint32_t)ld_le16(sv.keys + 2 * (2 * Nt + rel)) |
                             ((uint32_t)ld_le16(sv.keys + 2 * (3 * Nt + rel)) << 16);
-                    store1<OUT>(out_s, N, v, make_entry<OUT>(ent, fU, m.nU, status, s));
+                    store1<OUT>(out_s, N, v, make_entry<OUT, false>(ent, fu_g, bad));
                 }
             }
         }
+        if (bad) report(status, SPP_ERR_CORRUPT, s);
     }
 }
 
@@ -360,7 +435,7 @@ spp_status launch_expand(const void *const *d_src, int n, const float *fU, const
                          const spp_decode_opts &o, uint64_t N, cudaStream_t stream, const DeviceProps &dp) {
     auto kern = kc_expand<OUT, VEC>;
     const int entry_bytes = OUT == SPP_OUT_F32 ? 16 : 8;
-    const int smem = kHotBytes;
+    const int smem = kHotBytes + kUCap * (int)sizeof(float);
     static int attr_done[8] = {0};  // per template instance (device-agnostic attribute)
     const int key = (OUT - 1) * 2 + (VEC ? 1 : 0);
     if (!attr_done[key]) {
@@ -381,7 +456,7 @@ spp_status launch_expand(const void *const *d_src, int n, const float *fU, const
     const uint64_t items = (uint64_t)n * ips;
     const int grid = (int)std::min<uint64_t>(items, (uint64_t)ctas);
     kern<<<grid, kThreads, smem, stream>>>(d_src, n, fU, meta, dst, o.H, o.W, N, chunk, ips,
-                                           (uint32_t)(smem / entry_bytes), o.status);
+                                           (uint32_t)(kHotBytes / entry_bytes), o.status);
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }
 
