@@ -331,10 +331,11 @@ int orc_deepcam_code(int b) {
 /* Decodes line l of the stream into xhat[W] (before normalisation). */
 int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat) {
     if (!src || !xhat || size < 64 || rd32(src) != 0x44505053u || rd16(src + 4) != 1) return ORC_ECORRUPT;
-    int C = rd16(src + 8), H = rd16(src + 10), W = rd16(src + 12);
+    int C = rd16(src + 8), H = rd16(src + 10), W = rd16(src + 12), A = rd16(src + 14);
     uint32_t L = rd32(src + 16);
     uint64_t dir_off = rd64(src + 24), payload_off = rd64(src + 32), total = rd64(src + 40);
     if (C < 1 || H < 1 || W < 1 || L != (uint32_t)C * (uint32_t)H || total > size) return ORC_ECORRUPT;
+    if (A < 1 || W % A != 0) return ORC_ECORRUPT;            /* segment alignment (FORMAT.md 2.1) */
     if (l < 0 || (uint32_t)l >= L) return ORC_EINVAL;
     if (dir_off + 4 * ((uint64_t)L + 1) > total) return ORC_ECORRUPT;
     uint32_t a = rd32(src + dir_off + 4 * (uint64_t)l), b = rd32(src + dir_off + 4 * (uint64_t)l + 4);
@@ -357,7 +358,7 @@ int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat)
         const uint8_t *d = p + 4 + 4 * (uint64_t)s;
         int len = rd16(d), kind = d[2], emin_b = d[3];
         float h = f32_of_bits(rd32(p + 4 + 4 * (uint64_t)nseg + 4 * (uint64_t)s));
-        if (len < 1 || pos + len > W) return ORC_ECORRUPT;
+        if (len < 1 || pos + len > W || pos % A != 0) return ORC_ECORRUPT;
         if (kind == 0) {                                 /* REPEAT: broadcast the head */
             for (int j = 0; j < len; j++) xhat[pos + j] = h;
         } else if (kind == 1) {                          /* DIFF */
@@ -431,10 +432,16 @@ static int ceil_log2(double q) {
     return (f == 0.5) ? e - 1 : e;
 }
 
-/* Encode one line; returns SEG byte size, fills seg (or NULL to size only). */
+/* Encode one line (FORMAT.md 2.4) with segment alignment A; returns the SEG
+ * byte size, or -1 if no aligned segmentation exists (the line is then RAW). */
 typedef struct { int len, kind, emin_b; float head; } seg_t;
 
-static int64_t encode_line(const float *x, int W, seg_t *segs, int *nseg_out, uint8_t *deltas,
+static int rep_len(const int *run, int i, int W, int A) {
+    int r = run[i];
+    return (i + r == W) ? r : (r / A) * A;
+}
+
+static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_out, uint8_t *deltas,
                            int64_t *ndelta_out, int *run) {
     /* run lengths of bit-identical values */
     run[W - 1] = 1;
@@ -444,10 +451,11 @@ static int64_t encode_line(const float *x, int W, seg_t *segs, int *nseg_out, ui
     int64_t nd = 0;
     int i = 0;
     while (i < W) {
-        if (run[i] >= 16) {
-            segs[nseg].len = run[i]; segs[nseg].kind = 0; segs[nseg].emin_b = 0; segs[nseg].head = x[i];
+        int rl = rep_len(run, i, W, A);
+        if (rl >= 16) {
+            segs[nseg].len = rl; segs[nseg].kind = 0; segs[nseg].emin_b = 0; segs[nseg].head = x[i];
             nseg++;
-            i += run[i];
+            i += rl;
             continue;
         }
         float h = x[i];
@@ -462,32 +470,43 @@ static int64_t encode_line(const float *x, int W, seg_t *segs, int *nseg_out, ui
             if (emin < -149) emin = -149;
             if (emin > 96) emin = 96;
         }
-        float unit = ldexpf(1.0f, emin);
-        int64_t S = 0;
-        float prev = h;
-        int j = i + 1;
-        while (j < W) {
-            if (run[j] >= 16) break;
-            double t = ldexp((double)x[j] - (double)prev, -emin);
-            if (fabs(t) > 1984.5) break;
-            int b = quantise(t);
-            int k = orc_deepcam_code(b);
-            if (llabs(S + k) > 1983LL * 1984LL) break;
-            S += k;
-            float xh = h + (float)S * unit;
-            if (deltas) deltas[nd] = (uint8_t)b;
-            nd++;
-            prev = xh;
-            j++;
+        int64_t nd0 = nd;
+        int end;
+        for (;;) {                                       /* (re)encode the segment from i */
+            float unit = ldexpf(1.0f, emin);
+            int64_t S = 0;
+            float prev = h;
+            int j = i + 1, overflow = 0;
+            nd = nd0;
+            while (j < W) {
+                if (j % A == 0 && rep_len(run, j, W, A) >= 16) break;
+                double t = ldexp((double)x[j] - (double)prev, -emin);
+                if (fabs(t) > 1984.5) { overflow = 1; break; }
+                int b = quantise(t);
+                int k = orc_deepcam_code(b);
+                if (llabs(S + k) > 1983LL * 1984LL) { overflow = 1; break; }
+                S += k;
+                prev = h + (float)S * unit;
+                if (deltas) deltas[nd] = (uint8_t)b;
+                nd++;
+                j++;
+            }
+            if (!overflow) { end = j; break; }
+            end = (j / A) * A;
+            if (end > i) { nd = nd0 + (end - i - 1); break; }   /* drop deltas of positions >= end */
+            if (emin >= 96) return -1;                          /* no aligned segmentation: RAW */
+            emin++;                                             /* overflow inside the first A values */
         }
-        segs[nseg].len = j - i; segs[nseg].kind = 1; segs[nseg].emin_b = emin + 150; segs[nseg].head = h;
+        segs[nseg].len = end - i; segs[nseg].kind = 1; segs[nseg].emin_b = emin + 150; segs[nseg].head = h;
         nseg++;
-        i = j;
+        i = end;
     }
     *nseg_out = nseg;
     *ndelta_out = nd;
     return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
 }
+
+int orc_deepcam_align(int W) { return W % 384 == 0 ? 12 : (W % 8 == 0 ? 8 : 1); }
 
 size_t orc_deepcam_max_encoded_size(int C, int H, int W) {
     uint64_t L = (uint64_t)C * H;
@@ -498,6 +517,7 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     if ((uint64_t)C * H > 0xFFFFFFFFull) return ORC_EINVAL;
     init_mags();
+    const int A = orc_deepcam_align(W);
     uint64_t L = (uint64_t)C * H;
     uint64_t dir_off = 64, payload_off = up16(dir_off + 4 * (L + 1));
     uint64_t raw_size = up16(16 + 4 * (uint64_t)W);
@@ -513,8 +533,8 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
         uint64_t sz = raw_size;
         if (finite) {
             int nseg; int64_t nd;
-            uint64_t seg_size = (uint64_t)encode_line(xl, W, segs, &nseg, NULL, &nd, run);
-            if (seg_size < raw_size) sz = seg_size;
+            int64_t seg_size = encode_line(xl, W, A, segs, &nseg, NULL, &nd, run);
+            if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
         }
         pay += sz;
     }
@@ -525,6 +545,7 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
     memset(dst, 0, (size_t)total);
     wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);
     wr16(dst + 8, (uint16_t)C); wr16(dst + 10, (uint16_t)H); wr16(dst + 12, (uint16_t)W);
+    wr16(dst + 14, (uint16_t)A);
     wr32(dst + 16, (uint32_t)L);
     wr64(dst + 24, dir_off); wr64(dst + 32, payload_off); wr64(dst + 40, total);
     uint64_t cur = 0;
@@ -535,8 +556,8 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
         int finite = 1;
         for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
         int nseg = 0; int64_t nd = 0;
-        uint64_t seg_size = finite ? (uint64_t)encode_line(xl, W, segs, &nseg, deltas, &nd, run) : raw_size + 1;
-        if (seg_size < raw_size) {
+        int64_t seg_size = finite ? encode_line(xl, W, A, segs, &nseg, deltas, &nd, run) : -1;
+        if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
             p[0] = 1; wr16(p + 2, (uint16_t)nseg);
             for (int s = 0; s < nseg; s++) {
                 wr16(p + 4 + 4 * s, (uint16_t)segs[s].len);
@@ -545,7 +566,7 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
                 wr32(p + 4 + 4 * (uint64_t)nseg + 4 * s, bits_of_f32(segs[s].head));
             }
             memcpy(p + 4 + 8 * (uint64_t)nseg, deltas, (size_t)nd);
-            cur += seg_size;
+            cur += (uint64_t)seg_size;
         } else {
             p[0] = 0;
             for (int k = 0; k < W; k++) wr32(p + 16 + 4 * (uint64_t)k, bits_of_f32(xl[k]));

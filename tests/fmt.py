@@ -38,10 +38,10 @@ def cosmo_keys(b, slab, Nt):
 
 def deepcam_header(b: np.ndarray):
     raw = bytes(b[:64])
-    magic, ver, flags, C, H, W, pad, L, res, dir_off, payload_off, total = struct.unpack_from(
+    magic, ver, flags, C, H, W, A, L, res, dir_off, payload_off, total = struct.unpack_from(
         "<IHHHHHHIIQQQ", raw, 0)
     d = np.frombuffer(bytes(b[dir_off:dir_off + 4 * (L + 1)]), dtype="<u4")
-    return dict(magic=magic, ver=ver, C=C, H=H, W=W, L=L, dir=d, dir_off=dir_off,
+    return dict(magic=magic, ver=ver, C=C, H=H, W=W, A=A, L=L, dir=d, dir_off=dir_off,
                 payload_off=payload_off, total=total)
 
 
@@ -80,8 +80,9 @@ def build_raw_line(x):
     return bytes(out)
 
 
-def build_deepcam_stream(C, H, W, lines):
-    """Assemble a whole DeepCAM stream from per-line payloads (FORMAT.md 2.1)."""
+def build_deepcam_stream(C, H, W, lines, A=1):
+    """Assemble a whole DeepCAM stream from per-line payloads (FORMAT.md 2.1);
+    A is the declared segment alignment."""
     L = C * H
     assert len(lines) == L
     dir_off = 64
@@ -91,7 +92,7 @@ def build_deepcam_stream(C, H, W, lines):
     for ln in lines:
         offs.append(offs[-1] + len(ln))
     total = payload_off + offs[-1]
-    hdr = struct.pack("<IHHHHHHIIQQQ", 0x44505053, 1, 0, C, H, W, 0, L, 0, dir_off, payload_off, total)
+    hdr = struct.pack("<IHHHHHHIIQQQ", 0x44505053, 1, 0, C, H, W, A, L, 0, dir_off, payload_off, total)
     hdr += b"\0" * 16
     body = bytearray(hdr)
     body += np.asarray(offs, dtype="<u4").tobytes()

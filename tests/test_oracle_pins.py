@@ -427,3 +427,36 @@ def test_deepcam_decoder_rejects_corruption(orc):
     for ln in (bad_len, bad_kind, bad_emin):
         with pytest.raises(orc.OracleError):
             orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [ln]), 0, W)
+
+
+def test_deepcam_segment_alignment(orc):
+    """FORMAT.md 2.1/2.4: the encoder aligns segment starts to A (12 when
+    W % 384 == 0, 8 when W % 8 == 0, else 1) and decoders reject violations."""
+    rng = np.random.default_rng(33)
+    for W, A in ((384, 12), (1152, 12), (64, 8), (200, 8), (37, 1)):
+        x = np.cumsum(rng.standard_normal((1, 6, W)) * 0.05, axis=2).astype(np.float32)
+        x[0, 1, W // 3: W // 3 + 40] = 2.5                  # a run
+        x[0, 2, W // 2] += 1e4                              # an abrupt jump (forces a split)
+        x[0, 3] = np.where(rng.random(W) < 0.7, 0.0, rng.random(W) * 1e-6)
+        b = orc.deepcam_encode(x)
+        h = fmt.deepcam_header(b)
+        assert h["A"] == A
+        for l in range(6):
+            info = fmt.deepcam_line(b, h, l)
+            xh = orc.deepcam_decode_line(b, l, W)
+            if info["mode"] == 1:
+                starts = np.cumsum([0] + [s["len"] for s in info["segs"]])[:-1]
+                assert all(int(st) % A == 0 for st in starts)
+                _check_bound(x[0, l], xh, info["segs"])
+            else:
+                assert np.array_equal(xh.view(np.uint32), x[0, l].view(np.uint32))
+    # a declared alignment the segments violate is corrupt; A must divide W
+    W = 16
+    line = fmt.build_seg_line(W, [(4, 1, 140, 1.0), (12, 0, 0, 2.0)], [1, 2, 3])
+    orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=4), 0, W)
+    with pytest.raises(orc.OracleError):
+        orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=8), 0, W)
+    with pytest.raises(orc.OracleError):
+        orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=3), 0, W)
+    with pytest.raises(orc.OracleError):
+        orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=0), 0, W)
