@@ -176,7 +176,8 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
     B = args.batch or W["batch"]
     dims = W["dims"]
     t_setup = time.perf_counter()
-    bufs, stats = make_pool(args.workload, args.pool or W["pool"], W["seed"] + 1000 * rank,
+    from paper_conf_ipps_ibrahimo22_b200.shard import aggregate_throughput, max_over_ranks, rank_seed_base
+    bufs, stats = make_pool(args.workload, args.pool or W["pool"], rank_seed_base(W["seed"], rank),
                             threads=max(1, (os.cpu_count() or 1) // max(1, world)))
     sizes = [int(b.size) for b in bufs]
     P = len(bufs)
@@ -238,11 +239,8 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
     dec.check_status()
     k_main = float(np.mean([evs[i][1].elapsed_time(evs[i][2]) for i in range(nev)])) / 1e3
     k_pro = float(np.mean([evs[i][0].elapsed_time(evs[i][1]) for i in range(nev)])) / 1e3
-    t = torch.tensor([elapsed], dtype=torch.float64, device=dev)
-    if dist:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    tmax = float(t.item())
-    value = world * B * args.steps / tmax
+    tmax = max_over_ranks(elapsed, dist, dev)          # device-timed, max over ranks
+    value = aggregate_throughput(B, world, args.steps, tmax)
 
     # ---- end to end: pinned host -> H2D (copy stream) overlapped with decode
     e2e_steps = max(1, min(args.steps, args.e2e_steps))
@@ -268,10 +266,8 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
     assert int(st_host.item()) == 0, "decode status"
     e2e_launches = pipe.launches()
     pipe.close()
-    t2 = torch.tensor([s2.elapsed_time(e2) / 1e3], dtype=torch.float64, device=dev)
-    if dist:
-        dist.all_reduce(t2, op=dist.ReduceOp.MAX)
-    e2e_value = world * B * e2e_steps / float(t2.item())
+    t2 = max_over_ranks(s2.elapsed_time(e2) / 1e3, dist, dev)
+    e2e_value = aggregate_throughput(B, world, e2e_steps, t2)
 
     peak, peak_src = _peaks()
     alg = in_bytes + out_bytes

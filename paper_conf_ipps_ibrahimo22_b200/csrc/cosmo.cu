@@ -249,78 +249,115 @@ __device__ __forceinline__ void store1(uint8_t *out_s, uint64_t N, uint64_t v, t
     }
 }
 
-template <int KW>
-struct KeyVec;
-template <>
-struct KeyVec<2> {
+// 8 keys of one group as eight 16-bit lanes of a uint4 (kw = 1 keys are widened
+// at load, so one code path serves both key widths)
+struct Keys8 {
     uint4 v;
-    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel) { v = ld_stream_u4(keys + 2 * rel); }
-    __device__ __forceinline__ uint32_t get(int j) const {
+    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel, int kw) {
+        if (kw == 2) {
+            v = ld_stream_u4(keys + 2 * rel);
+        } else {
+            const uint2 t = ld_stream_u2(keys + rel);
+            v.x = __byte_perm(t.x, 0u, 0x4140);
+            v.y = __byte_perm(t.x, 0u, 0x4342);
+            v.z = __byte_perm(t.y, 0u, 0x4140);
+            v.w = __byte_perm(t.y, 0u, 0x4342);
+        }
+    }
+    __device__ __forceinline__ uint32_t get(int j) const {  // j compile-time
         const uint32_t w = j < 2 ? v.x : j < 4 ? v.y : j < 6 ? v.z : v.w;
         return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
     }
-};
-template <>
-struct KeyVec<1> {
-    uint2 v;
-    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel) { v = ld_stream_u2(keys + rel); }
-    __device__ __forceinline__ uint32_t get(int j) const { return ((j < 4 ? v.x : v.y) >> (8 * (j & 3))) & 0xFFu; }
+    __device__ __forceinline__ uint32_t get_dyn(uint32_t j) const {  // j runtime (rare cold path)
+        const uint32_t w = (j & 4) ? ((j & 2) ? v.w : v.z) : ((j & 2) ? v.y : v.x);
+        return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
+    }
 };
 
-// 8 consecutive voxels: hot tuples from smem; the rare cold keys (beyond the
-// staged prefix) are fetched together in one warp-uniform branch
-template <int OUT, int KW>
-__device__ __forceinline__ void expand8(const KeyVec<KW> &k, const SlabView &sv, uint32_t hot_base, uint32_t n_hot,
-                                        const FuView &fu, uint8_t *out_s, uint64_t N, uint64_t v0, uint32_t &bad) {
-    using E = typename Entry<OUT>::T;
-    constexpr uint32_t EB = sizeof(E);
-    uint32_t g[8];
-    E e[8];
-    uint32_t cold = 0;
-#pragma unroll
-    for (int j = 0; j < 8; j++) {
-        uint32_t gj = k.get(j);
-        bad |= gj >= sv.G;
-        gj = gj < sv.G ? gj : 0u;
-        g[j] = gj;
-        if (gj < n_hot) e[j] = lds_entry<OUT>(hot_base + gj * EB);
-        else cold |= 1u << j;
-    }
-    if (__any_sync(0xffffffffu, cold != 0)) {
-        uint2 lv[8];
-#pragma unroll
-        for (int j = 0; j < 8; j++)
-            if ((cold >> j) & 1u) lv[j] = ld_ro_u2(sv.lut + 8ull * g[j]);
-#pragma unroll
-        for (int j = 0; j < 8; j++)
-            if ((cold >> j) & 1u) e[j] = make_entry<OUT, true>(lv[j], fu, bad);
-    }
-    store8<OUT>(out_s, N, v0, e);
+constexpr uint32_t kNone = 0xFFFFFFFFu;
+
+// resolve one deferred cold voxel: its LUT row `lv` was loaded one iteration
+// earlier; overwrite the placeholder tuple this thread stored for it
+template <int OUT>
+__device__ __forceinline__ void cold_fixup(uint32_t rel, uint2 lv, const FuView &fu, uint8_t *out_s, uint64_t N,
+                                           uint64_t slab_v0, uint32_t &bad) {
+    store1<OUT>(out_s, N, slab_v0 + rel, make_entry<OUT, true>(lv, fu, bad));
 }
 
-// voxels [a, b) of one slab (relative indices), 8 per thread per group; the
-// keys of the next two groups are in flight while a group is expanded
-template <int OUT, int KW>
+// Voxels [a, b) of one slab (relative indices), 8 consecutive voxels per
+// thread per iteration (a warp writes 512 contiguous bytes per plane store),
+// keys prefetched two iterations ahead.  Hot tuples come from the shared
+// memory prefix.  Cold keys (the power-law tail beyond the prefix) are
+// deferred: up to two per thread are queued in registers, their LUT rows are
+// requested at the start of the next iteration and the tuples are rewritten
+// after that iteration's stores (same thread: program order), so no warp
+// waits on an L2 round trip inside an iteration.  A key >= G (corrupt) can
+// only be cold; it is clamped and flagged there.
+template <int OUT>
 __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
                                                 uint32_t hot_base, uint32_t n_hot, const FuView &fu, uint8_t *out_s,
                                                 uint64_t N, uint32_t &bad) {
+    using E = typename Entry<OUT>::T;
+    constexpr uint32_t EB = sizeof(E);
     const uint64_t step = (uint64_t)blockDim.x * 8;
+    const uint32_t Gm1 = sv.G - 1;
     uint64_t q = a + (uint64_t)threadIdx.x * 8;
-    KeyVec<KW> k0, k1;
-    if (q < b) k0.load(sv.keys, q);
-    if (q + step < b) k1.load(sv.keys, q + step);
+    Keys8 k0, k1;
+    if (q < b) k0.load(sv.keys, q, sv.kw);
+    if (q + step < b) k1.load(sv.keys, q + step, sv.kw);
+    uint32_t pv0 = kNone, pv1 = kNone, pg0 = 0, pg1 = 0;  // deferred cold voxels (rel index, key)
 #pragma unroll 1
     for (; q < b; q += step) {
-        KeyVec<KW> k2;
-        if (q + 2 * step < b) k2.load(sv.keys, q + 2 * step);
-        expand8<OUT, KW>(k0, sv, hot_base, n_hot, fu, out_s, N, slab_v0 + q, bad);
+        uint2 lv0, lv1;
+        if (pv0 != kNone) lv0 = ld_ro_u2(sv.lut + 8ull * pg0);
+        if (pv1 != kNone) lv1 = ld_ro_u2(sv.lut + 8ull * pg1);
+        Keys8 k2;
+        if (q + 2 * step < b) k2.load(sv.keys, q + 2 * step, sv.kw);
+        E e[8];
+        uint32_t cold = 0;
+#pragma unroll
+        for (int j = 0; j < 8; j++) {
+            const uint32_t g = k0.get(j);
+            if (g < n_hot) e[j] = lds_entry<OUT>(hot_base + g * EB);
+            else cold |= 1u << j;
+        }
+        store8<OUT>(out_s, N, slab_v0 + q, e);
+        if (pv0 != kNone) cold_fixup<OUT>(pv0, lv0, fu, out_s, N, slab_v0, bad);
+        if (pv1 != kNone) cold_fixup<OUT>(pv1, lv1, fu, out_s, N, slab_v0, bad);
+        pv0 = pv1 = kNone;
+        if (cold) {
+            uint32_t j = __ffs(cold) - 1;
+            uint32_t g = k0.get_dyn(j);
+            bad |= g > Gm1;
+            pv0 = (uint32_t)q + j;
+            pg0 = min(g, Gm1);
+            cold &= cold - 1;
+            if (cold) {
+                j = __ffs(cold) - 1;
+                g = k0.get_dyn(j);
+                bad |= g > Gm1;
+                pv1 = (uint32_t)q + j;
+                pg1 = min(g, Gm1);
+                cold &= cold - 1;
+                while (cold) {  // more than two cold voxels in 8: resolve synchronously (rare)
+                    j = __ffs(cold) - 1;
+                    g = k0.get_dyn(j);
+                    bad |= g > Gm1;
+                    cold_fixup<OUT>((uint32_t)q + j, ld_ro_u2(sv.lut + 8ull * min(g, Gm1)), fu, out_s, N, slab_v0,
+                                    bad);
+                    cold &= cold - 1;
+                }
+            }
+        }
         k0 = k1;
         k1 = k2;
     }
+    if (pv0 != kNone) cold_fixup<OUT>(pv0, ld_ro_u2(sv.lut + 8ull * pg0), fu, out_s, N, slab_v0, bad);
+    if (pv1 != kNone) cold_fixup<OUT>(pv1, ld_ro_u2(sv.lut + 8ull * pg1), fu, out_s, N, slab_v0, bad);
 }
 
 template <int OUT, bool VEC>
-__global__ void __launch_bounds__(kThreads, 2) kc_expand(const void *const *__restrict__ src, int n,
+__global__ void __launch_bounds__(kThreads, 3) kc_expand(const void *const *__restrict__ src, int n,
                                                          const float *__restrict__ fU_ws,
                                                          const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
                                                          int H, int W, uint64_t N, uint64_t chunk,
@@ -386,10 +423,7 @@ __global__ void __launch_bounds__(kThreads, 2) kc_expand(const void *const *__re
                     cached_t = (int)t;
                 }
                 if (VEC && fu.in_smem) {
-                    if constexpr (VEC) {
-                    if (sv.kw == 2) expand_keys_vec<OUT, 2>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
-                    else expand_keys_vec<OUT, 1>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
-                    }
+                    if constexpr (VEC) expand_keys_vec<OUT>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
                 } else {  // scalar path: odd shapes, or |U| too large for shared memory
                     for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
                         const uint64_t rel = v - sa;

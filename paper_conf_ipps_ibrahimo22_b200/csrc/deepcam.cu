@@ -46,7 +46,7 @@ struct DcMeta {  // written by KD0, read by KD (32 B)
     const uint8_t *payload;
     uint64_t limit;  // bytes available from payload
     uint32_t valid;
-    uint32_t pad;
+    uint32_t align;  // declared segment alignment A (FORMAT.md 2.1)
 };
 
 constexpr int kMaxWarpsPerCta = 8;
@@ -65,9 +65,10 @@ __global__ void kd0_parse(const void *const *__restrict__ src, const uint64_t *_
         ok = ld_le32(b) == kDeepcamMagic && ld_le16(b + 4) == kVersion && ld_le16(b + kC) == C &&
              ld_le16(b + kH) == H && ld_le16(b + kW) == W && ld_le32(b + kL) == L;
         const uint64_t dir_off = ld_le64(b + kDirOff), pay = ld_le64(b + kPayloadOff), total = ld_le64(b + kTotal);
+        const uint32_t A = ld_le16(b + kAlign);
         ok = ok && total <= limit && (dir_off & 3) == 0 && dir_off + 4 * (L + 1) <= total && (pay & 15) == 0 &&
-             pay <= total;
-        if (ok) m = DcMeta{b + dir_off, b + pay, total - pay, 1u, 0u};
+             pay <= total && A >= 1 && (uint32_t)W % A == 0;
+        if (ok) m = DcMeta{b + dir_off, b + pay, total - pay, 1u, A};
     }
     if (!ok) report(status, SPP_ERR_CORRUPT, s);
     meta[s] = m;
@@ -139,8 +140,9 @@ __device__ __forceinline__ void emit_scalar(uint8_t *row, uint32_t p0, uint32_t 
 
 // Decode one staged line (warp-cooperative).  Returns false if malformed.
 template <int OUT, bool VEC>
-__device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *sbits,
-                                            uint32_t nwords, float shv, float scv, uint8_t *row, int lane) {
+__device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t A, uint32_t *sbits,
+                                            uint32_t *wpre, uint32_t nwords, float shv, float scv, uint8_t *row,
+                                            int lane) {
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t mode = hdr & 0xFFu;
     if (mode == kModeRaw) {
@@ -191,7 +193,7 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
         const uint32_t st = cl + il - len, db = cd + id - dlen;
         if (s < nseg) {
             bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
-                   st + len > W;
+                   st + len > W || st % A != 0;
             if (st < W) atomicOr(&sbits[st >> 5], 1u << (st & 31));
             const int a = (int)db - (int)st - 1;
             desc[s] = (uint32_t)(a + 16384) | (kind << 16) | (eb << 24);
@@ -202,33 +204,51 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
     bad = __any_sync(0xffffffffu, bad) || cl != W || 4u + 8u * nseg + cd > bytes;
     if (bad) return false;
     __syncwarp();
+    // starts in the bitmap words before word w (segment index of a position =
+    // starts before it + starts at or below it in its word - 1)
+    {
+        uint32_t carry_w = 0;
+        for (uint32_t w0 = 0; w0 < nwords; w0 += kWarp) {
+            const uint32_t w = w0 + lane;
+            const uint32_t c = w < nwords ? __popc(sbits[w]) : 0u;
+            const uint32_t ic = warp_incl_scan(c, lane);
+            if (w < nwords) wpre[w] = carry_w + ic - c;
+            carry_w += __shfl_sync(0xffffffffu, ic, 31);
+        }
+    }
+    __syncwarp();
 
-    // 2. chunks of 256 positions, 8 per lane
-    float carry = 0.f;
-    uint32_t segc = 0;
+    // 2. chunks of 256 positions, lane owns [p0, p0 + 8).  All code sums are
+    // fp32 multiples of 2^-130 below 2^-106 in magnitude: exact in any order.
+    const uint32_t dl_s = smem_u32(dl);
+    float carry_P = 0.f;     // line prefix of codes before this chunk
+    float carry_base = 0.f;  // line prefix before the head of the segment open at the chunk start
+    const uint32_t below_mask = (1u << lane) - 1u;
     for (uint32_t c0 = 0; c0 < W; c0 += 256) {
         const uint32_t p0 = c0 + 8 * lane;
         const bool act = p0 < W;
-        uint32_t sb = 0, valid = 0;
+        uint32_t sb = 0, valid = 0, nbefore = 0;
         if (act) {
-            sb = (sbits[p0 >> 5] >> (p0 & 31)) & 0xFFu;
+            const uint32_t word = sbits[p0 >> 5];
+            sb = (word >> (p0 & 31)) & 0xFFu;
             valid = W - p0 >= 8 ? 0xFFu : ((1u << (W - p0)) - 1u);
             sb &= valid;
+            nbefore = wpre[p0 >> 5] + __popc(word & ((1u << (p0 & 31)) - 1u));
         }
-        const uint32_t cnt = __popc(sb);
-        const uint32_t icnt = warp_incl_scan(cnt, lane);
-        const int s_prev = (int)(segc + icnt - cnt) - 1;
-        segc += __shfl_sync(0xffffffffu, icnt, 31);
+        const int s_prev = (int)nbefore - 1;  // segment of position p0 - 1
 
-        float v[8], hj[8], scj[8];
-        uint32_t keep = 0, reset = 0, bigm = 0;
-        if ((sb >> 1) == 0) {
-            // fast path: all 8 positions in one segment (a head may sit at position 0)
+        // local sums: r[j] = codes since the last head in the lane (or since p0),
+        // pl = plain lane total, lv = plain prefix before the lane's last head
+        float r[8], hj[8], scj[8];
+        uint32_t started = 0, keep = 0, bigm = 0;
+        float pl = 0.f, lv = 0.f;
+        if (!__any_sync(0xffffffffu, (sb >> 1) != 0)) {
+            // fast path: every lane's 8 positions lie in one segment (head allowed at p0)
             const int s = act ? s_prev + (int)(sb & 1u) : 0;
             const SegInfo si = seg_info(desc, heads, s);
             float f[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
             if (act && si.kind == kDiff) {
-                const uint32_t addr = smem_u32(dl) + (uint32_t)(si.a + (int)p0);
+                const uint32_t addr = dl_s + (uint32_t)(si.a + (int)p0);
                 const uint32_t al = addr & ~3u, shb = (addr & 3u) * 8u;
                 uint32_t w0, w1, w2;
                 asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w0) : "r"(al));
@@ -244,16 +264,17 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
                 f[0] = code_f<0>(lo); f[1] = code_f<1>(lo); f[2] = code_f<2>(lo); f[3] = code_f<3>(lo);
                 f[4] = code_f<0>(hi); f[5] = code_f<1>(hi); f[6] = code_f<2>(hi); f[7] = code_f<3>(hi);
             }
-            v[0] = f[0];
+            r[0] = f[0];
 #pragma unroll
-            for (int j = 1; j < 8; j++) v[j] = v[j - 1] + f[j];
+            for (int j = 1; j < 8; j++) r[j] = r[j - 1] + f[j];
+            pl = r[7];
 #pragma unroll
             for (int j = 0; j < 8; j++) { hj[j] = si.h; scj[j] = si.sc; }
+            started = (sb & 1u) ? 0xFFu : 0u;
             keep = si.kind == kRepeat ? 0xFFu : (sb & 1u);
-            reset = (sb & 1u) ? 0xFFu : 0u;
             bigm = si.big ? 0xFFu : 0u;
         } else {
-            // general path: segment boundaries inside the lane's 8 positions
+            // general path: segment heads inside the lane's 8 positions
             int s = s_prev;
             SegInfo si = seg_info(desc, heads, s < 0 ? 0 : s);
             float run = 0.f;
@@ -263,43 +284,50 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
                 if ((sb >> j) & 1u) {
                     s++;
                     si = seg_info(desc, heads, s);
+                    lv = pl;  // plain prefix before this head
                     run = 0.f;
-                    reset |= 0xFFu << j;
+                    started |= 0xFFu << j;
                     keep |= 1u << j;
                 } else if ((valid >> j) & 1u) {
-                    if (si.kind == kRepeat) keep |= 1u << j;
-                    else run += code_f_byte(dl[si.a + (int)p]);
+                    if (si.kind == kRepeat) {
+                        keep |= 1u << j;
+                    } else {
+                        const float f = code_f_byte(dl[si.a + (int)p]);
+                        run += f;
+                        pl += f;
+                    }
                 }
-                v[j] = run;
+                r[j] = run;
                 hj[j] = si.h;
                 scj[j] = si.sc;
                 if (si.big) bigm |= 1u << j;
             }
+            started &= 0xFFu;
         }
-        // warp segmented inclusive scan of the lane totals (reset at heads)
-        float x = v[7];
-        uint32_t fl = sb != 0;
+        // plain inclusive warp scan of the lane totals
+        float P = pl;
 #pragma unroll
         for (int d = 1; d < kWarp; d <<= 1) {
-            const float y = __shfl_up_sync(0xffffffffu, x, d);
-            const uint32_t fy = __shfl_up_sync(0xffffffffu, fl, d);
-            if (lane >= d) {
-                if (!fl) x += y;
-                fl |= fy;
-            }
+            const float y = __shfl_up_sync(0xffffffffu, P, d);
+            if (lane >= d) P += y;
         }
-        const float xe = __shfl_up_sync(0xffffffffu, x, 1);
-        const uint32_t fe = __shfl_up_sync(0xffffffffu, fl, 1);
-        const float excl = lane == 0 ? carry : (fe ? xe : xe + carry);
-        const float xl = __shfl_sync(0xffffffffu, x, 31);
-        const uint32_t fll = __shfl_sync(0xffffffffu, fl, 31);
-        carry = fll ? xl : xl + carry;
+        const float P_excl = carry_P + (P - pl);      // line prefix before p0
+        const float lastbase = P_excl + lv;           // prefix before this lane's last head
+        const uint32_t smask = __ballot_sync(0xffffffffu, sb != 0);
+        const uint32_t below = smask & below_mask;
+        const int src = below ? 31 - __clz(below) : lane;
+        const float gotb = __shfl_sync(0xffffffffu, lastbase, src);
+        const float B_in = below ? gotb : carry_base;  // prefix before the head of the segment open at p0
+        const float dlt = P_excl - B_in;
+        carry_P += __shfl_sync(0xffffffffu, P, 31);
+        const float topb = __shfl_sync(0xffffffffu, lastbase, smask ? 31 - __clz(smask) : 0);
+        if (smask) carry_base = topb;
         if (!act) continue;
         float y[8];
 #pragma unroll
         for (int j = 0; j < 8; j++) {
-            float S = ((reset >> j) & 1u) ? v[j] : v[j] + excl;  // exact: multiples of 2^-130 below 2^-106
-            if ((bigm >> j) & 1u) S *= 0x1p100f;                  // keep the scale representable
+            float S = ((started >> j) & 1u) ? r[j] : r[j] + dlt;  // exact
+            if ((bigm >> j) & 1u) S *= 0x1p100f;                   // keep the scale representable
             const float xh = ((keep >> j) & 1u) ? hj[j] : __fmaf_rn(S, scj[j], hj[j]);
             y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
         }
@@ -309,8 +337,188 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
     return true;
 }
 
-template <int OUT, bool VEC>
-__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
+// ---------------------------------------------------------------------------
+// Aligned fast path: the sample declares segment alignment A == VPL, so each
+// lane's VPL positions lie in exactly one segment and a segment head can only
+// sit at a lane's first position.  One bitmap word per 32*VPL-position chunk
+// (bit = "a segment starts at this lane's p0") gives every lane its segment
+// index with one shared load and a popc.
+template <int VPL>
+struct Bytes;  // VPL delta bytes starting at an arbitrary shared address, as words
+template <>
+struct Bytes<8> {
+    uint32_t w[2];
+    __device__ __forceinline__ void load(uint32_t addr) {
+        const uint32_t al = addr & ~3u, sh = (addr & 3u) * 8u;
+        uint32_t v0, v1, v2;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(al));
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(al + 4));
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v2) : "r"(al + 8));
+        w[0] = __funnelshift_r(v0, v1, sh);
+        w[1] = __funnelshift_r(v1, v2, sh);
+    }
+};
+template <>
+struct Bytes<12> {
+    uint32_t w[3];
+    __device__ __forceinline__ void load(uint32_t addr) {
+        const uint32_t al = addr & ~3u, sh = (addr & 3u) * 8u;
+        uint32_t v0, v1, v2, v3;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(al));
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(al + 4));
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v2) : "r"(al + 8));
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v3) : "r"(al + 12));
+        w[0] = __funnelshift_r(v0, v1, sh);
+        w[1] = __funnelshift_r(v1, v2, sh);
+        w[2] = __funnelshift_r(v2, v3, sh);
+    }
+};
+
+template <int OUT, int VPL>
+__device__ __forceinline__ void emit_vpl(uint8_t *row, uint32_t p0, const float (&y)[VPL]) {
+    if constexpr (VPL == 8) {
+        emit8<OUT>(row, p0, 0, y);
+    } else if constexpr (OUT == SPP_OUT_F32) {
+#pragma unroll
+        for (int k = 0; k < VPL / 4; k++)
+            st_stream_u4(row + 4ull * (p0 + 4 * k), make_uint4(__float_as_uint(y[4 * k]), __float_as_uint(y[4 * k + 1]),
+                                                               __float_as_uint(y[4 * k + 2]), __float_as_uint(y[4 * k + 3])));
+    } else {
+        uint32_t h[VPL / 2];
+#pragma unroll
+        for (int k = 0; k < VPL / 2; k++) {
+            __half2 v = __floats2half2_rn(y[2 * k], y[2 * k + 1]);
+            h[k] = *reinterpret_cast<uint32_t *>(&v);
+        }
+#pragma unroll
+        for (int k = 0; k < VPL / 4; k++)  // 8-B aligned: p0 is a multiple of 4 halves
+            asm volatile("st.global.cs.v2.u32 [%0], {%1,%2};" ::"l"(row + 2ull * (p0 + 4 * k)), "r"(h[2 * k]),
+                         "r"(h[2 * k + 1])
+                         : "memory");
+    }
+}
+
+template <int OUT, int VPL>
+__device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
+                                                    uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
+    const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
+    const uint32_t nseg = hdr >> 16;
+    if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;
+    uint32_t *desc = reinterpret_cast<uint32_t *>(buf + 4);
+    const float *heads = reinterpret_cast<const float *>(buf + 4 + 4 * nseg);
+    const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
+
+    // segment table: starts (block bitmap), byte bases (in place), validation
+    if ((uint32_t)lane < nbw) bbits[lane] = 0;
+    __syncwarp();
+    uint32_t cl = 0, cd = 0;
+    bool bad = false;
+    for (uint32_t b0 = 0; b0 < nseg; b0 += kWarp) {
+        const uint32_t s = b0 + lane;
+        uint32_t len = 0, kind = 0, eb = 0;
+        if (s < nseg) {
+            const uint32_t d = desc[s];
+            len = d & 0xFFFFu;
+            kind = (d >> 16) & 0xFFu;
+            eb = d >> 24;
+        }
+        const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
+        const uint32_t il = warp_incl_scan(len, lane), id = warp_incl_scan(dlen, lane);
+        const uint32_t st = cl + il - len, db = cd + id - dlen;
+        if (s < nseg) {
+            const uint32_t blk = st / VPL;
+            bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
+                   st + len > W || blk * VPL != st;
+            if (st < W) atomicOr(&bbits[blk >> 5], 1u << (blk & 31));
+            desc[s] = (uint32_t)((int)db - (int)st - 1 + 16384) | (kind << 16) | (eb << 24);
+        }
+        cl += __shfl_sync(0xffffffffu, il, 31);
+        cd += __shfl_sync(0xffffffffu, id, 31);
+    }
+    bad = __any_sync(0xffffffffu, bad) || cl != W || 4u + 8u * nseg + cd > bytes;
+    if (bad) return false;
+    __syncwarp();
+
+    const uint32_t below = (1u << lane) - 1u;
+    const uint32_t le_mask = 0xFFFFFFFFu >> (31 - lane);
+    float carry_P = 0.f, carry_base = 0.f;
+    uint32_t carry_seg = 0;
+    for (uint32_t c = 0, c0 = 0; c0 < W; c++, c0 += 32 * VPL) {
+        const uint32_t p0 = c0 + VPL * lane;
+        const bool act = p0 < W;
+        const uint32_t word = bbits[c];
+        const uint32_t flag = act ? (word >> lane) & 1u : 0u;  // a segment starts at p0
+        const int s = act ? (int)(carry_seg + __popc(word & below) + flag) - 1 : 0;
+        carry_seg += __popc(word);
+        const SegInfo si = seg_info(desc, heads, s);
+        float pl[VPL];
+        if (act && si.kind == kDiff) {
+            Bytes<VPL> bt;
+            bt.load(dl_s + (uint32_t)(si.a + (int)p0));
+            if (flag) bt.w[0] &= 0xFFFFFF00u;  // the head has no delta byte
+            if constexpr (VPL == 8) {
+                if (W - p0 < 8) {  // positions past the line end (W % 256 != 0)
+                    const uint64_t m = (1ull << (8 * (W - p0))) - 1ull;
+                    bt.w[0] &= (uint32_t)m;
+                    bt.w[1] &= (uint32_t)(m >> 32);
+                }
+            }
+            float f[VPL];
+#pragma unroll
+            for (int k = 0; k < VPL / 4; k++) {
+                f[4 * k + 0] = code_f<0>(bt.w[k]);
+                f[4 * k + 1] = code_f<1>(bt.w[k]);
+                f[4 * k + 2] = code_f<2>(bt.w[k]);
+                f[4 * k + 3] = code_f<3>(bt.w[k]);
+            }
+            pl[0] = f[0];
+#pragma unroll
+            for (int j = 1; j < VPL; j++) pl[j] = pl[j - 1] + f[j];
+        } else {
+#pragma unroll
+            for (int j = 0; j < VPL; j++) pl[j] = 0.f;
+        }
+        // plain inclusive scan of lane totals; base = prefix before the head of
+        // this lane's segment (its head lane in this chunk, else carried)
+        const float tot = pl[VPL - 1];
+        float P = tot;
+#pragma unroll
+        for (int d = 1; d < kWarp; d <<= 1) {
+            const float y = __shfl_up_sync(0xffffffffu, P, d);
+            if (lane >= d) P += y;
+        }
+        const float P_excl = carry_P + (P - tot);
+        const uint32_t smask = __ballot_sync(0xffffffffu, flag != 0);
+        const uint32_t mle = smask & le_mask;
+        const float gotb = __shfl_sync(0xffffffffu, P_excl, mle ? 31 - __clz(mle) : lane);
+        const float base = mle ? gotb : carry_base;
+        const float dlt = P_excl - base;
+        carry_P += __shfl_sync(0xffffffffu, P, 31);
+        const float topb = __shfl_sync(0xffffffffu, P_excl, smask ? 31 - __clz(smask) : 0);
+        if (smask) carry_base = topb;
+        if (!act) continue;
+        float y[VPL];
+        if (si.kind == kRepeat) {
+            const float yr = __fmul_rn(__fsub_rn(si.h, shv), scv);
+#pragma unroll
+            for (int j = 0; j < VPL; j++) y[j] = yr;
+        } else {
+            const float pre = si.big ? 0x1p100f : 1.0f;  // keeps 2^(emin+k) representable
+#pragma unroll
+            for (int j = 0; j < VPL; j++) {
+                const float S = (pl[j] + dlt) * pre;                 // exact
+                const float xh = __fmaf_rn(S, si.sc, si.h);          // RN(h + S * 2^emin)
+                y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+            }
+            if (flag) y[0] = __fmul_rn(__fsub_rn(si.h, shv), scv);  // the head is exact
+        }
+        emit_vpl<OUT, VPL>(row, p0, y);
+    }
+    return true;
+}
+
+template <int OUT, bool VEC, int VPL>
+__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
     uint32_t *__restrict__ status) {
@@ -318,16 +526,19 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int wpc = blockDim.x >> 5;
     uint8_t *base = smem_raw + (size_t)warp * warp_bytes;
-    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + 2 * cap);
-    uint64_t *mbar = reinterpret_cast<uint64_t *>(base + 2 * cap + 4 * nwords);
+    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + 2 * cap);  // also the aligned path's block bitmap
+    uint32_t *wpre = sbits + nwords;
+    uint64_t *mbar = reinterpret_cast<uint64_t *>(base + 2 * cap + 8 * nwords);
     const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
     const uint32_t cap_data = cap - 16;       // one slot; the last 16 B are read slack
     const uint32_t big_cap = 2 * cap - 16;    // both slots (any legal SEG line fits, FORMAT.md 2.1)
+    const uint32_t nbw = (W / VPL + 31) / 32;
 
     const uint64_t T = (uint64_t)n * L;
     const uint64_t NW = (uint64_t)gridDim.x * wpc;
     const uint64_t gw = (uint64_t)blockIdx.x * wpc + warp;
     const uint64_t g_begin = gw * T / NW, g_end = (gw + 1) * T / NW;
+    if (g_begin >= g_end) return;
 
     if (lane == 0) {
         mbar_init(&mbar[0], 1);
@@ -336,35 +547,44 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
     }
     __syncwarp();
 
-    // lane-0 pipeline state: directory entries are loaded one line ahead of the
-    // line whose copy is being issued, so their latency hides behind a decode.
+    // line coordinates tracked incrementally (no divisions per line): decode
+    // position (s, l, y, c) and the lane-0 directory prefetch position (ps, pl)
+    uint32_t s_cur = (uint32_t)(g_begin / L), l_cur = (uint32_t)(g_begin - (uint64_t)s_cur * L);
+    uint32_t c_cur = l_cur / H, y_cur = l_cur - c_cur * H;
+    uint32_t ps = s_cur, pline = l_cur;
+
+    // lane-0 pipeline state
     int64_t cs = -1;
     DcMeta cm{nullptr, nullptr, 0, 0, 0};
     uint32_t da = 0, db = 0;
     const uint8_t *dpay = nullptr;
     uint64_t dlim = 0;
-    uint32_t dvalid = 0;
+    uint32_t dvalid = 0, dalign = 0;
     int64_t dsample = 0;
-    auto load_dir = [&](uint64_t g) {
-        const int64_t s = (int64_t)(g / L);
-        const uint32_t l = (uint32_t)(g - (uint64_t)s * L);
-        if (s != cs) {
-            cm = meta[s];
-            cs = s;
+    auto load_dir = [&]() {  // directory entry of line (ps, pline), then advance
+        if ((int64_t)ps != cs) {
+            cm = meta[ps];
+            cs = ps;
         }
         dvalid = cm.valid;
+        dalign = cm.align;
         dpay = cm.payload;
         dlim = cm.limit;
-        dsample = s;
+        dsample = ps;
         if (dvalid) {
             const uint32_t *dir = reinterpret_cast<const uint32_t *>(cm.dir);
-            da = __ldg(dir + l);
-            db = __ldg(dir + l + 1);
+            da = __ldg(dir + pline);
+            db = __ldg(dir + pline + 1);
+        }
+        if (++pline == L) {
+            pline = 0;
+            ps++;
         }
     };
     // validate the loaded entry: bytes (0 = skip), big = needs both slots
-    auto prepare = [&](const uint8_t *&src, uint32_t &big) -> uint32_t {
+    auto prepare = [&](const uint8_t *&src, uint32_t &big, uint32_t &al) -> uint32_t {
         big = 0;
+        al = dalign;
         if (!dvalid) return 0;
         const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= dlim && db - da >= 16;
         if (!ok) {
@@ -386,31 +606,32 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
         bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
     };
 
-    uint32_t cur_bytes = 0, cur_big = 0, phase0 = 0, phase1 = 0;
+    uint32_t cur_bytes = 0, cur_big = 0, cur_al = 0, phase0 = 0, phase1 = 0;
     const uint8_t *cur_src = nullptr;
     int slot = 0;
-    if (lane == 0 && g_begin < g_end) {
-        load_dir(g_begin);
-        cur_bytes = prepare(cur_src, cur_big);
+    if (lane == 0) {
+        load_dir();
+        cur_bytes = prepare(cur_src, cur_big, cur_al);
         if (cur_bytes && !cur_big) issue(0, cur_src, cur_bytes);
-        if (g_begin + 1 < g_end) load_dir(g_begin + 1);
+        if (g_begin + 1 < g_end) load_dir();
     }
     for (uint64_t g = g_begin; g < g_end; g++) {
-        uint32_t nxt_bytes = 0, nxt_big = 0, nxt_issued = 0;
+        uint32_t nxt_bytes = 0, nxt_big = 0, nxt_issued = 0, nxt_al = 0;
         const uint8_t *nxt_src = nullptr;
         if (lane == 0) {
             if (g + 1 < g_end) {
-                nxt_bytes = prepare(nxt_src, nxt_big);
+                nxt_bytes = prepare(nxt_src, nxt_big, nxt_al);
                 // an oversize current line occupies both slots: issue the next later
                 if (nxt_bytes && !nxt_big && !cur_big) {
                     issue(slot ^ 1, nxt_src, nxt_bytes);
                     nxt_issued = 1;
                 }
             }
-            if (g + 2 < g_end) load_dir(g + 2);
+            if (g + 2 < g_end) load_dir();
         }
         const uint32_t bytes = __shfl_sync(0xffffffffu, cur_bytes, 0);
         const uint32_t big = __shfl_sync(0xffffffffu, cur_big, 0);
+        const uint32_t al = __shfl_sync(0xffffffffu, cur_al, 0);
         if (bytes) {
             uint8_t *buf = base + slot * cap;
             if (big) {
@@ -427,13 +648,15 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
                 mbar_wait(&mbar[1], phase1);
                 phase1 ^= 1;
             }
-            const uint32_t l = (uint32_t)(g % L);
-            const uint32_t c = l / H;
-            const float shv = shift ? __ldg(shift + c) : 0.f;
-            const float scv = scale ? __ldg(scale + c) : 1.f;
+            const float shv = shift ? __ldg(shift + c_cur) : 0.f;
+            const float scv = scale ? __ldg(scale + c_cur) : 1.f;
             uint8_t *row = dst + g * (uint64_t)W * ob;
-            const bool ok = decode_line<OUT, VEC>(buf, bytes, W, sbits, nwords, shv, scv, row, lane);
-            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
+            bool ok;
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg))
+                ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            else
+                ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)s_cur);
         }
         __syncwarp();
         if (lane == 0 && nxt_bytes && !nxt_big && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
@@ -441,21 +664,32 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp) kd_decode(
         cur_bytes = nxt_bytes;
         cur_big = nxt_big;
         cur_src = nxt_src;
+        cur_al = nxt_al;
+        if (++y_cur == H) {
+            y_cur = 0;
+            c_cur++;
+        }
+        if (++l_cur == L) {
+            l_cur = 0;
+            s_cur++;
+            c_cur = 0;
+            y_cur = 0;
+        }
     }
 }
 
-template <int OUT, bool VEC>
+template <int OUT, bool VEC, int VPL>
 spp_status launch_kd(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
                      const DeviceProps &dp) {
     const uint32_t W = (uint32_t)o.W;
     const uint32_t cap = (uint32_t)round_up16(16 + 4ull * W) + 16;
-    const uint32_t nwords = (((W + 31) / 32 + 1) + 3) & ~3u;
-    const uint32_t warp_bytes = 2 * cap + 4 * nwords + 16;
+    const uint32_t nwords = (W + 31) / 32 + 1;  // start bitmap (+1 spare word), and its prefix counts
+    const uint32_t warp_bytes = (uint32_t)round_up16(2 * cap + 8 * nwords + 16);  // keeps every warp region 16-B aligned
     int wpc = kMaxWarpsPerCta;
     while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
     if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
     const int smem = wpc * (int)warp_bytes;
-    auto kern = kd_decode<OUT, VEC>;
+    auto kern = kd_decode<OUT, VEC, VPL>;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return SPP_ERR_CUDA;
     int occ = 0;
@@ -487,13 +721,16 @@ spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const sp
     if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
     const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
     const bool vec = o.W % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
+    const bool v12 = vec && o.W % 384 == 0;  // 12 positions per lane, 3 full chunks for W = 1152
     spp_status r = SPP_ERR_INVALID_ARG;
     if (o.out == SPP_OUT_F32)
-        r = vec ? launch_kd<SPP_OUT_F32, true>(meta, n, d_dst, o, stream, dp)
-                : launch_kd<SPP_OUT_F32, false>(meta, n, d_dst, o, stream, dp);
+        r = v12 ? launch_kd<SPP_OUT_F32, true, 12>(meta, n, d_dst, o, stream, dp)
+                : vec ? launch_kd<SPP_OUT_F32, true, 8>(meta, n, d_dst, o, stream, dp)
+                      : launch_kd<SPP_OUT_F32, false, 8>(meta, n, d_dst, o, stream, dp);
     else if (o.out == SPP_OUT_F16)
-        r = vec ? launch_kd<SPP_OUT_F16, true>(meta, n, d_dst, o, stream, dp)
-                : launch_kd<SPP_OUT_F16, false>(meta, n, d_dst, o, stream, dp);
+        r = v12 ? launch_kd<SPP_OUT_F16, true, 12>(meta, n, d_dst, o, stream, dp)
+                : vec ? launch_kd<SPP_OUT_F16, true, 8>(meta, n, d_dst, o, stream, dp)
+                      : launch_kd<SPP_OUT_F16, false, 8>(meta, n, d_dst, o, stream, dp);
     if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;
     return r;
 }

@@ -60,24 +60,34 @@ inline int ceil_log2(double q) {
 
 struct Seg { uint16_t len; uint8_t kind, emin_b; float head; };
 
+// segment alignment (FORMAT.md 2.4): the GPU decodes 12 (W % 384 == 0) or 8
+// positions per lane; aligned segment starts keep every lane inside one segment
+inline int alignment_for(int W) { return W % 384 == 0 ? 12 : (W % 8 == 0 ? 8 : 1); }
+
 struct LineEncoder {
-    int W;
+    int W, A;
     std::vector<int> run;
     std::vector<Seg> segs;
     std::vector<uint8_t> deltas;
-    explicit LineEncoder(int w) : W(w), run(w), segs(), deltas() { segs.reserve(w); deltas.reserve(w); }
+    LineEncoder(int w, int a) : W(w), A(a), run(w), segs(), deltas() { segs.reserve(w); deltas.reserve(w); }
 
-    // returns the SEG payload size; fills segs/deltas
-    uint64_t encode(const float *x) {
+    int rep(int i) const {
+        const int r = run[i];
+        return i + r == W ? r : (r / A) * A;
+    }
+
+    // SEG payload size, or -1 when no aligned segmentation exists (RAW)
+    int64_t encode(const float *x) {
         segs.clear();
         deltas.clear();
         run[W - 1] = 1;
         for (int i = W - 2; i >= 0; i--) run[i] = fbits(x[i]) == fbits(x[i + 1]) ? run[i + 1] + 1 : 1;
         int i = 0;
         while (i < W) {
-            if (run[i] >= kRepeatMin) {
-                segs.push_back(Seg{(uint16_t)run[i], kRepeat, 0, x[i]});
-                i += run[i];
+            const int rl = rep(i);
+            if (rl >= kRepeatMin) {
+                segs.push_back(Seg{(uint16_t)rl, kRepeat, 0, x[i]});
+                i += rl;
                 continue;
             }
             const float h = x[i];
@@ -92,25 +102,36 @@ struct LineEncoder {
                 emin = ceil_log2(m / (double)kMaxCode);
                 emin = emin < -149 ? -149 : (emin > 96 ? 96 : emin);
             }
-            const float unit = ldexpf(1.0f, emin);
-            int64_t S = 0;
-            float prev = h;
-            int j = i + 1;
-            for (; j < W; j++) {
-                if (run[j] >= kRepeatMin) break;
-                double t = ldexp((double)x[j] - (double)prev, -emin);
-                if (fabs(t) > kMaxCode + 0.5) break;
-                int k;
-                int b = kCodes.quantise(t, &k);
-                if (llabs(S + k) > kMaxAbsS) break;
-                S += k;
-                prev = h + (float)S * unit;                // decoder's x̂_j (fp32, one rounding)
-                deltas.push_back((uint8_t)b);
+            const size_t nd0 = deltas.size();
+            int end;
+            for (;;) {  // (re)encode the segment starting at i
+                deltas.resize(nd0);
+                const float unit = ldexpf(1.0f, emin);
+                int64_t S = 0;
+                float prev = h;
+                int j = i + 1;
+                bool overflow = false;
+                for (; j < W; j++) {
+                    if (j % A == 0 && rep(j) >= kRepeatMin) break;
+                    double t = ldexp((double)x[j] - (double)prev, -emin);
+                    if (fabs(t) > kMaxCode + 0.5) { overflow = true; break; }
+                    int k;
+                    int b = kCodes.quantise(t, &k);
+                    if (llabs(S + k) > kMaxAbsS) { overflow = true; break; }
+                    S += k;
+                    prev = h + (float)S * unit;                // decoder's x̂_j (fp32, one rounding)
+                    deltas.push_back((uint8_t)b);
+                }
+                if (!overflow) { end = j; break; }
+                end = (j / A) * A;
+                if (end > i) { deltas.resize(nd0 + (size_t)(end - i - 1)); break; }
+                if (emin >= 96) return -1;
+                emin++;
             }
-            segs.push_back(Seg{(uint16_t)(j - i), kDiff, (uint8_t)(emin + kEminBias), h});
-            i = j;
+            segs.push_back(Seg{(uint16_t)(end - i), kDiff, (uint8_t)(emin + kEminBias), h});
+            i = end;
         }
-        return round_up16(4 + 8 * (uint64_t)segs.size() + deltas.size());
+        return (int64_t)round_up16(4 + 8 * (uint64_t)segs.size() + deltas.size());
     }
 };
 
@@ -136,7 +157,8 @@ extern "C" spp_status spp_encode_deepcam(const float *x, int C, int H, int W, vo
     const uint64_t dir_off = spp::kHeaderBytes;
     const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
     const uint64_t raw_size = round_up16(16 + 4 * (uint64_t)W);
-    LineEncoder enc(W);
+    const int A = alignment_for(W);
+    LineEncoder enc(W, A);
     // pass 1: per-line size (SEG vs RAW)
     std::vector<uint8_t> is_seg(L);
     std::vector<uint32_t> dir(L + 1);
@@ -146,8 +168,8 @@ extern "C" spp_status spp_encode_deepcam(const float *x, int C, int H, int W, vo
         uint64_t sz = raw_size;
         is_seg[l] = 0;
         if (all_finite(xl, W)) {
-            uint64_t seg = enc.encode(xl);
-            if (seg < raw_size) { sz = seg; is_seg[l] = 1; }
+            const int64_t seg = enc.encode(xl);
+            if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
         }
         if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;
         dir[l] = (uint32_t)cur;
@@ -167,6 +189,7 @@ extern "C" spp_status spp_encode_deepcam(const float *x, int C, int H, int W, vo
     u16 = (uint16_t)C; memcpy(out + kC, &u16, 2);
     u16 = (uint16_t)H; memcpy(out + kH, &u16, 2);
     u16 = (uint16_t)W; memcpy(out + kW, &u16, 2);
+    u16 = (uint16_t)A; memcpy(out + kAlign, &u16, 2);
     u32 = (uint32_t)L; memcpy(out + kL, &u32, 4);
     memcpy(out + kDirOff, &dir_off, 8);
     memcpy(out + kPayloadOff, &payload_off, 8);

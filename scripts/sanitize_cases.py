@@ -1,0 +1,46 @@
+"""Small decodes (valid and corrupted streams) for compute-sanitizer runs:
+   compute-sanitizer --tool memcheck|racecheck|synccheck python scripts/sanitize_cases.py
+Corrupt streams must be reported through the status word with no
+out-of-bounds access (SURVEY.md §5 failure detection)."""
+import sys
+from pathlib import Path
+
+import numpy as np
+
+sys.path.insert(0, str(Path(__file__).resolve().parent.parent))
+import torch  # noqa: E402
+
+from paper_conf_ipps_ibrahimo22_b200 import Decoder, spp  # noqa: E402
+from synth import gen_cosmo, gen_deepcam  # noqa: E402
+from tests import fmt  # noqa: E402
+
+
+def run(fmt_name, bufs, dims, **kw):
+    dec = Decoder(fmt_name, dims, **kw)
+    srcs = [torch.from_numpy(b).cuda() for b in bufs]
+    sizes = torch.tensor([b.size for b in bufs], dtype=torch.int64, device="cuda")
+    dec.decode(srcs, src_bytes=sizes)
+    torch.cuda.synchronize()
+    return int(dec.status.item())
+
+
+x = gen_cosmo(1001, n=32)
+b = spp.spp_encode_cosmo(x)
+h = fmt.cosmo_header(b)
+bad = b.copy(); bad[h["slabs"][0]["keys_off"]:h["slabs"][0]["keys_off"] + 64] = 0xFF
+trunc = b[: b.size // 2].copy()
+lut = b.copy(); lut[h["slabs"][0]["lut_off"]:h["slabs"][0]["lut_off"] + 16] = 0xFF
+print("cosmo ok", run("cosmo", [b, b], x.shape))
+print("cosmo bad keys", run("cosmo", [b, bad], x.shape))
+print("cosmo bad lut", run("cosmo", [lut, b], x.shape, out="f32"))
+print("cosmo truncated", run("cosmo", [b, trunc], x.shape))
+y = gen_deepcam(2001, H=16)
+d = spp.spp_encode_deepcam(y)
+hd = fmt.deepcam_header(d)
+dbad = d.copy(); dbad[hd["payload_off"] + 2: hd["payload_off"] + 4] = 0xFF      # nseg huge
+dtr = d[: d.size // 3].copy()
+ddir = d.copy(); ddir[hd["dir_off"] + 8: hd["dir_off"] + 12] = 0xFF             # bad directory entry
+print("deepcam ok", run("deepcam", [d, d], y.shape))
+print("deepcam bad nseg", run("deepcam", [d, dbad], y.shape))
+print("deepcam truncated", run("deepcam", [dtr, d], y.shape))
+print("deepcam bad dir", run("deepcam", [d, ddir], y.shape, out="f32"))
