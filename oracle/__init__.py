@@ -63,6 +63,8 @@ def lib():
         L.orc_deepcam_decode.argtypes = [P, SZ, P, P, I, P, I, I, I]; L.orc_deepcam_decode.restype = I
         L.orc_deepcam_max_encoded_size.argtypes = [I, I, I]; L.orc_deepcam_max_encoded_size.restype = SZ
         L.orc_deepcam_encode.argtypes = [P, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_deepcam_encode.restype = I
+        L.orc_deepcam_encode_a.argtypes = [P, I, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_deepcam_encode_a.restype = I
+        L.orc_deepcam_align.argtypes = [I]; L.orc_deepcam_align.restype = I
         _lib = L
     return _lib
 
@@ -123,14 +125,16 @@ def deepcam_code(b: int) -> int:
     return int(lib().orc_deepcam_code(int(b)))
 
 
-def deepcam_encode(x: np.ndarray) -> np.ndarray:
+def deepcam_encode(x: np.ndarray, align: int | None = None) -> np.ndarray:
+    """FORMAT.md 2.4 encoder; `align` overrides the default alignment rule."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     assert a.ndim == 3
     Cc, H, W = a.shape
     cap = lib().orc_deepcam_max_encoded_size(Cc, H, W)
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
-    _check(lib().orc_deepcam_encode(_p(a), Cc, H, W, _p(dst), cap, C.byref(size)), "deepcam_encode")
+    A = lib().orc_deepcam_align(W) if align is None else int(align)
+    _check(lib().orc_deepcam_encode_a(_p(a), Cc, H, W, A, _p(dst), cap, C.byref(size)), "deepcam_encode")
     return dst[: size.value].copy()
 
 

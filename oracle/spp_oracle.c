@@ -506,18 +506,24 @@ static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_
     return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
 }
 
-int orc_deepcam_align(int W) { return W % 384 == 0 ? 12 : (W % 8 == 0 ? 8 : 1); }
+int orc_deepcam_align(int W) { return W == 1152 ? 36 : (W % 8 == 0 ? 8 : 1); }
 
 size_t orc_deepcam_max_encoded_size(int C, int H, int W) {
     uint64_t L = (uint64_t)C * H;
     return (size_t)(64 + up16(4 * (L + 1)) + L * up16(16 + 4 * (uint64_t)W));
 }
 
+int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *dst, size_t cap, size_t *size);
+
 int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_deepcam_encode_a(x, C, H, W, orc_deepcam_align(W), dst, cap, size);
+}
+
+/* same policy with an explicit alignment A (W % A == 0) */
+int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *dst, size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
-    if ((uint64_t)C * H > 0xFFFFFFFFull) return ORC_EINVAL;
+    if ((uint64_t)C * H > 0xFFFFFFFFull || A < 1 || W % A != 0) return ORC_EINVAL;
     init_mags();
-    const int A = orc_deepcam_align(W);
     uint64_t L = (uint64_t)C * H;
     uint64_t dir_off = 64, payload_off = up16(dir_off + 4 * (L + 1));
     uint64_t raw_size = up16(16 + 4 * (uint64_t)W);

@@ -35,15 +35,17 @@ def _stale() -> bool:
     return any(p.stat().st_mtime > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> Path:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: Path | None = None) -> Path:
+    """Build libspp.so (or, for experiments, a variant with extra -D defines at `out`)."""
+    target = Path(out) if out else LIB
+    if not force and not defines and out is None and not _stale():
         return LIB
-    objdir = PKG / "_build"
+    objdir = PKG / ("_build" if not defines else "_build_" + "_".join(d.replace("=", "") for d in defines))
     objdir.mkdir(exist_ok=True)
     objs = []
     for src in sources():
         obj = objdir / (src.name + ".o")
-        cmd = [NVCC, *NVCC_FLAGS, "-c", str(src), "-o", str(obj)]
+        cmd = [NVCC, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-c", str(src), "-o", str(obj)]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
@@ -52,15 +54,15 @@ def build(force: bool = False, verbose: bool = False) -> Path:
         if verbose:
             sys.stderr.write(r.stderr)
         objs.append(str(obj))
-    tmp = LIB.with_suffix(".so.tmp")
+    tmp = target.with_suffix(".so.tmp")
     cmd = [NVCC, *GENCODE, "-shared", "-cudart", "shared", "-o", str(tmp), *objs,
            "-Xlinker", "-rpath,/usr/local/cuda/lib64"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc link failed")
-    tmp.replace(LIB)
-    return LIB
+    tmp.replace(target)
+    return target
 
 
 if __name__ == "__main__":

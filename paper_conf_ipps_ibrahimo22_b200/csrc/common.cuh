@@ -36,14 +36,23 @@ __device__ __forceinline__ float ld_ro_f32(const float *p) {
     asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(p));
     return r;
 }
-// write-once outputs: streaming (evict-first) so they do not displace LUTs in L2
+// write-once outputs (SPP_STORE_CS=1: streaming / evict-first, else default write-back)
+#ifndef SPP_STORE_CS
+#define SPP_STORE_CS 0
+#endif
+#if SPP_STORE_CS
+#define SPP_ST_POLICY ".cs"
+#else
+#define SPP_ST_POLICY ""
+#endif
 __device__ __forceinline__ void st_stream_u4(void *p, uint4 v) {
-    asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+    asm volatile("st.global" SPP_ST_POLICY ".v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+                 "r"(v.w)
                  : "memory");
 }
 // 256-bit store (Blackwell-only STG.E.ENL2.256)
 __device__ __forceinline__ void st_stream_f8(void *p, const float *v) {
-    asm volatile("st.global.cs.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v[0]), "f"(v[1]),
+    asm volatile("st.global" SPP_ST_POLICY ".v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v[0]), "f"(v[1]),
                  "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
                  : "memory");
 }

@@ -275,6 +275,10 @@ struct Keys8 {
 };
 
 constexpr uint32_t kNone = 0xFFFFFFFFu;
+#ifndef SPP_KC_PF
+#define SPP_KC_PF 2
+#endif
+constexpr int kKeyPF = SPP_KC_PF;  // key prefetch depth (iterations ahead)
 
 // resolve one deferred cold voxel: its LUT row `lv` was loaded one iteration
 // earlier; overwrite the placeholder tuple this thread stored for it
@@ -302,17 +306,20 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     const uint64_t step = (uint64_t)blockDim.x * 8;
     const uint32_t Gm1 = sv.G - 1;
     uint64_t q = a + (uint64_t)threadIdx.x * 8;
-    Keys8 k0, k1;
-    if (q < b) k0.load(sv.keys, q, sv.kw);
-    if (q + step < b) k1.load(sv.keys, q + step, sv.kw);
+    Keys8 kq[kKeyPF];  // keys of the next kKeyPF iterations (in flight)
+#pragma unroll
+    for (int i = 0; i < kKeyPF; i++)
+        if (q + i * step < b) kq[i].load(sv.keys, q + i * step, sv.kw);
     uint32_t pv0 = kNone, pv1 = kNone, pg0 = 0, pg1 = 0;  // deferred cold voxels (rel index, key)
 #pragma unroll 1
     for (; q < b; q += step) {
         uint2 lv0, lv1;
         if (pv0 != kNone) lv0 = ld_ro_u2(sv.lut + 8ull * pg0);
         if (pv1 != kNone) lv1 = ld_ro_u2(sv.lut + 8ull * pg1);
-        Keys8 k2;
-        if (q + 2 * step < b) k2.load(sv.keys, q + 2 * step, sv.kw);
+        const Keys8 k0 = kq[0];
+#pragma unroll
+        for (int i = 0; i + 1 < kKeyPF; i++) kq[i] = kq[i + 1];
+        if (q + kKeyPF * step < b) kq[kKeyPF - 1].load(sv.keys, q + kKeyPF * step, sv.kw);
         E e[8];
         uint32_t cold = 0;
 #pragma unroll
@@ -349,8 +356,6 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 }
             }
         }
-        k0 = k1;
-        k1 = k2;
     }
     if (pv0 != kNone) cold_fixup<OUT>(pv0, ld_ro_u2(sv.lut + 8ull * pg0), fu, out_s, N, slab_v0, bad);
     if (pv1 != kNone) cold_fixup<OUT>(pv1, ld_ro_u2(sv.lut + 8ull * pg1), fu, out_s, N, slab_v0, bad);

@@ -60,9 +60,10 @@ inline int ceil_log2(double q) {
 
 struct Seg { uint16_t len; uint8_t kind, emin_b; float head; };
 
-// segment alignment (FORMAT.md 2.4): the GPU decodes 12 (W % 384 == 0) or 8
-// positions per lane; aligned segment starts keep every lane inside one segment
-inline int alignment_for(int W) { return W % 384 == 0 ? 12 : (W % 8 == 0 ? 8 : 1); }
+// segment alignment (FORMAT.md 2.4): the GPU decodes 36 (W = 1152, one line per
+// warp pass) or 8 positions per lane; aligned segment starts keep every lane
+// inside one segment
+inline int alignment_for(int W) { return W == 1152 ? 36 : (W % 8 == 0 ? 8 : 1); }
 
 struct LineEncoder {
     int W, A;

@@ -8,13 +8,15 @@ Function names mirror the C ABI.
 from __future__ import annotations
 
 import ctypes as C
+import os
 from pathlib import Path
 from typing import Sequence
 
 import numpy as np
 
 _PKG = Path(__file__).resolve().parent
-LIB_PATH = _PKG / "libspp.so"
+# SPP_LIB may point at an experimental build variant (scripts/variants.py)
+LIB_PATH = Path(os.environ["SPP_LIB"]) if os.environ.get("SPP_LIB") else _PKG / "libspp.so"
 
 SPP_OK, SPP_ERR_INVALID_ARG, SPP_ERR_BUFFER_TOO_SMALL, SPP_ERR_CORRUPT, SPP_ERR_UNSUPPORTED, SPP_ERR_CUDA = range(6)
 SPP_FMT_COSMO, SPP_FMT_DEEPCAM = 1, 2

@@ -1,0 +1,52 @@
+"""Build libspp variants with compile-time knobs and time KC/KD on the GPU
+(experiments only; the product build is paper_conf_ipps_ibrahimo22_b200/build.py).
+usage: python scripts/variants.py build   (CPU)   |   python scripts/variants.py run (GPU)"""
+import json
+import os
+import subprocess
+import sys
+from pathlib import Path
+
+ROOT = Path(__file__).resolve().parent.parent
+sys.path.insert(0, str(ROOT))
+VARIANTS = {
+    "cs1_pf2": ["SPP_STORE_CS=1", "SPP_KC_PF=2"],
+    "cs0_pf2": ["SPP_STORE_CS=0", "SPP_KC_PF=2"],
+    "cs0_pf3": ["SPP_STORE_CS=0", "SPP_KC_PF=3"],
+    "cs0_pf4": ["SPP_STORE_CS=0", "SPP_KC_PF=4"],
+}
+OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
+
+
+def build():
+    from paper_conf_ipps_ibrahimo22_b200 import build as b
+    OUT.mkdir(exist_ok=True)
+    for name, d in VARIANTS.items():
+        b.build(force=True, defines=d, out=OUT / f"libspp_{name}.so")
+        print("built", name)
+
+
+def run():
+    res = {}
+    for name in VARIANTS:
+        env = dict(os.environ, SPP_LIB=str(OUT / f"libspp_{name}.so"))
+        out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--secondary", "none", "--cpu-seconds", "0.5",
+                              "--e2e-steps", "1", "--steps", "100"], env=env, capture_output=True, text=True)
+        try:
+            d = json.loads(out.stdout.strip().splitlines()[-1])
+            res[name] = {"cosmo": d["value"], "frac": d["roofline"]["frac"]}
+        except Exception as ex:
+            res[name] = {"error": str(ex), "stderr": out.stderr[-500:]}
+        out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--workload", "deepcam", "--cpu-seconds", "0.5",
+                              "--e2e-steps", "1", "--steps", "10"], env=env, capture_output=True, text=True)
+        try:
+            d = json.loads(out.stdout.strip().splitlines()[-1])
+            res[name].update({"deepcam": d["value"], "dfrac": d["roofline"]["frac"]})
+        except Exception as ex:
+            res[name]["derror"] = str(ex)
+        print(name, res[name], flush=True)
+    print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    {"build": build, "run": run}[sys.argv[1]]()
