@@ -47,8 +47,12 @@ struct CosmoMeta {  // written by KC0, read by KC
 
 constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 constexpr int kThreads = 256;
-constexpr int kHotBytes = 48 * 1024;  // shared-memory hot prefix of T per CTA
-constexpr int kUCap = 4096;           // unique values staged in shared memory (16 KB)
+constexpr int kHotBytes = 40 * 1024;  // shared-memory hot prefix of T per CTA
+constexpr int kUCap = 2048;           // unique values staged in shared memory (8 KB)
+constexpr int kKeyStages = 4;         // TMA ring of key tiles
+constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
+constexpr int kStageBytes = kTileVox * 2;
+constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + 2 * kKeyStages * 8;
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
 
@@ -250,20 +254,9 @@ __device__ __forceinline__ void store1(uint8_t *out_s, uint64_t N, uint64_t v, t
 }
 
 // 8 keys of one group as eight 16-bit lanes of a uint4 (kw = 1 keys are widened
-// at load, so one code path serves both key widths)
+// after the shared-memory load, so one code path serves both key widths)
 struct Keys8 {
     uint4 v;
-    __device__ __forceinline__ void load(const uint8_t *keys, uint64_t rel, int kw) {
-        if (kw == 2) {
-            v = ld_stream_u4(keys + 2 * rel);
-        } else {
-            const uint2 t = ld_stream_u2(keys + rel);
-            v.x = __byte_perm(t.x, 0u, 0x4140);
-            v.y = __byte_perm(t.x, 0u, 0x4342);
-            v.z = __byte_perm(t.y, 0u, 0x4140);
-            v.w = __byte_perm(t.y, 0u, 0x4342);
-        }
-    }
     __device__ __forceinline__ uint32_t get(int j) const {  // j compile-time
         const uint32_t w = j < 2 ? v.x : j < 4 ? v.y : j < 6 ? v.z : v.w;
         return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
@@ -274,91 +267,125 @@ struct Keys8 {
     }
 };
 
-constexpr uint32_t kNone = 0xFFFFFFFFu;
-#ifndef SPP_KC_PF
-#define SPP_KC_PF 2
-#endif
-constexpr int kKeyPF = SPP_KC_PF;  // key prefetch depth (iterations ahead)
+// The key stream of the CTA's current range is staged into shared memory by
+// 1-D TMA bulk copies (cp.async.bulk + mbarrier): a ring of kKeyStages tiles of
+// 2048 voxels, refilled by thread 0 as soon as all 8 warps have released a
+// stage (per-stage "empty" mbarriers, one arrival per warp: no CTA barrier),
+// so many KB of key reads are in flight per SM without spending registers.
+// Tile indices are CTA-global (`count` = tiles consumed so far) and select the
+// stage and both mbarrier phases.
+struct KeyRing {
+    uint8_t *buf;      // kKeyStages * kStageBytes
+    uint64_t *full;    // kKeyStages, completed by the TMA transaction count
+    uint64_t *empty;   // kKeyStages, 8 warp arrivals
+    uint32_t count;
+};
 
-// resolve one deferred cold voxel: its LUT row `lv` was loaded one iteration
-// earlier; overwrite the placeholder tuple this thread stored for it
-template <int OUT>
-__device__ __forceinline__ void cold_fixup(uint32_t rel, uint2 lv, const FuView &fu, uint8_t *out_s, uint64_t N,
-                                           uint64_t slab_v0, uint32_t &bad) {
-    store1<OUT>(out_s, N, slab_v0 + rel, make_entry<OUT, true>(lv, fu, bad));
+__device__ __forceinline__ Keys8 keys_from_smem(const uint8_t *stage, uint32_t kwb) {
+    Keys8 k;
+    const uint32_t ka = smem_u32(stage) + threadIdx.x * 8u * kwb;
+    if (kwb == 2) {
+        k.v = lds_u4(ka);
+    } else {
+        const uint2 t = lds_u2(ka);
+        k.v.x = __byte_perm(t.x, 0u, 0x4140);
+        k.v.y = __byte_perm(t.x, 0u, 0x4342);
+        k.v.z = __byte_perm(t.y, 0u, 0x4140);
+        k.v.w = __byte_perm(t.y, 0u, 0x4342);
+    }
+    return k;
 }
 
-// Voxels [a, b) of one slab (relative indices), 8 consecutive voxels per
-// thread per iteration (a warp writes 512 contiguous bytes per plane store),
-// keys prefetched two iterations ahead.  Hot tuples come from the shared
-// memory prefix.  Cold keys (the power-law tail beyond the prefix) are
-// deferred: up to two per thread are queued in registers, their LUT rows are
-// requested at the start of the next iteration and the tuples are rewritten
-// after that iteration's stores (same thread: program order), so no warp
-// waits on an L2 round trip inside an iteration.  A key >= G (corrupt) can
-// only be cold; it is clamped and flagged there.
+// Voxels [a, b) of one slab (relative indices, multiples of 16), 8 consecutive
+// voxels per thread per tile (a warp writes 512 contiguous bytes per plane
+// store).  Hot tuples come from the shared-memory prefix.  Cold keys (the
+// power-law tail beyond the prefix) are looked up one tile ahead: while
+// tile t is expanded, each thread has already classified its keys of tile t+1
+// and requested their LUT rows (up to two per thread; more are fetched in
+// place, rarely), so every group is stored once, complete, and no warp waits
+// on an L2 round trip.  A key >= G (corrupt) can only be cold: clamped, flagged.
 template <int OUT>
 __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
                                                 uint32_t hot_base, uint32_t n_hot, const FuView &fu, uint8_t *out_s,
-                                                uint64_t N, uint32_t &bad) {
+                                                uint64_t N, uint32_t &bad, KeyRing &ring) {
     using E = typename Entry<OUT>::T;
     constexpr uint32_t EB = sizeof(E);
-    const uint64_t step = (uint64_t)blockDim.x * 8;
+    const uint32_t kwb = (uint32_t)sv.kw;
     const uint32_t Gm1 = sv.G - 1;
-    uint64_t q = a + (uint64_t)threadIdx.x * 8;
-    Keys8 kq[kKeyPF];  // keys of the next kKeyPF iterations (in flight)
-#pragma unroll
-    for (int i = 0; i < kKeyPF; i++)
-        if (q + i * step < b) kq[i].load(sv.keys, q + i * step, sv.kw);
-    uint32_t pv0 = kNone, pv1 = kNone, pg0 = 0, pg1 = 0;  // deferred cold voxels (rel index, key)
-#pragma unroll 1
-    for (; q < b; q += step) {
-        uint2 lv0, lv1;
-        if (pv0 != kNone) lv0 = ld_ro_u2(sv.lut + 8ull * pg0);
-        if (pv1 != kNone) lv1 = ld_ro_u2(sv.lut + 8ull * pg1);
-        const Keys8 k0 = kq[0];
-#pragma unroll
-        for (int i = 0; i + 1 < kKeyPF; i++) kq[i] = kq[i + 1];
-        if (q + kKeyPF * step < b) kq[kKeyPF - 1].load(sv.keys, q + kKeyPF * step, sv.kw);
-        E e[8];
+    const uint32_t ntiles = (uint32_t)((b - a + kTileVox - 1) / kTileVox);
+    const uint32_t lane = threadIdx.x & 31;
+    auto issue = [&](uint32_t t) {  // thread 0: bulk copy of tile t's keys once its stage is free
+        const uint32_t gt = ring.count + t;
+        const uint32_t stg = gt % kKeyStages;
+        if (gt >= (uint32_t)kKeyStages) mbar_wait(&ring.empty[stg], ((gt / kKeyStages) - 1) & 1u);
+        const uint64_t st = a + (uint64_t)t * kTileVox;
+        const uint64_t rem = b - st;
+        const uint32_t nvox = rem < (uint64_t)kTileVox ? (uint32_t)rem : (uint32_t)kTileVox;
+        const uint32_t bytes = (nvox * kwb + 15u) & ~15u;
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&ring.full[stg], bytes);
+        bulk_g2s(ring.buf + stg * kStageBytes, sv.keys + st * kwb, bytes, &ring.full[stg]);
+    };
+    auto wait_full = [&](uint32_t t) {
+        const uint32_t gt = ring.count + t;
+        mbar_wait(&ring.full[gt % kKeyStages], (gt / kKeyStages) & 1u);
+        return ring.buf + (gt % kKeyStages) * kStageBytes;
+    };
+    // cold lookahead state for the tile about to be expanded: up to two cold
+    // positions (j) with their LUT rows in flight
+    uint32_t cj0 = 8, cj1 = 8;
+    uint2 lv0 = make_uint2(0, 0), lv1 = make_uint2(0, 0);
+    auto classify = [&](const uint8_t *stage, uint64_t q, uint32_t &j0, uint32_t &j1, uint2 &l0, uint2 &l1) {
+        j0 = j1 = 8;
+        if (q >= b) return;
+        const Keys8 k = keys_from_smem(stage, kwb);
         uint32_t cold = 0;
 #pragma unroll
-        for (int j = 0; j < 8; j++) {
-            const uint32_t g = k0.get(j);
-            if (g < n_hot) e[j] = lds_entry<OUT>(hot_base + g * EB);
-            else cold |= 1u << j;
-        }
-        store8<OUT>(out_s, N, slab_v0 + q, e);
-        if (pv0 != kNone) cold_fixup<OUT>(pv0, lv0, fu, out_s, N, slab_v0, bad);
-        if (pv1 != kNone) cold_fixup<OUT>(pv1, lv1, fu, out_s, N, slab_v0, bad);
-        pv0 = pv1 = kNone;
+        for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
         if (cold) {
-            uint32_t j = __ffs(cold) - 1;
-            uint32_t g = k0.get_dyn(j);
-            bad |= g > Gm1;
-            pv0 = (uint32_t)q + j;
-            pg0 = min(g, Gm1);
+            j0 = __ffs(cold) - 1;
+            l0 = ld_ro_u2(sv.lut + 8ull * min(k.get_dyn(j0), Gm1));
             cold &= cold - 1;
             if (cold) {
-                j = __ffs(cold) - 1;
-                g = k0.get_dyn(j);
-                bad |= g > Gm1;
-                pv1 = (uint32_t)q + j;
-                pg1 = min(g, Gm1);
-                cold &= cold - 1;
-                while (cold) {  // more than two cold voxels in 8: resolve synchronously (rare)
-                    j = __ffs(cold) - 1;
-                    g = k0.get_dyn(j);
-                    bad |= g > Gm1;
-                    cold_fixup<OUT>((uint32_t)q + j, ld_ro_u2(sv.lut + 8ull * min(g, Gm1)), fu, out_s, N, slab_v0,
-                                    bad);
-                    cold &= cold - 1;
-                }
+                j1 = __ffs(cold) - 1;
+                l1 = ld_ro_u2(sv.lut + 8ull * min(k.get_dyn(j1), Gm1));
             }
         }
+    };
+    if (threadIdx.x == 0)
+        for (uint32_t t = 0; t < ntiles && t < (uint32_t)(kKeyStages - 1); t++) issue(t);
+    if (ntiles) classify(wait_full(0), a + 8u * threadIdx.x, cj0, cj1, lv0, lv1);
+#pragma unroll 1
+    for (uint32_t t = 0; t < ntiles; t++) {
+        if (threadIdx.x == 0 && t + kKeyStages - 1 < ntiles) issue(t + kKeyStages - 1);
+        uint32_t nj0 = 8, nj1 = 8;
+        uint2 nl0 = make_uint2(0, 0), nl1 = make_uint2(0, 0);
+        if (t + 1 < ntiles) classify(wait_full(t + 1), a + (uint64_t)(t + 1) * kTileVox + 8u * threadIdx.x, nj0, nj1, nl0, nl1);
+        const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
+        const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
+        if (q < b) {
+            const Keys8 k0 = keys_from_smem(stage, kwb);
+            E e[8];
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                const uint32_t g = k0.get(j);
+                if (g < n_hot) {
+                    e[j] = lds_entry<OUT>(hot_base + g * EB);
+                } else {
+                    bad |= g > Gm1;
+                    const uint2 lv = (uint32_t)j == cj0 ? lv0
+                                     : (uint32_t)j == cj1 ? lv1
+                                                          : ld_ro_u2(sv.lut + 8ull * min(g, Gm1));  // 3rd+ cold: rare
+                    e[j] = make_entry<OUT, true>(lv, fu, bad);
+                }
+            }
+            store8<OUT>(out_s, N, slab_v0 + q, e);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);  // this warp is done with the stage
+        cj0 = nj0; cj1 = nj1; lv0 = nl0; lv1 = nl1;
     }
-    if (pv0 != kNone) cold_fixup<OUT>(pv0, ld_ro_u2(sv.lut + 8ull * pg0), fu, out_s, N, slab_v0, bad);
-    if (pv1 != kNone) cold_fixup<OUT>(pv1, ld_ro_u2(sv.lut + 8ull * pg1), fu, out_s, N, slab_v0, bad);
+    ring.count += ntiles;
 }
 
 template <int OUT, bool VEC>
@@ -373,6 +400,16 @@ __global__ void __launch_bounds__(kThreads, 3) kc_expand(const void *const *__re
     extern __shared__ __align__(16) uint8_t smem_raw[];
     const uint32_t hot_base = smem_u32(smem_raw);
     const uint32_t fu_base = hot_base + kHotBytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes);
+    KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0};
+    if (VEC && threadIdx.x == 0) {
+        for (int i = 0; i < kKeyStages; i++) {
+            mbar_init(&ring.full[i], 1);
+            mbar_init(&ring.empty[i], kThreads / kWarp);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
     const uint64_t plane = (uint64_t)H * W;
     const uint64_t total_items = (uint64_t)n * items_per_sample;
     const uint64_t per = (total_items + gridDim.x - 1) / gridDim.x;
@@ -428,7 +465,7 @@ __global__ void __launch_bounds__(kThreads, 3) kc_expand(const void *const *__re
                     cached_t = (int)t;
                 }
                 if (VEC && fu.in_smem) {
-                    if constexpr (VEC) expand_keys_vec<OUT>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad);
+                    if constexpr (VEC) expand_keys_vec<OUT>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad, ring);
                 } else {  // scalar path: odd shapes, or |U| too large for shared memory
                     for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
                         const uint64_t rel = v - sa;
@@ -474,7 +511,7 @@ spp_status launch_expand(const void *const *d_src, int n, const float *fU, const
                          const spp_decode_opts &o, uint64_t N, cudaStream_t stream, const DeviceProps &dp) {
     auto kern = kc_expand<OUT, VEC>;
     const int entry_bytes = OUT == SPP_OUT_F32 ? 16 : 8;
-    const int smem = kHotBytes + kUCap * (int)sizeof(float);
+    const int smem = kSmemBytes;
     static int attr_done[8] = {0};  // per template instance (device-agnostic attribute)
     const int key = (OUT - 1) * 2 + (VEC ? 1 : 0);
     if (!attr_done[key]) {
@@ -532,7 +569,7 @@ static spp_status cosmo_expand(const void *const *d_src, int n, void *d_dst, con
     const uint64_t N = (uint64_t)o.D * o.H * o.W;
     const uint64_t plane = (uint64_t)o.H * o.W;
     const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
-    const bool vec = plane % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
+    const bool vec = plane % 16 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;  // 16-B key tiles
     uint8_t *dst = static_cast<uint8_t *>(d_dst);
     switch (o.out) {
         case SPP_OUT_F16:

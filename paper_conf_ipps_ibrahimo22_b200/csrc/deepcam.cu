@@ -50,6 +50,9 @@ struct DcMeta {  // written by KD0, read by KD (32 B)
 };
 
 constexpr int kMaxWarpsPerCta = 8;
+#ifndef SPP_KD_MINB
+#define SPP_KD_MINB 2  // CTAs per SM the register allocation targets (2: the 36-per-lane path needs ~128 registers)
+#endif
 constexpr int kMaxW = 16383;  // GPU path: per-segment byte base packed in 16 bits
 
 __global__ void kd0_parse(const void *const *__restrict__ src, const uint64_t *__restrict__ src_bytes, int n, int C,
@@ -344,63 +347,48 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
 // (bit = "a segment starts at this lane's p0") gives every lane its segment
 // index with one shared load and a popc.
 template <int VPL>
-struct Bytes;  // VPL delta bytes starting at an arbitrary shared address, as words
-template <>
-struct Bytes<8> {
-    uint32_t w[2];
+struct Bytes {  // VPL delta bytes starting at an arbitrary shared address, as VPL/4 words
+    static constexpr int NW = VPL / 4;
+    uint32_t w[NW];
     __device__ __forceinline__ void load(uint32_t addr) {
         const uint32_t al = addr & ~3u, sh = (addr & 3u) * 8u;
-        uint32_t v0, v1, v2;
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(al));
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(al + 4));
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v2) : "r"(al + 8));
-        w[0] = __funnelshift_r(v0, v1, sh);
-        w[1] = __funnelshift_r(v1, v2, sh);
-    }
-};
-template <>
-struct Bytes<12> {
-    uint32_t w[3];
-    __device__ __forceinline__ void load(uint32_t addr) {
-        const uint32_t al = addr & ~3u, sh = (addr & 3u) * 8u;
-        uint32_t v0, v1, v2, v3;
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(al));
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(al + 4));
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v2) : "r"(al + 8));
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v3) : "r"(al + 12));
-        w[0] = __funnelshift_r(v0, v1, sh);
-        w[1] = __funnelshift_r(v1, v2, sh);
-        w[2] = __funnelshift_r(v2, v3, sh);
+        uint32_t v[NW + 1];
+#pragma unroll
+        for (int k = 0; k <= NW; k++) asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v[k]) : "r"(al + 4 * k));
+#pragma unroll
+        for (int k = 0; k < NW; k++) w[k] = __funnelshift_r(v[k], v[k + 1], sh);
     }
 };
 
 template <int OUT, int VPL>
 __device__ __forceinline__ void emit_vpl(uint8_t *row, uint32_t p0, const float (&y)[VPL]) {
-    if constexpr (VPL == 8) {
-        emit8<OUT>(row, p0, 0, y);
-    } else if constexpr (OUT == SPP_OUT_F32) {
+    static_assert(VPL == 8, "direct stores: 16-B lanes");
+    emit8<OUT>(row, p0, 0, y);
+}
+
+// one-pass lines (VPL = 36): the warp's output row is staged in shared memory
+// (lane l writes its VPL values at l*VPL) and leaves with one TMA bulk store
+template <int OUT, int VPL>
+__device__ __forceinline__ void stage_vpl(uint32_t sdst, const float (&y)[VPL]) {
+    if constexpr (OUT == SPP_OUT_F32) {
 #pragma unroll
         for (int k = 0; k < VPL / 4; k++)
-            st_stream_u4(row + 4ull * (p0 + 4 * k), make_uint4(__float_as_uint(y[4 * k]), __float_as_uint(y[4 * k + 1]),
-                                                               __float_as_uint(y[4 * k + 2]), __float_as_uint(y[4 * k + 3])));
+            sts_u4(sdst + 16 * k, make_uint4(__float_as_uint(y[4 * k]), __float_as_uint(y[4 * k + 1]),
+                                             __float_as_uint(y[4 * k + 2]), __float_as_uint(y[4 * k + 3])));
     } else {
-        uint32_t h[VPL / 2];
 #pragma unroll
-        for (int k = 0; k < VPL / 2; k++) {
-            __half2 v = __floats2half2_rn(y[2 * k], y[2 * k + 1]);
-            h[k] = *reinterpret_cast<uint32_t *>(&v);
+        for (int k = 0; k < VPL / 4; k++) {
+            __half2 a = __floats2half2_rn(y[4 * k], y[4 * k + 1]);
+            __half2 b = __floats2half2_rn(y[4 * k + 2], y[4 * k + 3]);
+            sts_u2(sdst + 8 * k, make_uint2(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b)));
         }
-#pragma unroll
-        for (int k = 0; k < VPL / 4; k++)  // 8-B aligned: p0 is a multiple of 4 halves
-            asm volatile("st.global.cs.v2.u32 [%0], {%1,%2};" ::"l"(row + 2ull * (p0 + 4 * k)), "r"(h[2 * k]),
-                         "r"(h[2 * k + 1])
-                         : "memory");
     }
 }
 
 template <int OUT, int VPL>
 __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
                                                     uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
+    constexpr bool STAGED = VPL == 36;  // one pass per line (W = 32 * VPL), TMA bulk store of the row
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
     if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;
@@ -408,10 +396,11 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
     const float *heads = reinterpret_cast<const float *>(buf + 4 + 4 * nseg);
     const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
 
-    // segment table: starts (block bitmap), byte bases (in place), validation
+    // segment table: one packed scan of (len | delta-bytes << 16) gives starts
+    // and byte bases; starts go to the block bitmap, byte bases in place
     if ((uint32_t)lane < nbw) bbits[lane] = 0;
     __syncwarp();
-    uint32_t cl = 0, cd = 0;
+    uint32_t cacc = 0;
     bool bad = false;
     for (uint32_t b0 = 0; b0 < nseg; b0 += kWarp) {
         const uint32_t s = b0 + lane;
@@ -423,8 +412,10 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             eb = d >> 24;
         }
         const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
-        const uint32_t il = warp_incl_scan(len, lane), id = warp_incl_scan(dlen, lane);
-        const uint32_t st = cl + il - len, db = cd + id - dlen;
+        const uint32_t pk = len | (dlen << 16);  // both sums stay below 2^16 (W <= 16383)
+        const uint32_t inc = warp_incl_scan(pk, lane);
+        const uint32_t ex = cacc + inc - pk;
+        const uint32_t st = ex & 0xFFFFu, db = ex >> 16;
         if (s < nseg) {
             const uint32_t blk = st / VPL;
             bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
@@ -432,10 +423,9 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             if (st < W) atomicOr(&bbits[blk >> 5], 1u << (blk & 31));
             desc[s] = (uint32_t)((int)db - (int)st - 1 + 16384) | (kind << 16) | (eb << 24);
         }
-        cl += __shfl_sync(0xffffffffu, il, 31);
-        cd += __shfl_sync(0xffffffffu, id, 31);
+        cacc += __shfl_sync(0xffffffffu, inc, 31);
     }
-    bad = __any_sync(0xffffffffu, bad) || cl != W || 4u + 8u * nseg + cd > bytes;
+    bad = __any_sync(0xffffffffu, bad) || (cacc & 0xFFFFu) != W || 4u + 8u * nseg + (cacc >> 16) > bytes;
     if (bad) return false;
     __syncwarp();
 
@@ -463,17 +453,14 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
                     bt.w[1] &= (uint32_t)(m >> 32);
                 }
             }
-            float f[VPL];
+            float run = 0.f;
 #pragma unroll
             for (int k = 0; k < VPL / 4; k++) {
-                f[4 * k + 0] = code_f<0>(bt.w[k]);
-                f[4 * k + 1] = code_f<1>(bt.w[k]);
-                f[4 * k + 2] = code_f<2>(bt.w[k]);
-                f[4 * k + 3] = code_f<3>(bt.w[k]);
+                run += code_f<0>(bt.w[k]); pl[4 * k + 0] = run;
+                run += code_f<1>(bt.w[k]); pl[4 * k + 1] = run;
+                run += code_f<2>(bt.w[k]); pl[4 * k + 2] = run;
+                run += code_f<3>(bt.w[k]); pl[4 * k + 3] = run;
             }
-            pl[0] = f[0];
-#pragma unroll
-            for (int j = 1; j < VPL; j++) pl[j] = pl[j - 1] + f[j];
         } else {
 #pragma unroll
             for (int j = 0; j < VPL; j++) pl[j] = 0.f;
@@ -493,32 +480,49 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         const float gotb = __shfl_sync(0xffffffffu, P_excl, mle ? 31 - __clz(mle) : lane);
         const float base = mle ? gotb : carry_base;
         const float dlt = P_excl - base;
-        carry_P += __shfl_sync(0xffffffffu, P, 31);
-        const float topb = __shfl_sync(0xffffffffu, P_excl, smask ? 31 - __clz(smask) : 0);
-        if (smask) carry_base = topb;
+        if constexpr (!STAGED) {
+            carry_P += __shfl_sync(0xffffffffu, P, 31);
+            const float topb = __shfl_sync(0xffffffffu, P_excl, smask ? 31 - __clz(smask) : 0);
+            if (smask) carry_base = topb;
+        }
         if (!act) continue;
         float y[VPL];
         if (si.kind == kRepeat) {
             const float yr = __fmul_rn(__fsub_rn(si.h, shv), scv);
 #pragma unroll
             for (int j = 0; j < VPL; j++) y[j] = yr;
-        } else {
-            const float pre = si.big ? 0x1p100f : 1.0f;  // keeps 2^(emin+k) representable
+        } else if (!si.big) {
 #pragma unroll
             for (int j = 0; j < VPL; j++) {
-                const float S = (pl[j] + dlt) * pre;                 // exact
-                const float xh = __fmaf_rn(S, si.sc, si.h);          // RN(h + S * 2^emin)
+                const float xh = __fmaf_rn(pl[j] + dlt, si.sc, si.h);  // RN(h + S * 2^emin), S exact
                 y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
             }
             if (flag) y[0] = __fmul_rn(__fsub_rn(si.h, shv), scv);  // the head is exact
+        } else {
+#pragma unroll
+            for (int j = 0; j < VPL; j++) {
+                const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, si.sc, si.h);  // 2^(emin+30) scale
+                y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+            }
+            if (flag) y[0] = __fmul_rn(__fsub_rn(si.h, shv), scv);
         }
-        emit_vpl<OUT, VPL>(row, p0, y);
+        if constexpr (STAGED) {
+            __syncwarp();  // every lane has read its delta bytes and segment: reuse the slot for the row
+            stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+        } else {
+            emit_vpl<OUT, VPL>(row, p0, y);
+        }
+    }
+    if constexpr (STAGED) {
+        fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
+        __syncwarp();
+        if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
     }
     return true;
 }
 
 template <int OUT, bool VEC, int VPL>
-__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
+__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decode(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
     uint32_t *__restrict__ status) {
@@ -601,11 +605,14 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
         return bytes;
     };
     auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {
+        if constexpr (VPL == 36) bulk_wait_read_all();  // a staged row may still be leaving this slot
         fence_proxy_async_smem();
         mbar_arrive_expect_tx(&mbar[slot], bytes);
         bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
     };
 
+    uint32_t c_cached = 0xFFFFFFFFu;
+    float shv = 0.f, scv = 1.f;
     uint32_t cur_bytes = 0, cur_big = 0, cur_al = 0, phase0 = 0, phase1 = 0;
     const uint8_t *cur_src = nullptr;
     int slot = 0;
@@ -635,6 +642,10 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
         if (bytes) {
             uint8_t *buf = base + slot * cap;
             if (big) {
+                if constexpr (VPL == 36) {
+                    if (lane == 0) bulk_wait_read_all();  // both slots are about to be overwritten
+                    __syncwarp();
+                }
                 // stage across both slots with plain 16-B loads (rare: SEG line larger than RAW)
                 const uint64_t sp = __shfl_sync(0xffffffffu, reinterpret_cast<uint64_t>(cur_src), 0);
                 const uint4 *src4 = reinterpret_cast<const uint4 *>(sp);
@@ -648,8 +659,11 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
                 mbar_wait(&mbar[1], phase1);
                 phase1 ^= 1;
             }
-            const float shv = shift ? __ldg(shift + c_cur) : 0.f;
-            const float scv = scale ? __ldg(scale + c_cur) : 1.f;
+            if (c_cur != c_cached) {  // per-channel constants change every H lines
+                c_cached = c_cur;
+                shv = shift ? __ldg(shift + c_cur) : 0.f;
+                scv = scale ? __ldg(scale + c_cur) : 1.f;
+            }
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
             if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg))
@@ -675,6 +689,9 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, 3) kd_decode(
             c_cur = 0;
             y_cur = 0;
         }
+    }
+    if constexpr (VPL == 36) {
+        if (lane == 0) bulk_wait_all();  // shared memory must outlive the last row stores
     }
 }
 
@@ -721,14 +738,14 @@ spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const sp
     if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
     const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
     const bool vec = o.W % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
-    const bool v12 = vec && o.W % 384 == 0;  // 12 positions per lane, 3 full chunks for W = 1152
+    const bool v36 = vec && o.W == 1152;  // the DeepCAM line: 32 lanes x 36 positions, one pass
     spp_status r = SPP_ERR_INVALID_ARG;
     if (o.out == SPP_OUT_F32)
-        r = v12 ? launch_kd<SPP_OUT_F32, true, 12>(meta, n, d_dst, o, stream, dp)
+        r = v36 ? launch_kd<SPP_OUT_F32, true, 36>(meta, n, d_dst, o, stream, dp)
                 : vec ? launch_kd<SPP_OUT_F32, true, 8>(meta, n, d_dst, o, stream, dp)
                       : launch_kd<SPP_OUT_F32, false, 8>(meta, n, d_dst, o, stream, dp);
     else if (o.out == SPP_OUT_F16)
-        r = v12 ? launch_kd<SPP_OUT_F16, true, 12>(meta, n, d_dst, o, stream, dp)
+        r = v36 ? launch_kd<SPP_OUT_F16, true, 36>(meta, n, d_dst, o, stream, dp)
                 : vec ? launch_kd<SPP_OUT_F16, true, 8>(meta, n, d_dst, o, stream, dp)
                       : launch_kd<SPP_OUT_F16, false, 8>(meta, n, d_dst, o, stream, dp);
     if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;

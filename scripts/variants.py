@@ -10,10 +10,8 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "cs1_pf2": ["SPP_STORE_CS=1", "SPP_KC_PF=2"],
-    "cs0_pf2": ["SPP_STORE_CS=0", "SPP_KC_PF=2"],
-    "cs0_pf3": ["SPP_STORE_CS=0", "SPP_KC_PF=3"],
-    "cs0_pf4": ["SPP_STORE_CS=0", "SPP_KC_PF=4"],
+    "kd_minb3": ["SPP_KD_MINB=3"],
+    "kd_minb2": ["SPP_KD_MINB=2"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
@@ -30,13 +28,15 @@ def run():
     res = {}
     for name in VARIANTS:
         env = dict(os.environ, SPP_LIB=str(OUT / f"libspp_{name}.so"))
-        out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--secondary", "none", "--cpu-seconds", "0.5",
-                              "--e2e-steps", "1", "--steps", "100"], env=env, capture_output=True, text=True)
-        try:
-            d = json.loads(out.stdout.strip().splitlines()[-1])
-            res[name] = {"cosmo": d["value"], "frac": d["roofline"]["frac"]}
-        except Exception as ex:
-            res[name] = {"error": str(ex), "stderr": out.stderr[-500:]}
+        res[name] = {}
+        if os.environ.get("VARIANT_COSMO", "1") == "1":
+            out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--secondary", "none", "--cpu-seconds", "0.5",
+                                  "--e2e-steps", "1", "--steps", "100"], env=env, capture_output=True, text=True)
+            try:
+                d = json.loads(out.stdout.strip().splitlines()[-1])
+                res[name] = {"cosmo": d["value"], "frac": d["roofline"]["frac"]}
+            except Exception as ex:
+                res[name] = {"error": str(ex), "stderr": out.stderr[-500:]}
         out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--workload", "deepcam", "--cpu-seconds", "0.5",
                               "--e2e-steps", "1", "--steps", "10"], env=env, capture_output=True, text=True)
         try:
