@@ -31,6 +31,18 @@ __device__ __forceinline__ uint2 ld_ro_u2(const void *p) {
     asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
     return r;
 }
+// L2 evict-last policy for small tables re-read by many CTAs (LUT rows) so the
+// output stream does not push them out of L2
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint2 ld_ro_u2_keep(const void *p, uint64_t pol) {
+    uint2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
 __device__ __forceinline__ float ld_ro_f32(const float *p) {
     float r;
     asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(p));
@@ -38,7 +50,7 @@ __device__ __forceinline__ float ld_ro_f32(const float *p) {
 }
 // write-once outputs (SPP_STORE_CS=1: streaming / evict-first, else default write-back)
 #ifndef SPP_STORE_CS
-#define SPP_STORE_CS 0
+#define SPP_STORE_CS 1
 #endif
 #if SPP_STORE_CS
 #define SPP_ST_POLICY ".cs"

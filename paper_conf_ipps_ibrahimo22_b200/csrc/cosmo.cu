@@ -46,8 +46,15 @@ struct CosmoMeta {  // written by KC0, read by KC
 };
 
 constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
-constexpr int kThreads = 256;
-constexpr int kHotBytes = 40 * 1024;  // shared-memory hot prefix of T per CTA
+#ifndef SPP_KC_THREADS
+#define SPP_KC_THREADS 384
+#endif
+#ifndef SPP_KC_HOT_KB
+#define SPP_KC_HOT_KB 80
+#endif
+constexpr int kThreads = SPP_KC_THREADS;
+constexpr int kMinBlocks = kThreads <= 256 ? 3 : (kThreads <= 384 ? 2 : 1);  // CTAs per SM the registers target
+constexpr int kHotBytes = SPP_KC_HOT_KB * 1024;  // shared-memory hot prefix of T per CTA
 constexpr int kUCap = 2048;           // unique values staged in shared memory (8 KB)
 constexpr int kKeyStages = 4;         // TMA ring of key tiles
 constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
@@ -314,6 +321,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     const uint32_t Gm1 = sv.G - 1;
     const uint32_t ntiles = (uint32_t)((b - a + kTileVox - 1) / kTileVox);
     const uint32_t lane = threadIdx.x & 31;
+    const uint64_t pol = l2_policy_evict_last();  // keep this sample's LUT in L2 against the output stream
     auto issue = [&](uint32_t t) {  // thread 0: bulk copy of tile t's keys once its stage is free
         const uint32_t gt = ring.count + t;
         const uint32_t stg = gt % kKeyStages;
@@ -344,11 +352,11 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
         if (cold) {
             j0 = __ffs(cold) - 1;
-            l0 = ld_ro_u2(sv.lut + 8ull * min(k.get_dyn(j0), Gm1));
+            l0 = ld_ro_u2_keep(sv.lut + 8ull * min(k.get_dyn(j0), Gm1), pol);
             cold &= cold - 1;
             if (cold) {
                 j1 = __ffs(cold) - 1;
-                l1 = ld_ro_u2(sv.lut + 8ull * min(k.get_dyn(j1), Gm1));
+                l1 = ld_ro_u2_keep(sv.lut + 8ull * min(k.get_dyn(j1), Gm1), pol);
             }
         }
     };
@@ -375,7 +383,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     bad |= g > Gm1;
                     const uint2 lv = (uint32_t)j == cj0 ? lv0
                                      : (uint32_t)j == cj1 ? lv1
-                                                          : ld_ro_u2(sv.lut + 8ull * min(g, Gm1));  // 3rd+ cold: rare
+                                                          : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // 3rd+ cold: rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }
             }
@@ -389,7 +397,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
 }
 
 template <int OUT, bool VEC>
-__global__ void __launch_bounds__(kThreads, 3) kc_expand(const void *const *__restrict__ src, int n,
+__global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *const *__restrict__ src, int n,
                                                          const float *__restrict__ fU_ws,
                                                          const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
                                                          int H, int W, uint64_t N, uint64_t chunk,
@@ -405,7 +413,7 @@ __global__ void __launch_bounds__(kThreads, 3) kc_expand(const void *const *__re
     if (VEC && threadIdx.x == 0) {
         for (int i = 0; i < kKeyStages; i++) {
             mbar_init(&ring.full[i], 1);
-            mbar_init(&ring.empty[i], kThreads / kWarp);
+            mbar_init(&ring.empty[i], kThreads / kWarp);  // one arrival per warp
         }
         fence_mbar_init();
     }

@@ -441,29 +441,35 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         const int s = act ? (int)(carry_seg + __popc(word & below) + flag) - 1 : 0;
         carry_seg += __popc(word);
         const SegInfo si = seg_info(desc, heads, s);
-        float pl[VPL];
-        if (act && si.kind == kDiff) {
-            Bytes<VPL> bt;
-            bt.load(dl_s + (uint32_t)(si.a + (int)p0));
-            if (flag) bt.w[0] &= 0xFFFFFF00u;  // the head has no delta byte
-            if constexpr (VPL == 8) {
-                if (W - p0 < 8) {  // positions past the line end (W % 256 != 0)
-                    const uint64_t m = (1ull << (8 * (W - p0))) - 1ull;
-                    bt.w[0] &= (uint32_t)m;
-                    bt.w[1] &= (uint32_t)(m >> 32);
-                }
+        // Every lane runs the same straight-line code.  Signed zeros make the
+        // special cases exact without branches: a REPEAT lane decodes delta
+        // bytes 0x80 (code -0) and a head or REPEAT lane uses dlt = -0, so
+        // S = -0 there and fma(-0, sc, h) == h bit for bit (also for h = +-0).
+        const bool rep = si.kind == kRepeat || !act;
+        Bytes<VPL> bt;
+        bt.load(dl_s + (uint32_t)(rep ? 0 : si.a + (int)p0));
+        if (rep) {
+#pragma unroll
+            for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;
+        }
+        if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
+        if constexpr (VPL == 8) {
+            if (act && W - p0 < 8) {  // positions past the line end (W % 256 != 0)
+                const uint64_t m = (1ull << (8 * (W - p0))) - 1ull;
+                bt.w[0] &= (uint32_t)m;
+                bt.w[1] &= (uint32_t)(m >> 32);
             }
+        }
+        float pl[VPL];
+        {
             float run = 0.f;
 #pragma unroll
             for (int k = 0; k < VPL / 4; k++) {
-                run += code_f<0>(bt.w[k]); pl[4 * k + 0] = run;
+                run = (k == 0 ? code_f<0>(bt.w[k]) : run + code_f<0>(bt.w[k])); pl[4 * k + 0] = run;
                 run += code_f<1>(bt.w[k]); pl[4 * k + 1] = run;
                 run += code_f<2>(bt.w[k]); pl[4 * k + 2] = run;
                 run += code_f<3>(bt.w[k]); pl[4 * k + 3] = run;
             }
-        } else {
-#pragma unroll
-            for (int j = 0; j < VPL; j++) pl[j] = 0.f;
         }
         // plain inclusive scan of lane totals; base = prefix before the head of
         // this lane's segment (its head lane in this chunk, else carried)
@@ -479,7 +485,7 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         const uint32_t mle = smask & le_mask;
         const float gotb = __shfl_sync(0xffffffffu, P_excl, mle ? 31 - __clz(mle) : lane);
         const float base = mle ? gotb : carry_base;
-        const float dlt = P_excl - base;
+        const float dlt = (flag || rep) ? -0.0f : P_excl - base;
         if constexpr (!STAGED) {
             carry_P += __shfl_sync(0xffffffffu, P, 31);
             const float topb = __shfl_sync(0xffffffffu, P_excl, smask ? 31 - __clz(smask) : 0);
@@ -487,24 +493,18 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         }
         if (!act) continue;
         float y[VPL];
-        if (si.kind == kRepeat) {
-            const float yr = __fmul_rn(__fsub_rn(si.h, shv), scv);
-#pragma unroll
-            for (int j = 0; j < VPL; j++) y[j] = yr;
-        } else if (!si.big) {
+        if (!si.big) {
 #pragma unroll
             for (int j = 0; j < VPL; j++) {
                 const float xh = __fmaf_rn(pl[j] + dlt, si.sc, si.h);  // RN(h + S * 2^emin), S exact
                 y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
             }
-            if (flag) y[0] = __fmul_rn(__fsub_rn(si.h, shv), scv);  // the head is exact
         } else {
 #pragma unroll
             for (int j = 0; j < VPL; j++) {
                 const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, si.sc, si.h);  // 2^(emin+30) scale
                 y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
             }
-            if (flag) y[0] = __fmul_rn(__fsub_rn(si.h, shv), scv);
         }
         if constexpr (STAGED) {
             __syncwarp();  // every lane has read its delta bytes and segment: reuse the slot for the row
@@ -606,7 +606,6 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     };
     auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {
         if constexpr (VPL == 36) bulk_wait_read_all();  // a staged row may still be leaving this slot
-        fence_proxy_async_smem();
         mbar_arrive_expect_tx(&mbar[slot], bytes);
         bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
     };
@@ -650,6 +649,7 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
                 const uint64_t sp = __shfl_sync(0xffffffffu, reinterpret_cast<uint64_t>(cur_src), 0);
                 const uint4 *src4 = reinterpret_cast<const uint4 *>(sp);
                 for (uint32_t k = lane; k < bytes / 16; k += kWarp) reinterpret_cast<uint4 *>(base)[k] = src4[k];
+                fence_proxy_async_smem();  // generic writes before later TMA writes to these slots
                 __syncwarp();
                 buf = base;
             } else if (slot == 0) {

@@ -10,8 +10,9 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kd_minb3": ["SPP_KD_MINB=3"],
-    "kd_minb2": ["SPP_KD_MINB=2"],
+    "kc384_hot80": ["SPP_KC_THREADS=384", "SPP_KC_HOT_KB=80"],
+    "kc512_hot176": ["SPP_KC_THREADS=512", "SPP_KC_HOT_KB=176"],
+    "kc768_hot160": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=160"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
