@@ -551,60 +551,50 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     }
     __syncwarp();
 
-    // line coordinates tracked incrementally (no divisions per line): decode
-    // position (s, l, y, c) and the lane-0 directory prefetch position (ps, pl)
+    // line coordinates tracked incrementally (no divisions per line)
     uint32_t s_cur = (uint32_t)(g_begin / L), l_cur = (uint32_t)(g_begin - (uint64_t)s_cur * L);
     uint32_t c_cur = l_cur / H, y_cur = l_cur - c_cur * H;
-    uint32_t ps = s_cur, pline = l_cur;
 
-    // lane-0 pipeline state
-    int64_t cs = -1;
-    DcMeta cm{nullptr, nullptr, 0, 0, 0};
-    uint32_t da = 0, db = 0;
-    const uint8_t *dpay = nullptr;
-    uint64_t dlim = 0;
-    uint32_t dvalid = 0, dalign = 0;
-    int64_t dsample = 0;
-    auto load_dir = [&]() {  // directory entry of line (ps, pline), then advance
-        if ((int64_t)ps != cs) {
-            cm = meta[ps];
-            cs = ps;
-        }
-        dvalid = cm.valid;
-        dalign = cm.align;
-        dpay = cm.payload;
-        dlim = cm.limit;
-        dsample = ps;
-        if (dvalid) {
-            const uint32_t *dir = reinterpret_cast<const uint32_t *>(cm.dir);
-            da = __ldg(dir + pline);
-            db = __ldg(dir + pline + 1);
-        }
-        if (++pline == L) {
-            pline = 0;
-            ps++;
+    // Directory window: lane k holds the validated directory entry of line
+    // wbase + k (source pointer, bytes, flags), loaded and checked by all lanes
+    // at once every 32 lines; per line the pipeline only shuffles one entry.
+    uint64_t wbase = 0;
+    uint64_t w_src = 0;
+    uint32_t w_bytes = 0, w_flags = 0;  // flags: bit 0 big, bits 16.. alignment
+    auto load_window = [&](uint64_t wb) {
+        wbase = wb;
+        const uint64_t g = wb + lane;
+        w_bytes = 0;
+        w_flags = 0;
+        w_src = 0;
+        if (g < g_end) {
+            const uint64_t sk = g / L;
+            const uint32_t lk = (uint32_t)(g - sk * L);
+            const DcMeta m = meta[sk];
+            if (m.valid) {
+                const uint32_t *dir = reinterpret_cast<const uint32_t *>(m.dir);
+                const uint32_t da = __ldg(dir + lk), db = __ldg(dir + lk + 1);
+                const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= m.limit && db - da >= 16;
+                if (!ok) {
+                    report(status, SPP_ERR_CORRUPT, (int64_t)sk);
+                } else if (db - da > big_cap) {
+                    report(status, SPP_ERR_UNSUPPORTED, (int64_t)sk);
+                } else {
+                    w_bytes = db - da;
+                    w_src = reinterpret_cast<uint64_t>(m.payload + da);
+                    w_flags = (w_bytes > cap_data ? 1u : 0u) | (m.align << 16);
+                }
+            }
         }
     };
-    // validate the loaded entry: bytes (0 = skip), big = needs both slots
-    auto prepare = [&](const uint8_t *&src, uint32_t &big, uint32_t &al) -> uint32_t {
-        big = 0;
-        al = dalign;
-        if (!dvalid) return 0;
-        const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= dlim && db - da >= 16;
-        if (!ok) {
-            report(status, SPP_ERR_CORRUPT, dsample);
-            return 0;
-        }
-        const uint32_t bytes = db - da;
-        if (bytes > big_cap) {
-            report(status, SPP_ERR_UNSUPPORTED, dsample);
-            return 0;
-        }
-        big = bytes > cap_data;
-        src = dpay + da;
-        return bytes;
+    // entry of line g (g in the current window), broadcast to all lanes
+    auto entry = [&](uint64_t g, const uint8_t *&src, uint32_t &bytes, uint32_t &flags) {
+        const int k = (int)(g - wbase);
+        src = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_src, k));
+        bytes = __shfl_sync(0xffffffffu, w_bytes, k);
+        flags = __shfl_sync(0xffffffffu, w_flags, k);
     };
-    auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {
+    auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {  // lane 0
         if constexpr (VPL == 36) bulk_wait_read_all();  // a staged row may still be leaving this slot
         mbar_arrive_expect_tx(&mbar[slot], bytes);
         bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
@@ -612,32 +602,28 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
 
     uint32_t c_cached = 0xFFFFFFFFu;
     float shv = 0.f, scv = 1.f;
-    uint32_t cur_bytes = 0, cur_big = 0, cur_al = 0, phase0 = 0, phase1 = 0;
-    const uint8_t *cur_src = nullptr;
+    uint32_t phase0 = 0, phase1 = 0;
     int slot = 0;
-    if (lane == 0) {
-        load_dir();
-        cur_bytes = prepare(cur_src, cur_big, cur_al);
-        if (cur_bytes && !cur_big) issue(0, cur_src, cur_bytes);
-        if (g_begin + 1 < g_end) load_dir();
-    }
+    load_window(g_begin);
+    const uint8_t *cur_src;
+    uint32_t cur_bytes, cur_flags;
+    entry(g_begin, cur_src, cur_bytes, cur_flags);
+    if (lane == 0 && cur_bytes && !(cur_flags & 1u)) issue(0, cur_src, cur_bytes);
     for (uint64_t g = g_begin; g < g_end; g++) {
-        uint32_t nxt_bytes = 0, nxt_big = 0, nxt_issued = 0, nxt_al = 0;
         const uint8_t *nxt_src = nullptr;
-        if (lane == 0) {
-            if (g + 1 < g_end) {
-                nxt_bytes = prepare(nxt_src, nxt_big, nxt_al);
-                // an oversize current line occupies both slots: issue the next later
-                if (nxt_bytes && !nxt_big && !cur_big) {
-                    issue(slot ^ 1, nxt_src, nxt_bytes);
-                    nxt_issued = 1;
-                }
+        uint32_t nxt_bytes = 0, nxt_flags = 0, nxt_issued = 0;
+        if (g + 1 < g_end) {
+            if (g + 1 >= wbase + kWarp) load_window(g + 1);
+            entry(g + 1, nxt_src, nxt_bytes, nxt_flags);
+            // an oversize current line occupies both slots: issue the next one later
+            if (nxt_bytes && !(nxt_flags & 1u) && !(cur_flags & 1u)) {
+                if (lane == 0) issue(slot ^ 1, nxt_src, nxt_bytes);
+                nxt_issued = 1;
             }
-            if (g + 2 < g_end) load_dir();
         }
-        const uint32_t bytes = __shfl_sync(0xffffffffu, cur_bytes, 0);
-        const uint32_t big = __shfl_sync(0xffffffffu, cur_big, 0);
-        const uint32_t al = __shfl_sync(0xffffffffu, cur_al, 0);
+        const uint32_t bytes = cur_bytes;
+        const uint32_t big = cur_flags & 1u;
+        const uint32_t al = cur_flags >> 16;
         if (bytes) {
             uint8_t *buf = base + slot * cap;
             if (big) {
@@ -646,8 +632,7 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
                     __syncwarp();
                 }
                 // stage across both slots with plain 16-B loads (rare: SEG line larger than RAW)
-                const uint64_t sp = __shfl_sync(0xffffffffu, reinterpret_cast<uint64_t>(cur_src), 0);
-                const uint4 *src4 = reinterpret_cast<const uint4 *>(sp);
+                const uint4 *src4 = reinterpret_cast<const uint4 *>(cur_src);
                 for (uint32_t k = lane; k < bytes / 16; k += kWarp) reinterpret_cast<uint4 *>(base)[k] = src4[k];
                 fence_proxy_async_smem();  // generic writes before later TMA writes to these slots
                 __syncwarp();
@@ -673,12 +658,11 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
             if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)s_cur);
         }
         __syncwarp();
-        if (lane == 0 && nxt_bytes && !nxt_big && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
+        if (lane == 0 && nxt_bytes && !(nxt_flags & 1u) && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
         slot ^= 1;
         cur_bytes = nxt_bytes;
-        cur_big = nxt_big;
+        cur_flags = nxt_flags;
         cur_src = nxt_src;
-        cur_al = nxt_al;
         if (++y_cur == H) {
             y_cur = 0;
             c_cur++;
