@@ -10,11 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc768_hot160": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=160"],
-    "kc768_hot168": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=168"],
-    "kc768_hot176_s3": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=176", "SPP_KC_STAGES=3"],
-    "kc1024_hot160_s3": ["SPP_KC_THREADS=1024", "SPP_KC_HOT_KB=160", "SPP_KC_STAGES=3"],
-    "kc640_hot176": ["SPP_KC_THREADS=640", "SPP_KC_HOT_KB=176"],
+    "kc768_hot168_s4": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=168", "SPP_KC_STAGES=4"],
+    "kc768_hot152_s5": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=152", "SPP_KC_STAGES=5"],
+    "kc768_hot136_s6": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=136", "SPP_KC_STAGES=6"],
+    "kc768_hot112_s8": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=112", "SPP_KC_STAGES=8"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
