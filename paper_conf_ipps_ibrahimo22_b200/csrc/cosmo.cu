@@ -50,14 +50,14 @@ constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 #define SPP_KC_THREADS 768
 #endif
 #ifndef SPP_KC_HOT_KB
-#define SPP_KC_HOT_KB 160
+#define SPP_KC_HOT_KB 152
 #endif
 constexpr int kThreads = SPP_KC_THREADS;
 constexpr int kMinBlocks = kThreads <= 256 ? 3 : (kThreads <= 384 ? 2 : 1);  // CTAs per SM the registers target
 constexpr int kHotBytes = SPP_KC_HOT_KB * 1024;  // shared-memory hot prefix of T per CTA
 constexpr int kUCap = 2048;           // unique values staged in shared memory (8 KB)
 #ifndef SPP_KC_STAGES
-#define SPP_KC_STAGES 4
+#define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
