@@ -521,6 +521,105 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
     return true;
 }
 
+// One-pass decode of a W = 32*36 line with at most 32 segments (the common
+// case): lane s holds segment s's table entry in registers; the head lanes form
+// one bitmap word (one warp OR-reduction) and every lane fetches its segment's
+// parameters by shuffle.  Falls back to the shared-memory tables otherwise.
+template <int OUT>
+__device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
+                                                    uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
+    constexpr int VPL = 36;
+    const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
+    const uint32_t nseg = hdr >> 16;
+    if (nseg > (uint32_t)kWarp) return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, lane);
+    if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
+    const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
+    const bool have = (uint32_t)lane < nseg;
+    uint32_t len = 0, kind = 0, eb = 0;
+    float hs = 0.f;
+    if (have) {
+        const uint32_t d = reinterpret_cast<const uint32_t *>(buf + 4)[lane];
+        len = d & 0xFFFFu;
+        kind = (d >> 16) & 0xFFu;
+        eb = d >> 24;
+        hs = reinterpret_cast<const float *>(buf + 4 + 4 * nseg)[lane];
+    }
+    const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
+    const uint32_t pk = len | (dlen << 16);
+    const uint32_t inc = warp_incl_scan(pk, lane);
+    const uint32_t ex = inc - pk;
+    const uint32_t st = ex & 0xFFFFu, db = ex >> 16;
+    const uint32_t blk = st / VPL;
+    bool bad = have && (len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
+                        st + len > W || blk * VPL != st);
+    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+    bad = __any_sync(0xffffffffu, bad) || (tot & 0xFFFFu) != W || 4u + 8u * nseg + (tot >> 16) > bytes;
+    if (bad) return false;
+    const uint32_t word = __reduce_or_sync(0xffffffffu, have ? 1u << blk : 0u);  // head lanes
+    const uint32_t info = (uint32_t)((int)db - (int)st - 1 + 16384) | (kind << 16) | (eb << 24);
+
+    const uint32_t le_mask = 0xFFFFFFFFu >> (31 - lane);
+    const uint32_t p0 = VPL * lane;
+    const uint32_t flag = (word >> lane) & 1u;
+    const int s = __popc(word & le_mask) - 1;  // segment of this lane (position 0 is always a head)
+    const uint32_t d = __shfl_sync(0xffffffffu, info, s);
+    const float h = __shfl_sync(0xffffffffu, hs, s);
+    const int a = (int)(d & 0xFFFFu) - 16384;
+    const uint32_t skind = (d >> 16) & 0xFFu, seb = d >> 24;
+    const bool big = seb >= 148u;
+    const float sc = __uint_as_float((big ? (seb + 7u) : (seb + 107u)) << 23);
+    const bool rep = skind == kRepeat;
+    Bytes<VPL> bt;
+    bt.load(dl_s + (uint32_t)(rep ? 0 : a + (int)p0));
+    if (rep) {
+#pragma unroll
+        for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;  // code -0: S = -0 keeps h exact
+    }
+    if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
+    float pl[VPL];
+    {
+        float run = 0.f;
+#pragma unroll
+        for (int k = 0; k < VPL / 4; k++) {
+            run = (k == 0 ? code_f<0>(bt.w[k]) : run + code_f<0>(bt.w[k])); pl[4 * k + 0] = run;
+            run += code_f<1>(bt.w[k]); pl[4 * k + 1] = run;
+            run += code_f<2>(bt.w[k]); pl[4 * k + 2] = run;
+            run += code_f<3>(bt.w[k]); pl[4 * k + 3] = run;
+        }
+    }
+    const float lt = pl[VPL - 1];
+    float P = lt;
+#pragma unroll
+    for (int dd = 1; dd < kWarp; dd <<= 1) {
+        const float y = __shfl_up_sync(0xffffffffu, P, dd);
+        if (lane >= dd) P += y;
+    }
+    const float P_excl = P - lt;
+    const uint32_t mle = word & le_mask;
+    const float base = __shfl_sync(0xffffffffu, P_excl, 31 - __clz(mle));
+    const float dlt = (flag || rep) ? -0.0f : P_excl - base;
+    float y[VPL];
+    if (!big) {
+#pragma unroll
+        for (int j = 0; j < VPL; j++) {
+            const float xh = __fmaf_rn(pl[j] + dlt, sc, h);  // RN(h + S * 2^emin), S exact
+            y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < VPL; j++) {
+            const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, sc, h);
+            y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+        }
+    }
+    __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
+    stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+    fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
+    __syncwarp();
+    if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+    return true;
+}
+
 template <int OUT, bool VEC, int VPL>
 __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decode(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
@@ -651,8 +750,10 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
             }
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg))
-                ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
+                if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            }
             else
                 ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
             if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)s_cur);
