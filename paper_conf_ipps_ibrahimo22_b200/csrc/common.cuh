@@ -38,6 +38,11 @@ __device__ __forceinline__ uint64_t l2_policy_evict_last() {
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
+// TMA prefetch of a global range into L2 (no shared memory, no completion)
+__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes, uint64_t pol) {
+    asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes), "l"(pol)
+                 : "memory");
+}
 __device__ __forceinline__ uint2 ld_ro_u2_keep(const void *p, uint64_t pol) {
     uint2 r;
     asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
@@ -147,6 +152,24 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 // order prior generic-proxy smem accesses before later async-proxy (TMA) writes
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ---- packed fp32 pairs (sm_100: FADD2 / FFMA2 / FMUL2), IEEE RN, no FTZ ---------
+union F2U { float2 f; unsigned long long u; };
+__device__ __forceinline__ float2 fadd2_rn(float2 a, float2 b) {
+    F2U x{a}, y{b}, r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r.u) : "l"(x.u), "l"(y.u));
+    return r.f;
+}
+__device__ __forceinline__ float2 fmul2_rn(float2 a, float2 b) {
+    F2U x{a}, y{b}, r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r.u) : "l"(x.u), "l"(y.u));
+    return r.f;
+}
+__device__ __forceinline__ float2 ffma2_rn(float2 a, float2 b, float2 c) {
+    F2U x{a}, y{b}, z{c}, r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r.u) : "l"(x.u), "l"(y.u), "l"(z.u));
+    return r.f;
 }
 
 // ---- warp scans --------------------------------------------------------------

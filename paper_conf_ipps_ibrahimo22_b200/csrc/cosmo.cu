@@ -53,6 +53,7 @@ constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 #define SPP_KC_HOT_KB 152
 #endif
 constexpr int kThreads = SPP_KC_THREADS;
+constexpr int kPrologueThreads = 256;
 constexpr int kMinBlocks = kThreads <= 256 ? 3 : (kThreads <= 384 ? 2 : 1);  // CTAs per SM the registers target
 constexpr int kHotBytes = SPP_KC_HOT_KB * 1024;  // shared-memory hot prefix of T per CTA
 constexpr int kUCap = 2048;           // unique values staged in shared memory (8 KB)
@@ -60,6 +61,9 @@ constexpr int kUCap = 2048;           // unique values staged in shared memory (
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
+#ifndef SPP_KC_PREFETCH_TAIL
+#define SPP_KC_PREFETCH_TAIL 1
+#endif
 constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
 constexpr int kStageBytes = kTileVox * 2;
 constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + 2 * kKeyStages * 8;
@@ -68,7 +72,7 @@ size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(flo
 
 // --------------------------------------------------------------------------
 // KC0: header/slab validation and the unique-value transform
-__global__ void __launch_bounds__(kThreads) kc0_prologue(const void *const *__restrict__ src,
+__global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *const *__restrict__ src,
                                                          const uint64_t *__restrict__ src_bytes, int transform,
                                                          int D, int H, int W, float *__restrict__ fU_ws,
                                                          CosmoMeta *__restrict__ meta,
@@ -449,8 +453,19 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
             if (a >= e) continue;
             if (sv.kw == 1 || sv.kw == 2) {
                 if (cached_s != s || cached_t != (int)t) {
-                    // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples
+                    // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples;
+                    // the LUT tail (cold groups) is prefetched into L2 for the cold lookups
                     __syncthreads();
+#if SPP_KC_PREFETCH_TAIL
+                    if (threadIdx.x == 0 && sv.G > hot_cap) {
+                        const uint64_t off = 8ull * hot_cap, end = 8ull * sv.G;
+                        const uint64_t pol = l2_policy_evict_last();
+                        for (uint64_t o = off & ~15ull; o < end; o += 65536) {
+                            const uint64_t nb = end - o < 65536 ? ((end - o + 15) & ~15ull) : 65536;
+                            prefetch_l2(sv.lut + o, (uint32_t)nb, pol);
+                        }
+                    }
+#endif
                     if (cached_s != s && fu.in_smem)
                         for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
                     __syncthreads();
@@ -567,7 +582,7 @@ spp_status cosmo_decode(const void *const *d_src, int n, void *d_dst, const spp_
     CosmoMeta *meta = reinterpret_cast<CosmoMeta *>(ws + meta_offset(n));
     cudaEvent_t const *ev = reinterpret_cast<cudaEvent_t const *>(o.timing_events);
     if (ev && cudaEventRecord(ev[0], stream) != cudaSuccess) return SPP_ERR_CUDA;
-    kc0_prologue<<<n, kThreads, 0, stream>>>(d_src, o.src_bytes, o.transform, o.D, o.H, o.W, fU, meta, o.status);
+    kc0_prologue<<<n, kPrologueThreads, 0, stream>>>(d_src, o.src_bytes, o.transform, o.D, o.H, o.W, fU, meta, o.status);
     if (cudaGetLastError() != cudaSuccess) return SPP_ERR_CUDA;
     if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
     spp_status r = cosmo_expand(d_src, n, d_dst, o, stream, dp, fU, meta);

@@ -598,17 +598,24 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const uint32_t mle = word & le_mask;
     const float base = __shfl_sync(0xffffffffu, P_excl, 31 - __clz(mle));
     const float dlt = (flag || rep) ? -0.0f : P_excl - base;
+    // x̂ = RN(h + S * 2^emin) and y = RN(RN(x̂ - shift) * scale), two values per
+    // instruction (FADD2/FFMA2/FMUL2 round exactly like the scalar forms)
+    const float2 dl2 = make_float2(dlt, dlt), h2 = make_float2(h, h), nsh2 = make_float2(-shv, -shv),
+                 scv2 = make_float2(scv, scv);
+    const float2 sc2 = make_float2(sc, sc);
     float y[VPL];
     if (!big) {
 #pragma unroll
-        for (int j = 0; j < VPL; j++) {
-            const float xh = __fmaf_rn(pl[j] + dlt, sc, h);  // RN(h + S * 2^emin), S exact
-            y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+        for (int j = 0; j < VPL; j += 2) {
+            const float2 S = fadd2_rn(make_float2(pl[j], pl[j + 1]), dl2);  // exact
+            const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
+            y[j] = y2.x;
+            y[j + 1] = y2.y;
         }
     } else {
 #pragma unroll
         for (int j = 0; j < VPL; j++) {
-            const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, sc, h);
+            const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, sc, h);  // 2^(emin+30) scale
             y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
         }
     }

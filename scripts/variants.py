@@ -10,10 +10,9 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc768_hot168_s4": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=168", "SPP_KC_STAGES=4"],
-    "kc768_hot152_s5": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=152", "SPP_KC_STAGES=5"],
-    "kc768_hot136_s6": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=136", "SPP_KC_STAGES=6"],
-    "kc768_hot112_s8": ["SPP_KC_THREADS=768", "SPP_KC_HOT_KB=112", "SPP_KC_STAGES=8"],
+    "kc_pf0": ["SPP_KC_PREFETCH_TAIL=0"],
+    "kc_pf1": ["SPP_KC_PREFETCH_TAIL=1"],
+    "kc_pf1_hot144_s6": ["SPP_KC_PREFETCH_TAIL=1", "SPP_KC_HOT_KB=144", "SPP_KC_STAGES=6"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
