@@ -172,6 +172,7 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
 
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
+    l2_granted = spp.spp_set_l2_persisting(int(args.l2_persist_mb * 2**20)) if args.l2_persist_mb > 0 else 0
     W = WORKLOADS[args.workload]
     B = args.batch or W["batch"]
     dims = W["dims"]
@@ -292,6 +293,7 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
         "gpu_launches": spp.spp_decode_launches(args.workload) * args.steps,
         "clocks": clk.summary(),
         "batch": B, "in_bytes": in_bytes, "out_bytes": out_bytes, "pool": P, "setup_s": setup_s,
+        "l2_persist_bytes": l2_granted,
         "compression_ratio": float(np.prod(dims)) * (2 if args.workload == "cosmo" else 4) * P / sum(sizes),
     }
     del out, src_all
@@ -313,6 +315,8 @@ def main():
     ap.add_argument("--chunk", type=int, default=16, help="samples per H2D chunk in the e2e pipeline")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--l2-persist-mb", type=float, default=float(os.environ.get("SPP_L2_PERSIST_MB", "0")),
+                    help="L2 persisting set-aside for the CosmoFlow LUT rows (spp_set_l2_persisting)")
     args = ap.parse_args()
     if args.steps is None:
         args.steps = 200 if args.workload == "cosmo" else 30

@@ -165,6 +165,13 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
 /* Number of decode launches and copies the last spp_decode_host call enqueued. */
 int spp_pipeline_last_launches(const spp_pipeline *p);
 
+/* Optional performance hint (device-wide, opt-in): reserve `bytes` of L2 as the
+ * persisting set-aside (cudaLimitPersistingL2CacheSize) so that the CosmoFlow
+ * LUT rows, which the decoder reads with an L2 evict-last policy, survive the
+ * output stream.  0 releases the set-aside.  Affects the whole current device;
+ * the granted size is returned in *granted (may be clamped by the driver). */
+spp_status spp_set_l2_persisting(size_t bytes, size_t *granted);
+
 const char *spp_status_string(spp_status s);
 
 /* Library build identification: "spp <version> sm_100a". */

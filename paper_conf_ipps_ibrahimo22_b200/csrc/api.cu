@@ -147,6 +147,18 @@ spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, in
     return SPP_ERR_INVALID_ARG;
 }
 
+spp_status spp_set_l2_persisting(size_t bytes, size_t *granted) {
+    int dev = 0, maxp = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return SPP_ERR_CUDA;
+    if (cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess) return SPP_ERR_CUDA;
+    const size_t want = bytes < (size_t)maxp ? bytes : (size_t)maxp;
+    if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) != cudaSuccess) return SPP_ERR_CUDA;
+    size_t got = 0;
+    if (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) != cudaSuccess) return SPP_ERR_CUDA;
+    if (granted) *granted = got;
+    return SPP_OK;
+}
+
 const char *spp_status_string(spp_status s) {
     switch (s) {
         case SPP_OK: return "ok";

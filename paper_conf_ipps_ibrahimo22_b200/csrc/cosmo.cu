@@ -56,11 +56,15 @@ constexpr int kThreads = SPP_KC_THREADS;
 constexpr int kPrologueThreads = 256;
 constexpr int kMinBlocks = kThreads <= 256 ? 3 : (kThreads <= 384 ? 2 : 1);  // CTAs per SM the registers target
 constexpr int kHotBytes = SPP_KC_HOT_KB * 1024;  // shared-memory hot prefix of T per CTA
-constexpr int kUCap = 2048;           // unique values staged in shared memory (8 KB)
+constexpr int kUCap = 2048;           // part of the region nominally for f(U) (8 KB)
+constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot tuples
 #ifndef SPP_KC_STAGES
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
+#ifndef SPP_KC_DIAG_NOCOLD
+#define SPP_KC_DIAG_NOCOLD 0
+#endif
 #ifndef SPP_KC_PREFETCH_TAIL
 #define SPP_KC_PREFETCH_TAIL 1
 #endif
@@ -357,6 +361,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         uint32_t cold = 0;
 #pragma unroll
         for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
+#if SPP_KC_DIAG_NOCOLD
+        cold = 0;
+#endif
         if (cold) {
             j0 = __ffs(cold) - 1;
             l0 = ld_ro_u2_keep(sv.lut + 8ull * min(k.get_dyn(j0), Gm1), pol);
@@ -383,7 +390,11 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             E e[8];
 #pragma unroll
             for (int j = 0; j < 8; j++) {
+#if SPP_KC_DIAG_NOCOLD  // timing diagnostic only (wrong output): every key treated as hot
+                const uint32_t g = k0.get(j) % n_hot;
+#else
                 const uint32_t g = k0.get(j);
+#endif
                 if (g < n_hot) {
                     e[j] = lds_entry<OUT>(hot_base + g * EB);
                 } else {
@@ -413,8 +424,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     using E = typename Entry<OUT>::T;
     constexpr uint32_t EB = sizeof(E);
     extern __shared__ __align__(16) uint8_t smem_raw[];
-    const uint32_t hot_base = smem_u32(smem_raw);
-    const uint32_t fu_base = hot_base + kHotBytes;
+    const uint32_t region = smem_u32(smem_raw);
+    const uint32_t fu_base = region;  // f(U) at the start of the region, hot tuples after it
+    uint32_t hot_base = region;
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes);
     KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0};
     if (VEC && threadIdx.x == 0) {
@@ -441,7 +453,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
         const CosmoMeta m = meta[s];
         if (!m.valid) continue;
         const uint8_t *b = static_cast<const uint8_t *>(src[s]);
-        const FuView fu{fu_base, fU_ws + (size_t)s * kFuStride, m.nU, m.nU <= (uint32_t)kUCap};
+        // f(U) lives in shared memory unless |U| would take more than half the region
+        const FuView fu{fu_base, fU_ws + (size_t)s * kFuStride, m.nU, 4u * m.nU <= (uint32_t)kRegionBytes / 2};
         const FuView fu_g{fu_base, fu.global, m.nU, false};
         uint8_t *out_s = dst + (uint64_t)s * 4 * N * ob;
         uint32_t bad = 0;  // corrupt key / index seen by this thread in this item
@@ -457,7 +470,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     // the LUT tail (cold groups) is prefetched into L2 for the cold lookups
                     __syncthreads();
 #if SPP_KC_PREFETCH_TAIL
-                    if (threadIdx.x == 0 && sv.G > hot_cap) {
+                    if (threadIdx.x == 0 && sv.G > hot_cap) {  // (hot_cap: nominal prefix size)
                         const uint64_t off = 8ull * hot_cap, end = 8ull * sv.G;
                         const uint64_t pol = l2_policy_evict_last();
                         for (uint64_t o = off & ~15ull; o < end; o += 65536) {
@@ -469,7 +482,14 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     if (cached_s != s && fu.in_smem)
                         for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
                     __syncthreads();
-                    n_hot = min(sv.G, hot_cap);
+                    const uint32_t fu_bytes = fu.in_smem ? (4u * m.nU + 15u) & ~15u : 0u;
+                    hot_base = region + fu_bytes;
+                    // hot prefix: as many tuples as fit, but not more than this CTA's
+                    // voxels of the slab can amortise (multi-slab samples)
+                    const uint64_t cta_end = v0 + (i1 - it) * chunk;  // this CTA's remaining voxels of the sample
+                    const uint64_t span = (sb < cta_end ? sb : cta_end) - a;
+                    const uint32_t amort = span / 8 > 4096 ? (uint32_t)min(span / 8, (uint64_t)0xFFFFFFFFu) : 4096u;
+                    n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes) / EB), amort);
 #pragma unroll 1
                     for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * blockDim.x) {
                         uint2 lv[4];
@@ -514,6 +534,34 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                         store8<OUT>(out_s, N, q, e8);
                 } else {
                     for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) store1<OUT>(out_s, N, v, en);
+                }
+            } else if (VEC && fu.in_smem) {
+                // RAW escape slab: four planes of U indices (FORMAT.md 1.1, kw = 8), 8 voxels per thread
+                if (cached_s != s) {
+                    __syncthreads();
+                    for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
+                    __syncthreads();
+                    cached_s = s;
+                    cached_t = -1;
+                }
+                const uint64_t Nt = sb - sa;
+                for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)blockDim.x * 8) {
+                    const uint64_t rel = q - sa;
+                    uint4 pc[4];
+#pragma unroll
+                    for (int c = 0; c < 4; c++) pc[c] = ld_stream_u4(sv.keys + 2 * ((uint64_t)c * Nt + rel));
+                    E e8[8];
+#pragma unroll
+                    for (int j = 0; j < 8; j++) {
+                        uint32_t w[4];
+#pragma unroll
+                        for (int c = 0; c < 4; c++) {
+                            const uint32_t ww = (j >> 1) == 0 ? pc[c].x : (j >> 1) == 1 ? pc[c].y : (j >> 1) == 2 ? pc[c].z : pc[c].w;
+                            w[c] = (j & 1) ? ww >> 16 : ww & 0xFFFFu;
+                        }
+                        e8[j] = make_entry<OUT, true>(make_uint2(w[0] | (w[1] << 16), w[2] | (w[3] << 16)), fu, bad);
+                    }
+                    store8<OUT>(out_s, N, q, e8);
                 }
             } else {
                 // RAW escape slab: four planes of U indices (FORMAT.md 1.1, kw = 8)

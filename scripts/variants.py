@@ -10,9 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_pf0": ["SPP_KC_PREFETCH_TAIL=0"],
-    "kc_pf1": ["SPP_KC_PREFETCH_TAIL=1"],
-    "kc_pf1_hot144_s6": ["SPP_KC_PREFETCH_TAIL=1", "SPP_KC_HOT_KB=144", "SPP_KC_STAGES=6"],
+    "kc_base": [],
+    "kc_base@32": [],
+    "kc_base@64": [],
+    "kc_base@96": [],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
@@ -21,7 +22,7 @@ def build():
     from paper_conf_ipps_ibrahimo22_b200 import build as b
     OUT.mkdir(exist_ok=True)
     for name, d in VARIANTS.items():
-        b.build(force=True, defines=d, out=OUT / f"libspp_{name}.so")
+        b.build(force=True, defines=d, out=OUT / f"libspp_{name}.so")  # noqa
         print("built", name)
 
 
@@ -29,6 +30,8 @@ def run():
     res = {}
     for name in VARIANTS:
         env = dict(os.environ, SPP_LIB=str(OUT / f"libspp_{name}.so"))
+        if "@" in name:
+            env["SPP_L2_PERSIST_MB"] = name.split("@")[1]
         res[name] = {}
         if os.environ.get("VARIANT_COSMO", "1") == "1":
             out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--secondary", "none", "--cpu-seconds", "0.5",
