@@ -50,7 +50,7 @@ constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 #define SPP_KC_THREADS 768
 #endif
 #ifndef SPP_KC_HOT_KB
-#define SPP_KC_HOT_KB 152
+#define SPP_KC_HOT_KB 120
 #endif
 constexpr int kThreads = SPP_KC_THREADS;
 constexpr int kPrologueThreads = 256;
@@ -70,7 +70,12 @@ constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 #endif
 constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
 constexpr int kStageBytes = kTileVox * 2;
-constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + 2 * kKeyStages * 8;
+#ifndef SPP_KC_LA
+#define SPP_KC_LA 2
+#endif
+constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
+constexpr int kColdSlotBytes = (kColdLA + 1) * kThreads * 16;  // 2 rows per thread per tile in flight
+constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes + 2 * kKeyStages * 8;
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
 
@@ -295,8 +300,9 @@ struct Keys8 {
 struct KeyRing {
     uint8_t *buf;      // kKeyStages * kStageBytes
     uint64_t *full;    // kKeyStages, completed by the TMA transaction count
-    uint64_t *empty;   // kKeyStages, 8 warp arrivals
+    uint64_t *empty;   // kKeyStages, one arrival per warp
     uint32_t count;
+    uint32_t cold;     // shared address of the per-thread cold-row slots
 };
 
 __device__ __forceinline__ Keys8 keys_from_smem(const uint8_t *stage, uint32_t kwb) {
@@ -350,39 +356,67 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         mbar_wait(&ring.full[gt % kKeyStages], (gt / kKeyStages) & 1u);
         return ring.buf + (gt % kKeyStages) * kStageBytes;
     };
-    // cold lookahead state for the tile about to be expanded: up to two cold
-    // positions (j) with their LUT rows in flight
-    uint32_t cj0 = 8, cj1 = 8;
-    uint2 lv0 = make_uint2(0, 0), lv1 = make_uint2(0, 0);
-    auto classify = [&](const uint8_t *stage, uint64_t q, uint32_t &j0, uint32_t &j1, uint2 &l0, uint2 &l1) {
-        j0 = j1 = 8;
-        if (q >= b) return;
-        const Keys8 k = keys_from_smem(stage, kwb);
-        uint32_t cold = 0;
+    // Cold rows: while tile t is expanded, the thread classifies its keys of
+    // tile t + kColdLA and starts LDGSTS copies (cp.async) of up to two cold LUT
+    // rows into its own shared-memory slots; one copy group per tile, so the
+    // rows of tile t are waited for (per thread, no barrier) kColdLA tiles later.
+    // cj[t % (kColdLA+1)] = (j0 | j1 << 8) cold positions of that tile (8 = none).
+    uint32_t cj[kColdLA + 1];
 #pragma unroll
-        for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
+    for (int i = 0; i <= kColdLA; i++) cj[i] = 0x0808u;
+    auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k (0/1) of this thread for tile t
+        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kThreads + threadIdx.x) * 2 + k) * 8;
+    };
+    auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
+        const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
+        uint32_t j0 = 8, j1 = 8;
+        if (q < b) {
+            const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
+            const Keys8 k = keys_from_smem(stage, kwb);
+            uint32_t cold = 0;
+#pragma unroll
+            for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
 #if SPP_KC_DIAG_NOCOLD
-        cold = 0;
+            cold = 0;
 #endif
-        if (cold) {
-            j0 = __ffs(cold) - 1;
-            l0 = ld_ro_u2_keep(sv.lut + 8ull * min(k.get_dyn(j0), Gm1), pol);
-            cold &= cold - 1;
             if (cold) {
-                j1 = __ffs(cold) - 1;
-                l1 = ld_ro_u2_keep(sv.lut + 8ull * min(k.get_dyn(j1), Gm1), pol);
+                j0 = __ffs(cold) - 1;
+                cp_async8(slot_addr(t, 0), sv.lut + 8ull * min(k.get_dyn(j0), Gm1));
+                cold &= cold - 1;
+                if (cold) {
+                    j1 = __ffs(cold) - 1;
+                    cp_async8(slot_addr(t, 1), sv.lut + 8ull * min(k.get_dyn(j1), Gm1));
+                }
             }
         }
+        cp_async_commit();
+        return j0 | (j1 << 8);
     };
     if (threadIdx.x == 0)
         for (uint32_t t = 0; t < ntiles && t < (uint32_t)(kKeyStages - 1); t++) issue(t);
-    if (ntiles) classify(wait_full(0), a + 8u * threadIdx.x, cj0, cj1, lv0, lv1);
+#pragma unroll
+    for (int i = 0; i < kColdLA; i++) {
+        if ((uint32_t)i < ntiles) {
+            wait_full(i);
+            cj[i] = classify(i);
+        } else {
+            cp_async_commit();
+        }
+    }
 #pragma unroll 1
     for (uint32_t t = 0; t < ntiles; t++) {
         if (threadIdx.x == 0 && t + kKeyStages - 1 < ntiles) issue(t + kKeyStages - 1);
-        uint32_t nj0 = 8, nj1 = 8;
-        uint2 nl0 = make_uint2(0, 0), nl1 = make_uint2(0, 0);
-        if (t + 1 < ntiles) classify(wait_full(t + 1), a + (uint64_t)(t + 1) * kTileVox + 8u * threadIdx.x, nj0, nj1, nl0, nl1);
+        if (t + kColdLA < ntiles) {
+            wait_full(t + kColdLA);
+            cj[kColdLA] = classify(t + kColdLA);
+        } else {
+            cp_async_commit();  // keep one group per iteration
+        }
+        cp_async_wait<kColdLA>();  // the copies of tile t have landed (this thread's)
+        const uint32_t cjt = cj[0];
+#pragma unroll
+        for (int i = 0; i < kColdLA; i++) cj[i] = cj[i + 1];  // rotate (compile-time indices)
+        const uint32_t cj0 = cjt & 0xFFu, cj1 = cjt >> 8;
         const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         if (q < b) {
@@ -399,9 +433,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     e[j] = lds_entry<OUT>(hot_base + g * EB);
                 } else {
                     bad |= g > Gm1;
-                    const uint2 lv = (uint32_t)j == cj0 ? lv0
-                                     : (uint32_t)j == cj1 ? lv1
-                                                          : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // 3rd+ cold: rare
+                    const uint2 lv = (uint32_t)j == cj0 ? lds_u2(slot_addr(t, 0))
+                                     : (uint32_t)j == cj1 ? lds_u2(slot_addr(t, 1))
+                                                          : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // 3rd+: rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }
             }
@@ -409,8 +443,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);  // this warp is done with the stage
-        cj0 = nj0; cj1 = nj1; lv0 = nl0; lv1 = nl1;
     }
+    cp_async_wait<0>();
     ring.count += ntiles;
 }
 
@@ -427,8 +461,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     const uint32_t region = smem_u32(smem_raw);
     const uint32_t fu_base = region;  // f(U) at the start of the region, hot tuples after it
     uint32_t hot_base = region;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes);
-    KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0};
+    uint64_t *bars =
+        reinterpret_cast<uint64_t *>(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes);
+    KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0,
+                 smem_u32(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes)};
     if (VEC && threadIdx.x == 0) {
         for (int i = 0; i < kKeyStages; i++) {
             mbar_init(&ring.full[i], 1);

@@ -10,10 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_base": [],
-    "kc_base@32": [],
-    "kc_base@64": [],
-    "kc_base@96": [],
+    "kc_la1_hot136": ["SPP_KC_LA=1", "SPP_KC_HOT_KB=136"],
+    "kc_la2_hot120": ["SPP_KC_LA=2", "SPP_KC_HOT_KB=120"],
+    "kc_la3_hot108": ["SPP_KC_LA=3", "SPP_KC_HOT_KB=108"],
+    "kc_la2_hot128_s4": ["SPP_KC_LA=2", "SPP_KC_HOT_KB=128", "SPP_KC_STAGES=4"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
