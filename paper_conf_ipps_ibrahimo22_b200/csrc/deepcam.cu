@@ -89,6 +89,13 @@ __device__ __forceinline__ float code_f(uint32_t w) {
     else r = (w & 0x80000000u) | ((w >> 5) & 0x03F80000u);
     return __uint_as_float(r);
 }
+// same value, arithmetic-shift form: byte K moved to the top, sign-extending
+// shift by 5, then one mask keeps bit 31 (sign) and bits 19..25 (E|M)
+template <int K>
+__device__ __forceinline__ float code_f_sar(uint32_t w) {
+    const int32_t t = (int32_t)(w << (24 - 8 * K));
+    return __uint_as_float((uint32_t)(t >> 5) & 0x83F80000u);
+}
 __device__ __forceinline__ float code_f_byte(uint32_t b) {
     return __uint_as_float(((b & 0x80u) << 24) | ((b & 0x7Fu) << 19));
 }
@@ -576,18 +583,23 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
         for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;  // code -0: S = -0 keeps h exact
     }
     if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
-    float pl[VPL];
-    {
-        float run = 0.f;
+    // codes of the lane's 36 positions, then the lane prefix on pairs
+    // (position i, position i + 18) with FADD2: both halves at once (exact)
+    constexpr int HALF = VPL / 2;
+    float f[VPL];
 #pragma unroll
-        for (int k = 0; k < VPL / 4; k++) {
-            run = (k == 0 ? code_f<0>(bt.w[k]) : run + code_f<0>(bt.w[k])); pl[4 * k + 0] = run;
-            run += code_f<1>(bt.w[k]); pl[4 * k + 1] = run;
-            run += code_f<2>(bt.w[k]); pl[4 * k + 2] = run;
-            run += code_f<3>(bt.w[k]); pl[4 * k + 3] = run;
-        }
+    for (int k = 0; k < VPL / 4; k++) {
+        f[4 * k + 0] = code_f_sar<0>(bt.w[k]);
+        f[4 * k + 1] = code_f_sar<1>(bt.w[k]);
+        f[4 * k + 2] = code_f_sar<2>(bt.w[k]);
+        f[4 * k + 3] = code_f_sar<3>(bt.w[k]);
     }
-    const float lt = pl[VPL - 1];
+    float2 pp[HALF];
+    pp[0] = make_float2(f[0], f[HALF]);
+#pragma unroll
+    for (int i = 1; i < HALF; i++) pp[i] = fadd2_rn(pp[i - 1], make_float2(f[i], f[HALF + i]));
+    const float totA = pp[HALF - 1].x;
+    const float lt = totA + pp[HALF - 1].y;  // lane total
     float P = lt;
 #pragma unroll
     for (int dd = 1; dd < kWarp; dd <<= 1) {
@@ -600,23 +612,24 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const float dlt = (flag || rep) ? -0.0f : P_excl - base;
     // x̂ = RN(h + S * 2^emin) and y = RN(RN(x̂ - shift) * scale), two values per
     // instruction (FADD2/FFMA2/FMUL2 round exactly like the scalar forms)
-    const float2 dl2 = make_float2(dlt, dlt), h2 = make_float2(h, h), nsh2 = make_float2(-shv, -shv),
-                 scv2 = make_float2(scv, scv);
-    const float2 sc2 = make_float2(sc, sc);
+    const float2 dl2 = make_float2(dlt, dlt + totA), h2 = make_float2(h, h), nsh2 = make_float2(-shv, -shv),
+                 scv2 = make_float2(scv, scv), sc2 = make_float2(sc, sc);
     float y[VPL];
     if (!big) {
 #pragma unroll
-        for (int j = 0; j < VPL; j += 2) {
-            const float2 S = fadd2_rn(make_float2(pl[j], pl[j + 1]), dl2);  // exact
+        for (int i = 0; i < HALF; i++) {
+            const float2 S = fadd2_rn(pp[i], dl2);  // exact (positions i and i + 18)
             const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
-            y[j] = y2.x;
-            y[j + 1] = y2.y;
+            y[i] = y2.x;
+            y[HALF + i] = y2.y;
         }
     } else {
 #pragma unroll
-        for (int j = 0; j < VPL; j++) {
-            const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, sc, h);  // 2^(emin+30) scale
-            y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
+        for (int i = 0; i < HALF; i++) {
+            const float2 S = fmul2_rn(fadd2_rn(pp[i], dl2), make_float2(0x1p100f, 0x1p100f));  // 2^(emin+30) scale
+            const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
+            y[i] = y2.x;
+            y[HALF + i] = y2.y;
         }
     }
     __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
