@@ -50,8 +50,11 @@ struct DcMeta {  // written by KD0, read by KD (32 B)
 };
 
 constexpr int kMaxWarpsPerCta = 8;
+#ifndef SPP_KD_EARLY_SYNC
+#define SPP_KD_EARLY_SYNC 0  // one-pass path: release the slot once the delta bytes are in registers
+#endif
 #ifndef SPP_KD_MINB
-#define SPP_KD_MINB 2  // CTAs per SM the register allocation targets (2: the 36-per-lane path needs ~128 registers)
+#define SPP_KD_MINB 3  // CTAs per SM the register allocation targets (3 x 8 warps: 80 registers, no spills)
 #endif
 constexpr int kMaxW = 16383;  // GPU path: per-segment byte base packed in 16 bits
 
@@ -460,6 +463,9 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;
         }
         if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
+#if SPP_KD_EARLY_SYNC
+    __syncwarp();  // every lane holds its delta bytes: the slot may take the row from here on
+#endif
         if constexpr (VPL == 8) {
             if (act && W - p0 < 8) {  // positions past the line end (W % 256 != 0)
                 const uint64_t m = (1ull << (8 * (W - p0))) - 1ull;
@@ -632,7 +638,9 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
             y[HALF + i] = y2.y;
         }
     }
+#if !SPP_KD_EARLY_SYNC
     __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
+#endif
     stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
     fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
     __syncwarp();

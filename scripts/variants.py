@@ -10,10 +10,9 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_la1_hot136": ["SPP_KC_LA=1", "SPP_KC_HOT_KB=136"],
-    "kc_la2_hot120": ["SPP_KC_LA=2", "SPP_KC_HOT_KB=120"],
-    "kc_la3_hot108": ["SPP_KC_LA=3", "SPP_KC_HOT_KB=108"],
-    "kc_la2_hot128_s4": ["SPP_KC_LA=2", "SPP_KC_HOT_KB=128", "SPP_KC_STAGES=4"],
+    "kd_m3": ["SPP_KD_MINB=3"],
+    "kd_m3_half": ["SPP_KD_MINB=3", "SPP_KD_HALF_SLOTS=1"],
+    "kd_m4_half": ["SPP_KD_MINB=4", "SPP_KD_HALF_SLOTS=1"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
