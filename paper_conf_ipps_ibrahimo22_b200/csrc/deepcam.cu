@@ -50,9 +50,6 @@ struct DcMeta {  // written by KD0, read by KD (32 B)
 };
 
 constexpr int kMaxWarpsPerCta = 8;
-#ifndef SPP_KD_EARLY_SYNC
-#define SPP_KD_EARLY_SYNC 0  // one-pass path: release the slot once the delta bytes are in registers
-#endif
 #ifndef SPP_KD_MINB
 #define SPP_KD_MINB 3  // CTAs per SM the register allocation targets (3 x 8 warps: 80 registers, no spills)
 #endif
@@ -98,6 +95,25 @@ template <int K>
 __device__ __forceinline__ float code_f_sar(uint32_t w) {
     const int32_t t = (int32_t)(w << (24 - 8 * K));
     return __uint_as_float((uint32_t)(t >> 5) & 0x83F80000u);
+}
+// Two delta codes as an fp16 pair: the code's 7 E|M bits land on fp16 bits
+// 6..12 and its sign on bit 15, so the half equals code * 2^-18 exactly (E = 0
+// maps onto fp16 subnormals). prmt puts code byte `lo` in bits 8..15 with its
+// sign replicated into bits 16..23 and code byte `hi` in bits 24..31; one
+// arithmetic shift by 2 moves both E|M fields into place while copying each
+// sign into bits 13..15 / 29..31, and one mask keeps sign + E|M.
+template <uint32_t SEL>
+__device__ __forceinline__ uint32_t codes_h2(uint32_t w) {
+    uint32_t x;
+    asm("prmt.b32 %0, %1, 0, %2;" : "=r"(x) : "r"(w), "n"(SEL));
+    return (uint32_t)((int32_t)x >> 2) & 0x9FC09FC0u;
+}
+// RN(float(a) + c) with a an fp16 (mixed-precision add, sm_100: FHADD)
+__device__ __forceinline__ float fadd_h(uint32_t h2, int hi, float c) {
+    const uint16_t a = (uint16_t)(hi ? (h2 >> 16) : (h2 & 0xFFFFu));
+    float d;
+    asm("add.rn.f32.f16 %0, %1, %2;" : "=f"(d) : "h"(a), "f"(c));
+    return d;
 }
 __device__ __forceinline__ float code_f_byte(uint32_t b) {
     return __uint_as_float(((b & 0x80u) << 24) | ((b & 0x7Fu) << 19));
@@ -453,8 +469,11 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         const SegInfo si = seg_info(desc, heads, s);
         // Every lane runs the same straight-line code.  Signed zeros make the
         // special cases exact without branches: a REPEAT lane decodes delta
-        // bytes 0x80 (code -0) and a head or REPEAT lane uses dlt = -0, so
-        // S = -0 there and fma(-0, sc, h) == h bit for bit (also for h = +-0).
+        // bytes 0x80 (code -0) and uses dlt = -0, so S = -0 there and
+        // fma(-0, sc, h) == h bit for bit (also for h = +-0); a head lane's
+        // position 0 takes S = -0 the same way, while its other positions
+        // sum from dlt = +0 like the definition's running sum (a code -0 after
+        // the head must give S = +0, not -0).
         const bool rep = si.kind == kRepeat || !act;
         Bytes<VPL> bt;
         bt.load(dl_s + (uint32_t)(rep ? 0 : si.a + (int)p0));
@@ -463,9 +482,6 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;
         }
         if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
-#if SPP_KD_EARLY_SYNC
-    __syncwarp();  // every lane holds its delta bytes: the slot may take the row from here on
-#endif
         if constexpr (VPL == 8) {
             if (act && W - p0 < 8) {  // positions past the line end (W % 256 != 0)
                 const uint64_t m = (1ull << (8 * (W - p0))) - 1ull;
@@ -498,7 +514,7 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         const uint32_t mle = smask & le_mask;
         const float gotb = __shfl_sync(0xffffffffu, P_excl, mle ? 31 - __clz(mle) : lane);
         const float base = mle ? gotb : carry_base;
-        const float dlt = (flag || rep) ? -0.0f : P_excl - base;
+        const float dlt = rep ? -0.0f : (flag ? 0.0f : P_excl - base);
         if constexpr (!STAGED) {
             carry_P += __shfl_sync(0xffffffffu, P, 31);
             const float topb = __shfl_sync(0xffffffffu, P_excl, smask ? 31 - __clz(smask) : 0);
@@ -509,13 +525,15 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
         if (!si.big) {
 #pragma unroll
             for (int j = 0; j < VPL; j++) {
-                const float xh = __fmaf_rn(pl[j] + dlt, si.sc, si.h);  // RN(h + S * 2^emin), S exact
+                const float S = (j == 0 && flag) ? -0.0f : pl[j] + dlt;  // exact
+                const float xh = __fmaf_rn(S, si.sc, si.h);              // RN(h + S * 2^emin)
                 y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
             }
         } else {
 #pragma unroll
             for (int j = 0; j < VPL; j++) {
-                const float xh = __fmaf_rn((pl[j] + dlt) * 0x1p100f, si.sc, si.h);  // 2^(emin+30) scale
+                const float S = (j == 0 && flag) ? -0.0f : (pl[j] + dlt) * 0x1p100f;  // 2^(emin+30) scale
+                const float xh = __fmaf_rn(S, si.sc, si.h);
                 y[j] = __fmul_rn(__fsub_rn(xh, shv), scv);
             }
         }
@@ -579,8 +597,6 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const float h = __shfl_sync(0xffffffffu, hs, s);
     const int a = (int)(d & 0xFFFFu) - 16384;
     const uint32_t skind = (d >> 16) & 0xFFu, seb = d >> 24;
-    const bool big = seb >= 148u;
-    const float sc = __uint_as_float((big ? (seb + 7u) : (seb + 107u)) << 23);
     const bool rep = skind == kRepeat;
     Bytes<VPL> bt;
     bt.load(dl_s + (uint32_t)(rep ? 0 : a + (int)p0));
@@ -589,21 +605,22 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
         for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;  // code -0: S = -0 keeps h exact
     }
     if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
-    // codes of the lane's 36 positions, then the lane prefix on pairs
-    // (position i, position i + 18) with FADD2: both halves at once (exact)
+    // codes of the lane's 36 positions as fp16 pairs (value = code * 2^-18),
+    // then two exact fp32 prefix chains (positions 0..17 and 18..35) fed by
+    // mixed-precision adds
     constexpr int HALF = VPL / 2;
-    float f[VPL];
+    uint32_t hv[VPL / 2];
 #pragma unroll
     for (int k = 0; k < VPL / 4; k++) {
-        f[4 * k + 0] = code_f_sar<0>(bt.w[k]);
-        f[4 * k + 1] = code_f_sar<1>(bt.w[k]);
-        f[4 * k + 2] = code_f_sar<2>(bt.w[k]);
-        f[4 * k + 3] = code_f_sar<3>(bt.w[k]);
+        hv[2 * k] = codes_h2<0x1800u>(bt.w[k]);      // positions 4k, 4k+1
+        hv[2 * k + 1] = codes_h2<0x3A20u>(bt.w[k]);  // positions 4k+2, 4k+3
     }
     float2 pp[HALF];
-    pp[0] = make_float2(f[0], f[HALF]);
+    pp[0] = make_float2(fadd_h(hv[0], 0, -0.0f), fadd_h(hv[HALF / 2], HALF & 1, -0.0f));
 #pragma unroll
-    for (int i = 1; i < HALF; i++) pp[i] = fadd2_rn(pp[i - 1], make_float2(f[i], f[HALF + i]));
+    for (int i = 1; i < HALF; i++)
+        pp[i] = make_float2(fadd_h(hv[i >> 1], i & 1, pp[i - 1].x),
+                            fadd_h(hv[(HALF + i) >> 1], (HALF + i) & 1, pp[i - 1].y));
     const float totA = pp[HALF - 1].x;
     const float lt = totA + pp[HALF - 1].y;  // lane total
     float P = lt;
@@ -615,32 +632,26 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const float P_excl = P - lt;
     const uint32_t mle = word & le_mask;
     const float base = __shfl_sync(0xffffffffu, P_excl, 31 - __clz(mle));
-    const float dlt = (flag || rep) ? -0.0f : P_excl - base;
-    // x̂ = RN(h + S * 2^emin) and y = RN(RN(x̂ - shift) * scale), two values per
-    // instruction (FADD2/FFMA2/FMUL2 round exactly like the scalar forms)
+    // REPEAT lane: every S = -0 (x̂ = h exactly); head lane: S = -0 at the
+    // head only, the rest sums from +0 like the definition's running sum
+    const float dlt = rep ? -0.0f : (flag ? 0.0f : P_excl - base);
+    // x̂ = RN(h + S * 2^emin) with S in code * 2^-18 units: the multiplier is
+    // 2^(emin + 18) = 2^(emin_b - 132), a normal float for emin_b >= 6 and an
+    // exact subnormal below; y = RN(RN(x̂ - shift) * scale). Two values per
+    // instruction (FADD2/FFMA2/FMUL2 round exactly like the scalar forms).
+    const float sc = __uint_as_float(seb >= 6u ? (seb - 5u) << 23 : 1u << (seb + 17u));
     const float2 dl2 = make_float2(dlt, dlt + totA), h2 = make_float2(h, h), nsh2 = make_float2(-shv, -shv),
                  scv2 = make_float2(scv, scv), sc2 = make_float2(sc, sc);
     float y[VPL];
-    if (!big) {
 #pragma unroll
-        for (int i = 0; i < HALF; i++) {
-            const float2 S = fadd2_rn(pp[i], dl2);  // exact (positions i and i + 18)
-            const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
-            y[i] = y2.x;
-            y[HALF + i] = y2.y;
-        }
-    } else {
-#pragma unroll
-        for (int i = 0; i < HALF; i++) {
-            const float2 S = fmul2_rn(fadd2_rn(pp[i], dl2), make_float2(0x1p100f, 0x1p100f));  // 2^(emin+30) scale
-            const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
-            y[i] = y2.x;
-            y[HALF + i] = y2.y;
-        }
+    for (int i = 0; i < HALF; i++) {
+        float2 S = fadd2_rn(pp[i], dl2);  // exact (positions i and i + 18)
+        if (i == 0 && flag) S.x = -0.0f;  // the head: x̂ = h exactly
+        const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
+        y[i] = y2.x;
+        y[HALF + i] = y2.y;
     }
-#if !SPP_KD_EARLY_SYNC
     __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
-#endif
     stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
     fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
     __syncwarp();

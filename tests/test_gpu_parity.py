@@ -237,6 +237,88 @@ def test_deepcam_handbuilt_lines(dev, orc, W):
     _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, "f32"))
 
 
+_EB_EDGES = [1, 2, 3, 4, 5, 6, 7, 60, 120, 147, 148, 149, 170, 200, 246]
+
+
+def _random_aligned_line(rng, W, A, nseg_max, kinds=(0, 1)):
+    """SEG line whose segments start on multiples of A (FORMAT.md 2.1, S14):
+    lengths are multiples of A except the last, which ends at W."""
+    segs, deltas, pos = [], [], 0
+    nblk = (W + A - 1) // A
+    while pos < W:
+        left = nblk - pos // A
+        k = 1 if nseg_max >= nblk else int(rng.integers(1, max(2, min(left, 2 * nblk // nseg_max + 1)) + 1))
+        ln = min(W - pos, k * A)
+        if len(segs) == nseg_max - 1:
+            ln = W - pos
+        kind = int(rng.choice(kinds))
+        eb = int(rng.choice(_EB_EDGES))
+        h = np.float32(rng.choice([0.0, -0.0, 1.0, rng.standard_normal() * 10.0 ** rng.integers(-40, 30),
+                                   2.0 ** -140, -3.0e38]))
+        segs.append((ln, kind, eb, h))
+        if kind == 1:
+            deltas += [int(v) for v in rng.integers(0, 256, size=ln - 1)]
+        pos += ln
+    return fmt.build_seg_line(W, segs, deltas)
+
+
+@pytest.mark.parametrize("nseg_max", [1, 4, 16, 32])
+def test_deepcam_handbuilt_aligned_lines(dev, orc, nseg_max):
+    """W = 1152 with segment alignment A = 36: the one-pass path (a segment
+    starts on a 36-value lane block, so 1..32 segments per line; 32 = every
+    lane its own segment); emin_b on both sides of the subnormal-multiplier bound
+    (< 6) and of the former large-exponent split (148); REPEAT of signed zero;
+    heads at every lane block; RAW lines interleaved."""
+    W, A, C, H = 1152, 36, 2, 20
+    rng = np.random.default_rng(1000 + nseg_max)
+    lines = []
+    for l in range(C * H):
+        if l % 7 == 6:
+            lines.append(fmt.build_raw_line(rng.standard_normal(W).astype(np.float32)))
+        else:
+            lines.append(_random_aligned_line(rng, W, A, nseg_max))
+    b = fmt.build_deepcam_stream(C, H, W, lines, A=A)
+    shift = np.float32([0.25, -7.0])
+    scale = np.float32([4.0, 3e-2])
+    for out in ("f16", "f32"):
+        got, st = _decode("deepcam", [b], (C, H, W), out=out, shift=shift, scale=scale)
+        assert st == 0
+        _same_bits(got[0], _dc_ref(orc, b, (C, H, W), shift, scale, out))
+    got, st = _decode("deepcam", [b], (C, H, W), out="f32")
+    _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, "f32"))
+
+
+@pytest.mark.parametrize("W,A", [(1152, 36), (64, 8), (17, 1)])
+def test_deepcam_signed_zero_codes(dev, orc, W, A):
+    """FORMAT.md 2.3: S_j is an integer prefix (code 0x80 is 0), so after a
+    head h = -0.0 every zero-sum position decodes to RN(-0 + 0) = +0 while
+    the head itself stays -0; REPEAT of -0 stays -0 everywhere.  Covers the
+    one-pass (A = 36), aligned (A = 8) and general (A = 1) line paths."""
+    C, H = 1, 6
+    half = (W // 2) // A * A or W
+    lines = [
+        fmt.build_seg_line(W, [(W, 1, 100, np.float32(-0.0))], [0x80] * (W - 1)),
+        fmt.build_seg_line(W, [(W, 1, 3, np.float32(-0.0))], ([0x80, 0x00, 0x81, 0x01] * W)[:W - 1]),
+        fmt.build_seg_line(W, [(W, 1, 200, np.float32(0.0))], [0x80] * (W - 1)),
+        fmt.build_seg_line(W, [(W, 0, 0, np.float32(-0.0))], []),
+        fmt.build_seg_line(W, [(half, 1, 5, np.float32(-0.0)), (W - half, 1, 150, np.float32(-0.0))]
+                           if half < W else [(W, 1, 5, np.float32(-0.0))],
+                           [0x80] * (W - (2 if half < W else 1))),
+        fmt.build_seg_line(W, [(half, 0, 0, np.float32(-0.0)), (W - half, 1, 7, np.float32(-0.0))]
+                           if half < W else [(W, 0, 0, np.float32(-0.0))],
+                           [0x80] * (W - half - 1) if half < W else []),
+    ]
+    b = fmt.build_deepcam_stream(C, H, W, lines, A=A)
+    want = _dc_ref(orc, b, (C, H, W), None, None, "f32")
+    # the definition: only heads and REPEAT positions keep -0
+    assert np.signbit(want[0, 0, 0]) and not np.signbit(want[0, 0, 1:]).any()
+    assert np.signbit(want[0, 3]).all()
+    for out in ("f32", "f16"):
+        got, st = _decode("deepcam", [b], (C, H, W), out=out)
+        assert st == 0
+        _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, out))
+
+
 def test_deepcam_batch_order_independence(dev, orc):
     """P13: decoding samples alone, in a batch, or in another order gives the
     same bytes per sample."""
