@@ -10,9 +10,12 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kd_m3": ["SPP_KD_MINB=3"],
-    "kd_m3_half": ["SPP_KD_MINB=3", "SPP_KD_HALF_SLOTS=1"],
-    "kd_m4_half": ["SPP_KD_MINB=4", "SPP_KD_HALF_SLOTS=1"],
+    "kc_la1": ["SPP_KC_LA=1"],
+    "kc_la1_hot132": ["SPP_KC_LA=1", "SPP_KC_HOT_KB=132"],
+    "kc_la1_st4_hot140": ["SPP_KC_LA=1", "SPP_KC_STAGES=4", "SPP_KC_HOT_KB=140"],
+    "kc_la1_st6": ["SPP_KC_LA=1", "SPP_KC_STAGES=6"],
+    "kc_la0": ["SPP_KC_LA=0"],
+    "kc_la2": ["SPP_KC_LA=2"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
