@@ -50,7 +50,7 @@ constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 #define SPP_KC_THREADS 768
 #endif
 #ifndef SPP_KC_HOT_KB
-#define SPP_KC_HOT_KB 120
+#define SPP_KC_HOT_KB 132
 #endif
 constexpr int kThreads = SPP_KC_THREADS;
 constexpr int kPrologueThreads = 256;
@@ -71,7 +71,7 @@ constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
 constexpr int kStageBytes = kTileVox * 2;
 #ifndef SPP_KC_LA
-#define SPP_KC_LA 2
+#define SPP_KC_LA 1
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
 constexpr int kColdSlotBytes = (kColdLA + 1) * kThreads * 16;  // 2 rows per thread per tile in flight

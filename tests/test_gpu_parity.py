@@ -141,6 +141,29 @@ def test_cosmo_c2_launch_configuration(dev, orc):
         assert torch.equal(o16[i], want[i % 3]), i
 
 
+def test_cosmo_256_multi_lut(dev, orc):
+    """a 4x256^3 paper-preset volume (8x the paper's sample)
+    needs several z-slab lookup tables ("multiple LUTs"); also a
+    non-cubic 4x96x256x128 volume.  Both decoded bit-exactly, fp16 and fp32."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_cosmo(1001, n=256)
+    b = spp.spp_encode_cosmo(x)
+    nU, T, G, kw = spp.spp_stream_info("cosmo", b)
+    assert T > 1 and kw == 2                           # multiple tables, 2-byte keys
+    for out in ("f16", "f32"):
+        got, st = _decode("cosmo", [b], x.shape, out=out)
+        assert st == 0
+        _same_bits(got[0], orc.cosmo_direct(x, 1, out))
+    y = np.ascontiguousarray(x[:, :96, :, ::2])
+    b2 = spp.spp_encode_cosmo(y)
+    got, st = _decode("cosmo", [b2, b2], y.shape, out="f16")
+    assert st == 0
+    want = orc.cosmo_direct(y, 1, "f16")
+    _same_bits(got[0], want)
+    _same_bits(got[1], want)
+
+
 def test_cosmo_corruption_detected(dev):
     from synth import gen_cosmo
     from paper_conf_ipps_ibrahimo22_b200 import spp
