@@ -689,9 +689,6 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     }
     __syncwarp();
 
-    // line coordinates tracked incrementally (no divisions per line)
-    uint32_t s_cur = (uint32_t)(g_begin / L), l_cur = (uint32_t)(g_begin - (uint64_t)s_cur * L);
-    uint32_t c_cur = l_cur / H, y_cur = l_cur - c_cur * H;
 
     // Directory window: lane k holds the validated directory entry of line
     // wbase + k (source pointer, bytes, flags), loaded and checked by all lanes
@@ -699,6 +696,7 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     uint64_t wbase = 0;
     uint64_t w_src = 0;
     uint32_t w_bytes = 0, w_flags = 0;  // flags: bit 0 big, bits 16.. alignment
+    float w_shv = 0.f, w_scv = 1.f;     // the line's channel constants (c = (g mod L) / H)
     auto load_window = [&](uint64_t wb) {
         wbase = wb;
         const uint64_t g = wb + lane;
@@ -708,6 +706,9 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
         if (g < g_end) {
             const uint64_t sk = g / L;
             const uint32_t lk = (uint32_t)(g - sk * L);
+            const uint32_t ck = lk / H;
+            w_shv = shift ? __ldg(shift + ck) : 0.f;
+            w_scv = scale ? __ldg(scale + ck) : 1.f;
             const DcMeta m = meta[sk];
             if (m.valid) {
                 const uint32_t *dir = reinterpret_cast<const uint32_t *>(m.dir);
@@ -732,15 +733,18 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
         bytes = __shfl_sync(0xffffffffu, w_bytes, k);
         flags = __shfl_sync(0xffffffffu, w_flags, k);
     };
+    auto consts = [&](uint64_t g, float &sh, float &sc) {  // g in the current window
+        const int k = (int)(g - wbase);
+        sh = __shfl_sync(0xffffffffu, w_shv, k);
+        sc = __shfl_sync(0xffffffffu, w_scv, k);
+    };
     auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {  // lane 0
         if constexpr (VPL == 36) bulk_wait_read_all();  // a staged row may still be leaving this slot
         mbar_arrive_expect_tx(&mbar[slot], bytes);
         bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
     };
 
-    uint32_t c_cached = 0xFFFFFFFFu;
-    float shv = 0.f, scv = 1.f;
-    uint32_t phase0 = 0, phase1 = 0;
+    uint32_t phases = 0;  // bit k: parity of slot k's mbarrier
     int slot = 0;
     load_window(g_begin);
     const uint8_t *cur_src;
@@ -748,6 +752,8 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     entry(g_begin, cur_src, cur_bytes, cur_flags);
     if (lane == 0 && cur_bytes && !(cur_flags & 1u)) issue(0, cur_src, cur_bytes);
     for (uint64_t g = g_begin; g < g_end; g++) {
+        float shv, scv;
+        consts(g, shv, scv);  // before the window may move on to g + 1
         const uint8_t *nxt_src = nullptr;
         uint32_t nxt_bytes = 0, nxt_flags = 0, nxt_issued = 0;
         if (g + 1 < g_end) {
@@ -775,17 +781,9 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
                 fence_proxy_async_smem();  // generic writes before later TMA writes to these slots
                 __syncwarp();
                 buf = base;
-            } else if (slot == 0) {
-                mbar_wait(&mbar[0], phase0);
-                phase0 ^= 1;
             } else {
-                mbar_wait(&mbar[1], phase1);
-                phase1 ^= 1;
-            }
-            if (c_cur != c_cached) {  // per-channel constants change every H lines
-                c_cached = c_cur;
-                shv = shift ? __ldg(shift + c_cur) : 0.f;
-                scv = scale ? __ldg(scale + c_cur) : 1.f;
+                mbar_wait(&mbar[slot], (phases >> slot) & 1u);
+                phases ^= 1u << slot;
             }
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
@@ -795,7 +793,7 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
             }
             else
                 ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
-            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)s_cur);
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
         }
         __syncwarp();
         if (lane == 0 && nxt_bytes && !(nxt_flags & 1u) && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
@@ -803,16 +801,6 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
         cur_bytes = nxt_bytes;
         cur_flags = nxt_flags;
         cur_src = nxt_src;
-        if (++y_cur == H) {
-            y_cur = 0;
-            c_cur++;
-        }
-        if (++l_cur == L) {
-            l_cur = 0;
-            s_cur++;
-            c_cur = 0;
-            y_cur = 0;
-        }
     }
     if constexpr (VPL == 36) {
         if (lane == 0) bulk_wait_all();  // shared memory must outlive the last row stores

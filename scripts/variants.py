@@ -30,7 +30,8 @@ def build():
 
 def run():
     res = {}
-    for name in VARIANTS:
+    names = [v for v in os.environ.get("VARIANT_NAMES", ",".join(VARIANTS)).split(",") if v]
+    for name in names:
         env = dict(os.environ, SPP_LIB=str(OUT / f"libspp_{name}.so"))
         if "@" in name:
             env["SPP_L2_PERSIST_MB"] = name.split("@")[1]
