@@ -52,9 +52,14 @@ constexpr size_t kFuStride = kMaxU;  // floats per sample in the workspace
 #ifndef SPP_KC_HOT_KB
 #define SPP_KC_HOT_KB 132
 #endif
-constexpr int kThreads = SPP_KC_THREADS;
+#ifndef SPP_KC_PRODUCER
+#define SPP_KC_PRODUCER 1
+#endif
+constexpr int kConsumers = SPP_KC_THREADS;  // threads that expand voxels (8 per tile)
+constexpr bool kProducerWarp = SPP_KC_PRODUCER;  // one extra warp refills the key ring
+constexpr int kThreads = kConsumers + (kProducerWarp ? 32 : 0);
 constexpr int kPrologueThreads = 256;
-constexpr int kMinBlocks = kThreads <= 256 ? 3 : (kThreads <= 384 ? 2 : 1);  // CTAs per SM the registers target
+constexpr int kMinBlocks = kThreads <= 288 ? 3 : (kThreads <= 416 ? 2 : 1);  // CTAs per SM the registers target
 constexpr int kHotBytes = SPP_KC_HOT_KB * 1024;  // shared-memory hot prefix of T per CTA
 constexpr int kUCap = 2048;           // part of the region nominally for f(U) (8 KB)
 constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot tuples
@@ -68,13 +73,13 @@ constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 #ifndef SPP_KC_PREFETCH_TAIL
 #define SPP_KC_PREFETCH_TAIL 1
 #endif
-constexpr int kTileVox = kThreads * 8;  // voxels per CTA iteration (8 per thread)
+constexpr int kTileVox = kConsumers * 8;  // voxels per CTA iteration (8 per consumer thread)
 constexpr int kStageBytes = kTileVox * 2;
 #ifndef SPP_KC_LA
 #define SPP_KC_LA 1
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
-constexpr int kColdSlotBytes = (kColdLA + 1) * kThreads * 16;  // 2 rows per thread per tile in flight
+constexpr int kColdSlotBytes = (kColdLA + 1) * kConsumers * 16;  // 2 rows per thread per tile in flight
 constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes + 2 * kKeyStages * 8;
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
@@ -365,7 +370,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
 #pragma unroll
     for (int i = 0; i <= kColdLA; i++) cj[i] = 0x0808u;
     auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k (0/1) of this thread for tile t
-        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kThreads + threadIdx.x) * 2 + k) * 8;
+        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * 2 + k) * 8;
     };
     auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
@@ -392,8 +397,20 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         cp_async_commit();
         return j0 | (j1 << 8);
     };
-    if (threadIdx.x == 0)
+    if constexpr (kProducerWarp) {
+        // The producer warp keeps the ring full for the whole call: it refills a
+        // stage as soon as the last consumer warp releases it, independent of
+        // any consumer's own progress (an issuing consumer would lag the others).
+        if (threadIdx.x >= (uint32_t)kConsumers) {
+            if (threadIdx.x == (uint32_t)kConsumers)
+                for (uint32_t t = 0; t < ntiles; t++) issue(t);
+            __syncwarp();
+            ring.count += ntiles;
+            return;
+        }
+    } else if (threadIdx.x == 0) {
         for (uint32_t t = 0; t < ntiles && t < (uint32_t)(kKeyStages - 1); t++) issue(t);
+    }
 #pragma unroll
     for (int i = 0; i < kColdLA; i++) {
         if ((uint32_t)i < ntiles) {
@@ -405,7 +422,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     }
 #pragma unroll 1
     for (uint32_t t = 0; t < ntiles; t++) {
-        if (threadIdx.x == 0 && t + kKeyStages - 1 < ntiles) issue(t + kKeyStages - 1);
+        if (!kProducerWarp && threadIdx.x == 0 && t + kKeyStages - 1 < ntiles) issue(t + kKeyStages - 1);
         if (t + kColdLA < ntiles) {
             wait_full(t + kColdLA);
             cj[kColdLA] = classify(t + kColdLA);
@@ -468,7 +485,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     if (VEC && threadIdx.x == 0) {
         for (int i = 0; i < kKeyStages; i++) {
             mbar_init(&ring.full[i], 1);
-            mbar_init(&ring.empty[i], kThreads / kWarp);  // one arrival per warp
+            mbar_init(&ring.empty[i], kConsumers / kWarp);  // one arrival per consumer warp
         }
         fence_mbar_init();
     }

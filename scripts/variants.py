@@ -10,12 +10,12 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_la1": ["SPP_KC_LA=1"],
-    "kc_la1_hot132": ["SPP_KC_LA=1", "SPP_KC_HOT_KB=132"],
-    "kc_la1_st4_hot140": ["SPP_KC_LA=1", "SPP_KC_STAGES=4", "SPP_KC_HOT_KB=140"],
-    "kc_la1_st6": ["SPP_KC_LA=1", "SPP_KC_STAGES=6"],
-    "kc_la0": ["SPP_KC_LA=0"],
-    "kc_la2": ["SPP_KC_LA=2"],
+    "kc_prod0": ["SPP_KC_PRODUCER=0"],
+    "kc_prod1": ["SPP_KC_PRODUCER=1"],
+    "kc_prod1_st4_hot140": ["SPP_KC_PRODUCER=1", "SPP_KC_STAGES=4", "SPP_KC_HOT_KB=140"],
+    "kc_prod1_la2_hot120": ["SPP_KC_PRODUCER=1", "SPP_KC_LA=2", "SPP_KC_HOT_KB=120"],
+    "kc_prod1_c736": ["SPP_KC_PRODUCER=1", "SPP_KC_THREADS=736"],
+    "kc_prod1_c736_hot136": ["SPP_KC_PRODUCER=1", "SPP_KC_THREADS=736", "SPP_KC_HOT_KB=136"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
