@@ -807,6 +807,248 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
     }
 }
 
+// ---------------------------------------------------------------------------
+// Warp-specialised KD (default): the last warp of each CTA is a producer whose
+// lane k streams the lines of consumer warp k into that warp's two shared
+// slots (directory read + validation, channel constants, 1-D TMA bulk copy,
+// full/empty mbarriers per slot), so the decoding warps spend their issue
+// slots on decoding only.  A consumer waits for its slot, decodes the line
+// exactly as kd_decode does (same device functions), and releases the slot
+// once its staged row has left shared memory.  An oversize line (> one slot)
+// is copied across both slots after both are released.
+#ifndef SPP_KD_WS
+#define SPP_KD_WS 1
+#endif
+#ifndef SPP_KD_WS_WPC
+#define SPP_KD_WS_WPC 11  // consumer warps per CTA (+1 producer warp)
+#endif
+#ifndef SPP_KD_WS_MINB
+#define SPP_KD_WS_MINB 2
+#endif
+constexpr int kWsWarps = SPP_KD_WS_WPC + 1;
+#ifndef SPP_KD_WS_NS
+#define SPP_KD_WS_NS 3  // input slots per consumer warp (a ring)
+#endif
+#ifndef SPP_KD_WS_SLOT
+#define SPP_KD_WS_SLOT 2560  // target slot bytes (>= the staged row); longer lines take the whole ring
+#endif
+constexpr uint32_t kWsNs = SPP_KD_WS_NS;
+static_assert(kWsNs >= 2 && kWsNs <= 8, "slot ring");
+constexpr uint32_t kWsCtl = 32 * kWsNs;  // per consumer: full[NS], empty[NS] mbarriers + info[NS] (16 B each)
+
+template <int OUT, bool VEC, int VPL>
+__global__ void __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
+    const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
+    const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
+    uint32_t *__restrict__ status) {
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int wpc = (int)(blockDim.x >> 5) - 1;  // consumer warps; warp wpc produces
+    const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
+    const uint32_t cap_data = cap - 16;     // one slot; the last 16 B are read slack
+    const uint32_t big_cap = kWsNs * cap - 16;  // the whole ring
+    const uint64_t T = (uint64_t)n * L;
+    const uint64_t NW = (uint64_t)gridDim.x * wpc;
+    const uint32_t ctl_off = (kWsNs * cap + 8 * nwords + 15u) & ~15u;  // 16-B aligned: info[] is read as uint4
+    auto ctl = [&](int w) { return reinterpret_cast<uint64_t *>(smem_raw + (size_t)w * warp_bytes + ctl_off); };
+
+    if (warp == wpc && lane < wpc) {
+        uint64_t *c = ctl(lane);
+        for (uint32_t i = 0; i < 2 * kWsNs; i++) mbar_init(&c[i], 1);  // full[NS]: producer + TMA bytes; empty[NS]: consumer lane 0
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    if (warp == wpc) {
+        // ------------------------------------------------------------ producer
+        // Lane k streams consumer k's lines.  The directory is read one line
+        // ahead of need (dn = dir[lk + 2]), so the entry of the next line is
+        // ready, from registers, the moment its slot is released.
+        const int k = lane;
+        bool active = k < wpc;
+        uint64_t g = 0, ge = 0;
+        if (active) {
+            const uint64_t gw = (uint64_t)blockIdx.x * wpc + k;
+            g = gw * T / NW;
+            ge = (gw + 1) * T / NW;
+            active = g < ge;
+        }
+        uint8_t *rb = smem_raw + (size_t)(active ? k : 0) * warp_bytes;
+        uint64_t *full = ctl(active ? k : 0), *empty = full + kWsNs;
+        uint4 *info = reinterpret_cast<uint4 *>(full + 2 * kWsNs);
+        uint32_t sk = 0, lk = 0, ck = 0, yk = 0, da = 0, db = 0, dn = 0, s = 0;
+        uint32_t used = 0, par = 0;  // bit i: slot i filled before / parity of its next release
+        DcMeta m{nullptr, nullptr, 0, 0, 0};
+        float shv = 0.f, scv = 1.f;
+        uint32_t e_bytes = 0, e_flags = 0;
+        const uint8_t *e_src = nullptr;
+        auto dir_at = [&](uint32_t i) { return __ldg(reinterpret_cast<const uint32_t *>(m.dir) + i); };
+        auto start_sample = [&]() {  // line lk of sample sk (synchronous: once per sample)
+            m = meta[sk];
+            if (m.valid) {
+                da = dir_at(lk);
+                db = dir_at(lk + 1);
+                dn = lk + 2 <= L ? dir_at(lk + 2) : 0u;
+            }
+        };
+        auto load_consts = [&]() {
+            shv = shift ? __ldg(shift + ck) : 0.f;
+            scv = scale ? __ldg(scale + ck) : 1.f;
+        };
+        auto compute_entry = [&]() {  // line g from (da, db), validated once
+            e_bytes = 0;
+            e_flags = 0;
+            if (m.valid) {
+                const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= m.limit && db - da >= 16;
+                if (!ok) {
+                    report(status, SPP_ERR_CORRUPT, (int64_t)sk);
+                } else if (db - da > big_cap) {
+                    report(status, SPP_ERR_UNSUPPORTED, (int64_t)sk);
+                } else {
+                    e_bytes = db - da;
+                    e_src = m.payload + da;
+                    e_flags = (e_bytes > cap_data ? 1u : 0u) | (m.align << 16);
+                }
+            }
+        };
+        if (active) {
+            sk = (uint32_t)(g / L);
+            lk = (uint32_t)(g - (uint64_t)sk * L);
+            ck = lk / H;
+            yk = lk - ck * H;
+            start_sample();
+            load_consts();
+            compute_entry();
+        }
+        while (__any_sync(0xffffffffu, active)) {
+            bool did = false;
+            if (active) {
+                const bool big = e_flags & 1u;
+                bool ready;
+                if (!big) {
+                    ready = !((used >> s) & 1u) || mbar_test(&empty[s], (par >> s) & 1u);
+                } else {  // an oversize line takes the whole ring: every slot must be free
+                    ready = true;
+                    for (uint32_t i = 0; i < kWsNs; i++)
+                        ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
+                }
+                if (ready) {
+                    sts_u4(smem_u32(&info[s]), make_uint4(e_bytes, e_flags, __float_as_uint(shv), __float_as_uint(scv)));
+                    if (e_bytes) {
+                        mbar_arrive_expect_tx(&full[s], e_bytes);
+                        bulk_g2s(big ? rb : rb + s * cap, e_src, e_bytes, &full[s]);  // (s: this line's slot)
+                    } else {
+                        mbar_arrive(&full[s]);  // nothing to copy: the consumer skips the line
+                    }
+                    const uint32_t took = big ? (1u << kWsNs) - 1u : 1u << s;
+                    par ^= took & used;
+                    used |= took;
+                    s = s + 1 == kWsNs ? 0u : s + 1;
+                    g++;
+                    did = true;
+                    active = g < ge;
+                    if (active) {  // advance to line g and prepare its entry
+                        if (++yk == H) {
+                            yk = 0;
+                            ck++;
+                        }
+                        if (++lk == L) {
+                            lk = 0;
+                            ck = 0;
+                            yk = 0;
+                            sk++;
+                            start_sample();
+                        } else {
+                            da = db;
+                            db = dn;
+                            if (m.valid && lk + 2 <= L) dn = dir_at(lk + 2);  // used one line from now
+                        }
+                        if (yk == 0) load_consts();
+                        compute_entry();
+                    }
+                }
+            }
+            if (!__any_sync(0xffffffffu, did)) __nanosleep(100);
+        }
+        return;
+    }
+
+    // ---------------------------------------------------------------- consumer
+    const uint64_t gw = (uint64_t)blockIdx.x * wpc + warp;
+    const uint64_t g_begin = gw * T / NW, g_end = (gw + 1) * T / NW;
+    uint8_t *base = smem_raw + (size_t)warp * warp_bytes;
+    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + kWsNs * cap);
+    uint32_t *wpre = sbits + nwords;
+    uint64_t *full = ctl(warp), *empty = full + kWsNs;
+    const uint32_t info_s = smem_u32(full + 2 * kWsNs);
+    const uint32_t nbw = (W / VPL + 31) / 32;
+    uint32_t fph = 0;  // bit s: parity of slot s's next full phase
+    uint32_t s = 0;
+    for (uint64_t g = g_begin; g < g_end; g++, s = s + 1 == kWsNs ? 0u : s + 1) {
+        mbar_wait(&full[s], (fph >> s) & 1u);
+        fph ^= 1u << s;
+        const uint4 inf = lds_u4(info_s + 16u * s);
+        const uint32_t bytes = inf.x, flags = inf.y, al = flags >> 16;
+        if (bytes) {
+            uint8_t *buf = (flags & 1u) ? base : base + s * cap;
+            const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
+            uint8_t *row = dst + g * (uint64_t)W * ob;
+            bool ok;
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
+                if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            } else {
+                ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
+            }
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
+        }
+        __syncwarp();
+        if (lane == 0) {
+            if constexpr (VPL == 36) bulk_wait_read_all();  // the staged row has left the slot
+            if (flags & 1u) {
+                for (uint32_t i = 0; i < kWsNs; i++) mbar_arrive(&empty[i]);  // the line took the whole ring
+            } else {
+                mbar_arrive(&empty[s]);
+            }
+        }
+    }
+    if constexpr (VPL == 36) {
+        if (lane == 0) bulk_wait_all();  // shared memory must outlive the last row stores
+    }
+}
+
+template <int OUT, bool VEC, int VPL>
+spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
+                        const DeviceProps &dp) {
+    const uint32_t W = (uint32_t)o.W;
+    // slot: a typical SEG line (~1 B/value) and the staged output row; a RAW
+    // line (or any longer line) takes the whole ring, which always holds RAW
+    const uint32_t raw = (uint32_t)round_up16(16 + 4ull * W);
+    const uint32_t row = VPL == 36 ? W * (OUT == SPP_OUT_F32 ? 4u : 2u) : 0u;
+    uint32_t cap_in = std::min<uint32_t>(raw, SPP_KD_WS_SLOT);
+    cap_in = std::max<uint32_t>(cap_in, (uint32_t)round_up16((raw + kWsNs - 1) / kWsNs));
+    const uint32_t cap = (uint32_t)round_up16(std::max(cap_in, row)) + 16;
+    const uint32_t nwords = (W + 31) / 32 + 1;
+    const uint32_t warp_bytes = (uint32_t)round_up16(kWsNs * cap + 8 * nwords) + kWsCtl;
+    int wpc = SPP_KD_WS_WPC;
+    while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
+    if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
+    const int smem = wpc * (int)warp_bytes;
+    auto kern = kd_decode_ws<OUT, VEC, VPL>;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+        return SPP_ERR_CUDA;
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, (wpc + 1) * kWarp, smem) != cudaSuccess || occ < 1)
+        return SPP_ERR_CUDA;
+    const uint64_t lines = (uint64_t)n * o.C * o.H;
+    const uint64_t max_ctas = (uint64_t)dp.sms * occ;
+    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
+    kern<<<grid, (wpc + 1) * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift,
+                                                     o.scale, static_cast<uint8_t *>(d_dst), cap, nwords, warp_bytes,
+                                                     o.status);
+    return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
+}
+
 template <int OUT, bool VEC, int VPL>
 spp_status launch_kd(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
                      const DeviceProps &dp) {
@@ -852,14 +1094,20 @@ spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const sp
     const bool vec = o.W % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
     const bool v36 = vec && o.W == 1152;  // the DeepCAM line: 32 lanes x 36 positions, one pass
     spp_status r = SPP_ERR_INVALID_ARG;
+#if SPP_KD_WS
+#define SPP_LAUNCH_KD launch_kd_ws
+#else
+#define SPP_LAUNCH_KD launch_kd
+#endif
     if (o.out == SPP_OUT_F32)
-        r = v36 ? launch_kd<SPP_OUT_F32, true, 36>(meta, n, d_dst, o, stream, dp)
-                : vec ? launch_kd<SPP_OUT_F32, true, 8>(meta, n, d_dst, o, stream, dp)
-                      : launch_kd<SPP_OUT_F32, false, 8>(meta, n, d_dst, o, stream, dp);
+        r = v36 ? SPP_LAUNCH_KD<SPP_OUT_F32, true, 36>(meta, n, d_dst, o, stream, dp)
+                : vec ? SPP_LAUNCH_KD<SPP_OUT_F32, true, 8>(meta, n, d_dst, o, stream, dp)
+                      : SPP_LAUNCH_KD<SPP_OUT_F32, false, 8>(meta, n, d_dst, o, stream, dp);
     else if (o.out == SPP_OUT_F16)
-        r = v36 ? launch_kd<SPP_OUT_F16, true, 36>(meta, n, d_dst, o, stream, dp)
-                : vec ? launch_kd<SPP_OUT_F16, true, 8>(meta, n, d_dst, o, stream, dp)
-                      : launch_kd<SPP_OUT_F16, false, 8>(meta, n, d_dst, o, stream, dp);
+        r = v36 ? SPP_LAUNCH_KD<SPP_OUT_F16, true, 36>(meta, n, d_dst, o, stream, dp)
+                : vec ? SPP_LAUNCH_KD<SPP_OUT_F16, true, 8>(meta, n, d_dst, o, stream, dp)
+                      : SPP_LAUNCH_KD<SPP_OUT_F16, false, 8>(meta, n, d_dst, o, stream, dp);
+#undef SPP_LAUNCH_KD
     if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;
     return r;
 }

@@ -10,18 +10,22 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_prod0": ["SPP_KC_PRODUCER=0"],
-    "kc_prod1": ["SPP_KC_PRODUCER=1"],
-    "kc_prod1_st4_hot140": ["SPP_KC_PRODUCER=1", "SPP_KC_STAGES=4", "SPP_KC_HOT_KB=140"],
-    "kc_prod1_la2_hot120": ["SPP_KC_PRODUCER=1", "SPP_KC_LA=2", "SPP_KC_HOT_KB=120"],
-    "kc_prod1_c736": ["SPP_KC_PRODUCER=1", "SPP_KC_THREADS=736"],
-    "kc_prod1_c736_hot136": ["SPP_KC_PRODUCER=1", "SPP_KC_THREADS=736", "SPP_KC_HOT_KB=136"],
+    "kd_ws0": ["SPP_KD_WS=0"],
+    "kd_ns2": ["SPP_KD_WS_NS=2"],
+    "kd_ns3": ["SPP_KD_WS_NS=3"],
+    "kd_ns4_10x2": ["SPP_KD_WS_NS=4", "SPP_KD_WS_WPC=10"],
+    "kd_ns3_7x3": ["SPP_KD_WS_NS=3", "SPP_KD_WS_WPC=7", "SPP_KD_WS_MINB=3"],
+    "kd_ns3_23x1": ["SPP_KD_WS_NS=3", "SPP_KD_WS_WPC=23", "SPP_KD_WS_MINB=1"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
 
 def build():
+    import shutil
     from paper_conf_ipps_ibrahimo22_b200 import build as b
+    shutil.rmtree(OUT, ignore_errors=True)        # only this sweep's libraries travel to the box
+    for d in OUT.parent.glob("_build_*"):
+        shutil.rmtree(d, ignore_errors=True)
     OUT.mkdir(exist_ok=True)
     for name, d in VARIANTS.items():
         b.build(force=True, defines=d, out=OUT / f"libspp_{name}.so")  # noqa
