@@ -84,6 +84,26 @@ size_t spp_deepcam_max_encoded_size(int C, int H, int W);
 spp_status spp_encode_deepcam(const float *x, int C, int H, int W,
                               void *dst, size_t dst_capacity, size_t *encoded_size);
 
+/* Encoder policy knobs (FORMAT.md 2.4).  PAPER.md P:84 fixes
+ * the code (1 sign, 3 exponent, 4 mantissa bits, per-segment minimum
+ * exponent) but not how segments are chosen; these trade bytes for error:
+ *   lookahead  : positions whose differences set a new DIFF segment's emin
+ *                (default 64; shorter windows adapt emin faster: smaller
+ *                errors next to abrupt changes, more segments).  2..65535.
+ *   repeat_min : shortest run of bit-identical values that opens a REPEAT
+ *                segment (default 16).  2..65535.
+ * A zero field selects its default.  Every setting obeys the per-value
+ * error bound of DESIGN.md reading S19 and decodes on the unchanged decoders. */
+typedef struct {
+    int lookahead;
+    int repeat_min;
+} spp_deepcam_params;
+
+/* spp_encode_deepcam with explicit policy knobs (params may be NULL = defaults);
+ * out-of-range knobs -> SPP_ERR_INVALID_ARG. */
+spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W, const spp_deepcam_params *params,
+                                 void *dst, size_t dst_capacity, size_t *encoded_size);
+
 /* Host-side parse of one encoded sample's header (no CUDA).  For CosmoFlow
  * info[0..3] = nU, nslab, G of slab 0, kw of slab 0; for DeepCAM info[0..3] =
  * number of RAW lines, SEG lines, total segments, total delta bytes.

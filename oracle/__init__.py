@@ -64,6 +64,8 @@ def lib():
         L.orc_deepcam_max_encoded_size.argtypes = [I, I, I]; L.orc_deepcam_max_encoded_size.restype = SZ
         L.orc_deepcam_encode.argtypes = [P, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_deepcam_encode.restype = I
         L.orc_deepcam_encode_a.argtypes = [P, I, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_deepcam_encode_a.restype = I
+        L.orc_deepcam_encode_p.argtypes = [P, I, I, I, I, I, I, P, SZ, C.POINTER(SZ)]
+        L.orc_deepcam_encode_p.restype = I
         L.orc_deepcam_align.argtypes = [I]; L.orc_deepcam_align.restype = I
         _lib = L
     return _lib
@@ -125,8 +127,9 @@ def deepcam_code(b: int) -> int:
     return int(lib().orc_deepcam_code(int(b)))
 
 
-def deepcam_encode(x: np.ndarray, align: int | None = None) -> np.ndarray:
-    """FORMAT.md 2.4 encoder; `align` overrides the default alignment rule."""
+def deepcam_encode(x: np.ndarray, align: int | None = None, lookahead: int = 64, repeat_min: int = 16) -> np.ndarray:
+    """FORMAT.md 2.4 encoder; `align` overrides the default alignment rule,
+    `lookahead` / `repeat_min` the policy knobs (defaults 64 / 16)."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     assert a.ndim == 3
     Cc, H, W = a.shape
@@ -134,7 +137,8 @@ def deepcam_encode(x: np.ndarray, align: int | None = None) -> np.ndarray:
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
     A = lib().orc_deepcam_align(W) if align is None else int(align)
-    _check(lib().orc_deepcam_encode_a(_p(a), Cc, H, W, A, _p(dst), cap, C.byref(size)), "deepcam_encode")
+    _check(lib().orc_deepcam_encode_p(_p(a), Cc, H, W, A, int(lookahead), int(repeat_min), _p(dst), cap,
+                                      C.byref(size)), "deepcam_encode")
     return dst[: size.value].copy()
 
 

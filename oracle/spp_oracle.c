@@ -441,8 +441,8 @@ static int rep_len(const int *run, int i, int W, int A) {
     return (i + r == W) ? r : (r / A) * A;
 }
 
-static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_out, uint8_t *deltas,
-                           int64_t *ndelta_out, int *run) {
+static int64_t encode_line(const float *x, int W, int A, int lookahead, int repeat_min, seg_t *segs,
+                           int *nseg_out, uint8_t *deltas, int64_t *ndelta_out, int *run) {
     /* run lengths of bit-identical values */
     run[W - 1] = 1;
     for (int i = W - 2; i >= 0; i--)
@@ -452,7 +452,7 @@ static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_
     int i = 0;
     while (i < W) {
         int rl = rep_len(run, i, W, A);
-        if (rl >= 16) {
+        if (rl >= repeat_min) {
             segs[nseg].len = rl; segs[nseg].kind = 0; segs[nseg].emin_b = 0; segs[nseg].head = x[i];
             nseg++;
             i += rl;
@@ -460,7 +460,7 @@ static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_
         }
         float h = x[i];
         double m = 0.0;
-        for (int j = i + 1; j < W && j < i + 64; j++) {
+        for (int j = i + 1; j < W && j < i + lookahead; j++) {
             double d = fabs((double)x[j] - (double)x[j - 1]);
             if (d > m) m = d;
         }
@@ -479,7 +479,7 @@ static int64_t encode_line(const float *x, int W, int A, seg_t *segs, int *nseg_
             int j = i + 1, overflow = 0;
             nd = nd0;
             while (j < W) {
-                if (j % A == 0 && rep_len(run, j, W, A) >= 16) break;
+                if (j % A == 0 && rep_len(run, j, W, A) >= repeat_min) break;
                 double t = ldexp((double)x[j] - (double)prev, -emin);
                 if (fabs(t) > 1984.5) { overflow = 1; break; }
                 int b = quantise(t);
@@ -514,6 +514,8 @@ size_t orc_deepcam_max_encoded_size(int C, int H, int W) {
 }
 
 int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *dst, size_t cap, size_t *size);
+int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, uint8_t *dst,
+                         size_t cap, size_t *size);
 
 int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t cap, size_t *size) {
     return orc_deepcam_encode_a(x, C, H, W, orc_deepcam_align(W), dst, cap, size);
@@ -521,7 +523,15 @@ int orc_deepcam_encode(const float *x, int C, int H, int W, uint8_t *dst, size_t
 
 /* same policy with an explicit alignment A (W % A == 0) */
 int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_deepcam_encode_p(x, C, H, W, A, 64, 16, dst, cap, size);
+}
+
+/* ... and explicit policy knobs: the emin lookahead window and the shortest
+ * REPEAT run (FORMAT.md 2.4 uses 64 and 16) */
+int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, uint8_t *dst,
+                         size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
+    if (lookahead < 2 || lookahead > 65535 || repeat_min < 2 || repeat_min > 65535) return ORC_EINVAL;
     if ((uint64_t)C * H > 0xFFFFFFFFull || A < 1 || W % A != 0) return ORC_EINVAL;
     init_mags();
     uint64_t L = (uint64_t)C * H;
@@ -539,7 +549,7 @@ int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *ds
         uint64_t sz = raw_size;
         if (finite) {
             int nseg; int64_t nd;
-            int64_t seg_size = encode_line(xl, W, A, segs, &nseg, NULL, &nd, run);
+            int64_t seg_size = encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, NULL, &nd, run);
             if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
         }
         pay += sz;
@@ -562,7 +572,7 @@ int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *ds
         int finite = 1;
         for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
         int nseg = 0; int64_t nd = 0;
-        int64_t seg_size = finite ? encode_line(xl, W, A, segs, &nseg, deltas, &nd, run) : -1;
+        int64_t seg_size = finite ? encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) : -1;
         if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
             p[0] = 1; wr16(p + 2, (uint16_t)nseg);
             for (int s = 0; s < nseg; s++) {

@@ -124,6 +124,15 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         "l"(src), "r"(bytes), "r"(smem_u32(bar))
         : "memory");
 }
+// 16-B asynchronous shared store whose completion counts on `bar` (st.async,
+// complete_tx): a producer hands a small record to a consumer through the same
+// mbarrier that tracks the consumer's TMA bytes
+__device__ __forceinline__ void st_async_u4(uint32_t saddr, uint4 v, uint64_t *bar) {
+    asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                     saddr),
+                 "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(smem_u32(bar))
+                 : "memory");
+}
 // explicit shared-memory loads through 32-bit shared addresses (LDS, never generic LD)
 __device__ __forceinline__ uint2 lds_u2(uint32_t a) {
     uint2 r;

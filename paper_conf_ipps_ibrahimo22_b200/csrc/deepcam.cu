@@ -837,7 +837,7 @@ static_assert(kWsNs >= 2 && kWsNs <= 8, "slot ring");
 constexpr uint32_t kWsCtl = 32 * kWsNs;  // per consumer: full[NS], empty[NS] mbarriers + info[NS] (16 B each)
 
 template <int OUT, bool VEC, int VPL>
-__global__ void __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
+__global__ void __cluster_dims__(1, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
     uint32_t *__restrict__ status) {
@@ -854,7 +854,10 @@ __global__ void __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws
 
     if (warp == wpc && lane < wpc) {
         uint64_t *c = ctl(lane);
-        for (uint32_t i = 0; i < 2 * kWsNs; i++) mbar_init(&c[i], 1);  // full[NS]: producer + TMA bytes; empty[NS]: consumer lane 0
+        for (uint32_t i = 0; i < kWsNs; i++) {
+            mbar_init(&c[i], 1);            // full[i]: the producer lane's arrival + the TMA bytes
+            mbar_init(&c[kWsNs + i], kWarp);  // empty[i]: every consumer lane (each has read the slot)
+        }
         fence_mbar_init();
     }
     __syncthreads();
@@ -933,13 +936,12 @@ __global__ void __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws
                         ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
                 }
                 if (ready) {
-                    sts_u4(smem_u32(&info[s]), make_uint4(e_bytes, e_flags, __float_as_uint(shv), __float_as_uint(scv)));
-                    if (e_bytes) {
-                        mbar_arrive_expect_tx(&full[s], e_bytes);
-                        bulk_g2s(big ? rb : rb + s * cap, e_src, e_bytes, &full[s]);  // (s: this line's slot)
-                    } else {
-                        mbar_arrive(&full[s]);  // nothing to copy: the consumer skips the line
-                    }
+                    // the line record (16 B, st.async) and its bytes (TMA) both count
+                    // on full[s]; a zero-byte line delivers only the record
+                    mbar_arrive_expect_tx(&full[s], e_bytes + 16u);
+                    st_async_u4(smem_u32(&info[s]),
+                                make_uint4(e_bytes, e_flags, __float_as_uint(shv), __float_as_uint(scv)), &full[s]);
+                    if (e_bytes) bulk_g2s(big ? rb : rb + s * cap, e_src, e_bytes, &full[s]);
                     const uint32_t took = big ? (1u << kWsNs) - 1u : 1u << s;
                     par ^= took & used;
                     used |= took;
@@ -1002,14 +1004,15 @@ __global__ void __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws
             }
             if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
         }
+        if constexpr (VPL == 36) {
+            if (lane == 0) bulk_wait_read_all();  // the staged row has left the slot
+        }
         __syncwarp();
-        if (lane == 0) {
-            if constexpr (VPL == 36) bulk_wait_read_all();  // the staged row has left the slot
-            if (flags & 1u) {
-                for (uint32_t i = 0; i < kWsNs; i++) mbar_arrive(&empty[i]);  // the line took the whole ring
-            } else {
-                mbar_arrive(&empty[s]);
-            }
+        // every lane releases: its own reads of the slot and of info[s] precede its arrival
+        if (flags & 1u) {
+            for (uint32_t i = 0; i < kWsNs; i++) mbar_arrive(&empty[i]);  // the line took the whole ring
+        } else {
+            mbar_arrive(&empty[s]);
         }
     }
     if constexpr (VPL == 36) {

@@ -67,10 +67,15 @@ inline int alignment_for(int W) { return W == 1152 ? 36 : (W % 8 == 0 ? 8 : 1); 
 
 struct LineEncoder {
     int W, A;
+    int lookahead, repeat_min;  // FORMAT.md 2.4 policy knobs (defaults 64, 16)
     std::vector<int> run;
     std::vector<Seg> segs;
     std::vector<uint8_t> deltas;
-    LineEncoder(int w, int a) : W(w), A(a), run(w), segs(), deltas() { segs.reserve(w); deltas.reserve(w); }
+    LineEncoder(int w, int a, int la, int rm)
+        : W(w), A(a), lookahead(la), repeat_min(rm), run(w), segs(), deltas() {
+        segs.reserve(w);
+        deltas.reserve(w);
+    }
 
     int rep(int i) const {
         const int r = run[i];
@@ -86,14 +91,14 @@ struct LineEncoder {
         int i = 0;
         while (i < W) {
             const int rl = rep(i);
-            if (rl >= kRepeatMin) {
+            if (rl >= repeat_min) {
                 segs.push_back(Seg{(uint16_t)rl, kRepeat, 0, x[i]});
                 i += rl;
                 continue;
             }
             const float h = x[i];
             double m = 0.0;
-            const int jend = (i + kLookahead < W) ? i + kLookahead : W;
+            const int jend = (i + lookahead < W) ? i + lookahead : W;
             for (int j = i + 1; j < jend; j++) {
                 double d = fabs((double)x[j] - (double)x[j - 1]);
                 if (d > m) m = d;
@@ -113,7 +118,7 @@ struct LineEncoder {
                 int j = i + 1;
                 bool overflow = false;
                 for (; j < W; j++) {
-                    if (j % A == 0 && rep(j) >= kRepeatMin) break;
+                    if (j % A == 0 && rep(j) >= repeat_min) break;
                     double t = ldexp((double)x[j] - (double)prev, -emin);
                     if (fabs(t) > kMaxCode + 0.5) { overflow = true; break; }
                     int k;
@@ -152,14 +157,22 @@ extern "C" size_t spp_deepcam_max_encoded_size(int C, int H, int W) {
 
 extern "C" spp_status spp_encode_deepcam(const float *x, int C, int H, int W, void *dst,
                                          size_t dst_capacity, size_t *encoded_size) {
+    return spp_encode_deepcam_ex(x, C, H, W, nullptr, dst, dst_capacity, encoded_size);
+}
+
+extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W, const spp_deepcam_params *params,
+                                            void *dst, size_t dst_capacity, size_t *encoded_size) {
     if (!x || !encoded_size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535)
         return SPP_ERR_INVALID_ARG;
+    const int la = params && params->lookahead ? params->lookahead : kLookahead;
+    const int rm = params && params->repeat_min ? params->repeat_min : kRepeatMin;
+    if (la < 2 || la > 65535 || rm < 2 || rm > 65535) return SPP_ERR_INVALID_ARG;
     const uint64_t L = (uint64_t)C * H;
     const uint64_t dir_off = spp::kHeaderBytes;
     const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
     const uint64_t raw_size = round_up16(16 + 4 * (uint64_t)W);
     const int A = alignment_for(W);
-    LineEncoder enc(W, A);
+    LineEncoder enc(W, A, la, rm);
     // pass 1: per-line size (SEG vs RAW)
     std::vector<uint8_t> is_seg(L);
     std::vector<uint32_t> dir(L + 1);

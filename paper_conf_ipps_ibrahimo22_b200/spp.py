@@ -27,6 +27,7 @@ OUT = {"f16": SPP_OUT_F16, "f32": SPP_OUT_F32, "i16": SPP_OUT_I16}
 # every symbol include/spp.h declares (checked by tests/test_host.py)
 EXPORTS = (
     "spp_cosmo_max_encoded_size", "spp_encode_cosmo", "spp_deepcam_max_encoded_size", "spp_encode_deepcam",
+    "spp_encode_deepcam_ex",
     "spp_stream_info", "spp_decode_opts_init", "spp_decode_workspace_size", "spp_decoded_sample_bytes",
     "spp_decode_batch", "spp_decode_launches", "spp_pipeline_create", "spp_pipeline_destroy", "spp_decode_host",
     "spp_pipeline_last_launches", "spp_set_l2_persisting", "spp_status_string", "spp_version",
@@ -37,6 +38,10 @@ class SppError(RuntimeError):
     def __init__(self, code: int, what: str):
         super().__init__(f"{what}: {spp_status_string(code)} ({code})")
         self.code = code
+
+
+class spp_deepcam_params(C.Structure):
+    _fields_ = [("lookahead", C.c_int), ("repeat_min", C.c_int)]
 
 
 class spp_decode_opts(C.Structure):
@@ -64,6 +69,7 @@ def load() -> C.CDLL:
         "spp_encode_cosmo": ([P, I, I, I, I, P, SZ, C.POINTER(SZ)], I),
         "spp_deepcam_max_encoded_size": ([I, I, I], SZ),
         "spp_encode_deepcam": ([P, I, I, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_encode_deepcam_ex": ([P, I, I, I, C.POINTER(spp_deepcam_params), P, SZ, C.POINTER(SZ)], I),
         "spp_stream_info": ([I, P, SZ, C.POINTER(I64)], I),
         "spp_decode_opts_init": ([C.POINTER(spp_decode_opts), I, I, I, I, I], None),
         "spp_decode_workspace_size": ([I, I, C.POINTER(spp_decode_opts)], SZ),
@@ -122,8 +128,9 @@ def spp_deepcam_max_encoded_size(Cc: int, H: int, W: int) -> int:
     return int(load().spp_deepcam_max_encoded_size(Cc, H, W))
 
 
-def spp_encode_deepcam(x: np.ndarray) -> np.ndarray:
-    """fp32 [C, H, W] -> encoded uint8 stream (FORMAT.md 2)."""
+def spp_encode_deepcam(x: np.ndarray, lookahead: int = 0, repeat_min: int = 0) -> np.ndarray:
+    """fp32 [C, H, W] -> encoded uint8 stream (FORMAT.md 2); nonzero knobs go
+    through spp_encode_deepcam_ex (0 = the FORMAT.md 2.4 default)."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     if a.ndim != 3:
         raise ValueError("x must be [C, H, W]")
@@ -131,8 +138,13 @@ def spp_encode_deepcam(x: np.ndarray) -> np.ndarray:
     cap = spp_deepcam_max_encoded_size(Cc, H, W)
     dst = np.empty(max(cap, 64), dtype=np.uint8)
     size = C.c_size_t(0)
-    _check(load().spp_encode_deepcam(a.ctypes.data, Cc, H, W, dst.ctypes.data, dst.size, C.byref(size)),
-           "spp_encode_deepcam")
+    if lookahead or repeat_min:
+        prm = spp_deepcam_params(int(lookahead), int(repeat_min))
+        _check(load().spp_encode_deepcam_ex(a.ctypes.data, Cc, H, W, C.byref(prm), dst.ctypes.data, dst.size,
+                                            C.byref(size)), "spp_encode_deepcam_ex")
+    else:
+        _check(load().spp_encode_deepcam(a.ctypes.data, Cc, H, W, dst.ctypes.data, dst.size, C.byref(size)),
+               "spp_encode_deepcam")
     return dst[: size.value].copy()
 
 

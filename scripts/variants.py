@@ -10,12 +10,11 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kd_ws0": ["SPP_KD_WS=0"],
-    "kd_ns2": ["SPP_KD_WS_NS=2"],
     "kd_ns3": ["SPP_KD_WS_NS=3"],
-    "kd_ns4_10x2": ["SPP_KD_WS_NS=4", "SPP_KD_WS_WPC=10"],
-    "kd_ns3_7x3": ["SPP_KD_WS_NS=3", "SPP_KD_WS_WPC=7", "SPP_KD_WS_MINB=3"],
-    "kd_ns3_23x1": ["SPP_KD_WS_NS=3", "SPP_KD_WS_WPC=23", "SPP_KD_WS_MINB=1"],
+    "kd_ns3_s2304": ["SPP_KD_WS_NS=3", "SPP_KD_WS_SLOT=2304"],
+    "kd_ns4_s2304": ["SPP_KD_WS_NS=4", "SPP_KD_WS_SLOT=2304"],
+    "kd_ns3_s3072": ["SPP_KD_WS_NS=3", "SPP_KD_WS_SLOT=3072"],
+    "kd_ns3b": ["SPP_KD_WS_NS=3", "SPP_KD_TAG=1"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 

@@ -123,3 +123,29 @@ def test_deepcam_encoder_bound_on_product_streams(spp, orc):
         xh = orc.deepcam_decode_line(b, l, 200)
         if info["mode"] == 1:
             _check_bound(x[0, l], xh, info["segs"])
+
+
+@pytest.mark.parametrize("lookahead,repeat_min", [(2, 2), (8, 16), (36, 4), (300, 64), (1152, 2)])
+def test_deepcam_encoder_knobs_match_oracle_and_bound(spp, orc, lookahead, repeat_min):
+    """the policy knobs of spp_encode_deepcam_ex (FORMAT.md 2.4)
+    give byte-identical streams from the product and the oracle encoders, and
+    every SEG line stays within the per-value bound (reading S19, P11)."""
+    from synth import gen_deepcam
+    from tests.test_oracle_pins import _check_bound
+    x = gen_deepcam(2003, H=12)
+    a = spp.spp_encode_deepcam(x, lookahead, repeat_min)
+    b = orc.deepcam_encode(x, lookahead=lookahead, repeat_min=repeat_min)
+    assert a.size == b.size and np.array_equal(a, b)
+    h = fmt.deepcam_header(a)
+    for l in range(0, h["L"], 7):
+        info = fmt.deepcam_line(a, h, l)
+        if info["mode"] == 1:
+            assert all(s["kind"] == 1 or s["len"] >= repeat_min for s in info["segs"])  # REPEAT runs
+            _check_bound(x.reshape(-1, x.shape[-1])[l], orc.deepcam_decode_line(a, l, x.shape[-1]), info["segs"])
+
+
+def test_deepcam_encoder_knob_errors(spp):
+    x = np.zeros((1, 1, 8), np.float32)
+    for la, rm in ((1, 16), (64, 1), (70000, 16), (64, -3)):
+        with pytest.raises(spp.SppError):
+            spp.spp_encode_deepcam(x, la, rm)
