@@ -178,7 +178,9 @@ void spp_pipeline_destroy(spp_pipeline *p);
  *               (the pipeline owns its workspace)
  * All work is enqueued on `stream` (decode) and the pipeline's copy stream; the
  * call returns when everything is enqueued (it may block only while the
- * staging ring is full). */
+ * staging ring is full).  Samples of one chunk that lie back to back in host
+ * memory (h_src[k+1] == h_src[k] + src_bytes[k]) are copied with one
+ * transfer. */
 spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size_t *src_bytes,
                            int n, void *d_dst, const spp_decode_opts *opts, spp_stream_t stream);
 

@@ -837,7 +837,7 @@ static_assert(kWsNs >= 2 && kWsNs <= 8, "slot ring");
 constexpr uint32_t kWsCtl = 32 * kWsNs;  // per consumer: full[NS], empty[NS] mbarriers + info[NS] (16 B each)
 
 template <int OUT, bool VEC, int VPL>
-__global__ void __cluster_dims__(1, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
     uint32_t *__restrict__ status) {
@@ -1045,7 +1045,9 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
         return SPP_ERR_CUDA;
     const uint64_t lines = (uint64_t)n * o.C * o.H;
     const uint64_t max_ctas = (uint64_t)dp.sms * occ;
-    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
+    // st.async needs a cluster of at least 2 CTAs (they never touch each other's memory): even grid
+    int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
+    grid += grid & 1;
     kern<<<grid, (wpc + 1) * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift,
                                                      o.scale, static_cast<uint8_t *>(d_dst), cap, nwords, warp_bytes,
                                                      o.status);

@@ -128,15 +128,29 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
         uint8_t *stage = p->d_stage + (size_t)slot * p->slot_bytes;
         size_t off = 0;
         int k = 0;
+        // samples that sit back to back in host memory travel as one copy
+        // (large PCIe transfers run closer to the link rate than per-sample ones)
+        const uint8_t *run_src = nullptr;
+        size_t run_off = 0, run_len = 0;
         while (i + k < n && k < p->max_chunk && off + src_bytes[i + k] <= p->slot_bytes) {
+            const uint8_t *h = static_cast<const uint8_t *>(h_src[i + k]);
             hp[k] = stage + off;
             hs[k] = src_bytes[i + k];
-            if (cudaMemcpyAsync(stage + off, h_src[i + k], src_bytes[i + k], cudaMemcpyHostToDevice, p->copy) !=
-                cudaSuccess)
-                return SPP_ERR_CUDA;
+            if (run_len && h == run_src + run_len) {
+                run_len += src_bytes[i + k];
+            } else {
+                if (run_len && cudaMemcpyAsync(stage + run_off, run_src, run_len, cudaMemcpyHostToDevice, p->copy) !=
+                                   cudaSuccess)
+                    return SPP_ERR_CUDA;
+                run_src = h;
+                run_off = off;
+                run_len = src_bytes[i + k];
+            }
             off += src_bytes[i + k];
             k++;
         }
+        if (run_len && cudaMemcpyAsync(stage + run_off, run_src, run_len, cudaMemcpyHostToDevice, p->copy) != cudaSuccess)
+            return SPP_ERR_CUDA;
         const void **dp = p->d_ptrs + (size_t)slot * p->max_chunk;
         uint64_t *ds = p->d_sizes + (size_t)slot * p->max_chunk;
         if (cudaMemcpyAsync(dp, hp, k * sizeof(void *), cudaMemcpyHostToDevice, p->copy) != cudaSuccess ||

@@ -421,3 +421,36 @@ def test_host_pipeline_matches_device_decode(dev, fmt_name):
         assert torch.equal(out[i].view(torch.int16), ref[i % 5].view(torch.int16))
     assert pipe.launches() == 2 * ((len(host) + 1) // 2)
     pipe.close()
+
+
+@pytest.mark.parametrize("fmt_name", ["cosmo", "deepcam"])
+def test_host_pipeline_coalesced_runs(dev, fmt_name):
+    """spp_decode_host copies samples that lie back to back in host memory as
+    one transfer: a packed pinned pool (runs that break at the pool wrap and
+    at chunk and slot boundaries) decodes exactly like the device path."""
+    from synth import gen_cosmo, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, HostPipeline, spp
+    if fmt_name == "cosmo":
+        bs = [spp.spp_encode_cosmo(gen_cosmo(1101 + i, n=48)) for i in range(4)]
+        dims = (4, 48, 48, 48)
+    else:
+        bs = [spp.spp_encode_deepcam(gen_deepcam(2101 + i, H=40)) for i in range(4)]
+        dims = (16, 40, 1152)
+    offs = np.concatenate([[0], np.cumsum([b.size for b in bs])]).astype(np.int64)
+    packed = torch.empty(int(offs[-1]), dtype=torch.uint8).pin_memory()
+    for i, b in enumerate(bs):
+        packed[int(offs[i]):int(offs[i + 1])].copy_(torch.from_numpy(b))
+    views = [packed[int(offs[i]):int(offs[i + 1])] for i in range(4)]
+    order = [0, 1, 2, 3, 0, 1, 3, 2, 2, 3, 0, 1, 2]
+    host = [views[i] for i in order]
+    dec = Decoder(fmt_name, dims)
+    ref = dec.decode([_to_dev(b) for b in bs])
+    for max_chunk, slot in ((3, 3 * max(b.size for b in bs)), (8, 2 * max(b.size for b in bs) + 64)):
+        pipe = HostPipeline(dec, slot_bytes=slot, nslots=2, max_chunk=max_chunk)
+        out = dec.alloc_out(len(host))
+        pipe.decode(host, out)
+        torch.cuda.synchronize()
+        assert int(dec.status.item()) == 0
+        for j, i in enumerate(order):
+            assert torch.equal(out[j].view(torch.int16), ref[i].view(torch.int16)), (max_chunk, j)
+        pipe.close()
