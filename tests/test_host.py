@@ -149,3 +149,18 @@ def test_deepcam_encoder_knob_errors(spp):
     for la, rm in ((1, 16), (64, 1), (70000, 16), (64, -3)):
         with pytest.raises(spp.SppError):
             spp.spp_encode_deepcam(x, la, rm)
+
+
+def test_cosmo_ratio_vs_gzip_matches_paper(spp):
+    """PAPER.md P:98 "roughly 4x, compared with a 5x compression using the
+    general-purpose gzip" and P:219 "the gzipped files are roughly 75% the size
+    of our encoded samples": on the paper-shaped generator, zlib level 6 (gzip's
+    default) of the TFRecord layout (channels-last int16) vs our stream."""
+    import zlib
+    from synth import gen_cosmo
+    x = gen_cosmo(1001)
+    ours = spp.spp_encode_cosmo(x).size
+    gz = len(zlib.compress(np.ascontiguousarray(np.moveaxis(x, 0, -1)).tobytes(), 6))
+    assert 3.3 < x.nbytes / ours < 4.5          # "roughly 4x"
+    assert 4.5 < x.nbytes / gz < 5.5            # gzip "5x"
+    assert 0.65 < gz / ours < 0.85              # "roughly 75%"
