@@ -74,6 +74,24 @@ size_t spp_cosmo_max_encoded_size(int C, int D, int H, int W);
 spp_status spp_encode_cosmo(const int16_t *counts, int C, int D, int H, int W,
                             void *dst, size_t dst_capacity, size_t *encoded_size);
 
+/* CosmoFlow encoder policy (FORMAT.md 1.3 / 1.4).
+ *   localize : 0 (default) = one table for the whole volume, halved along z
+ *              only while a table would exceed 65,536 groups (FORMAT.md 1.3);
+ *              1 = "localized lookup tables" (multiple tables
+ *              P:100): the dyadic z-partition with the fewest encoded bytes,
+ *              so slabs whose groups fit 256 take 1-byte keys.  Never
+ *              larger than localize = 0.  Any other value -> SPP_ERR_INVALID_ARG.
+ * Both policies write FORMAT.md v1 streams; the decoders are unchanged. */
+typedef struct {
+    int localize;
+} spp_cosmo_params;
+
+/* spp_encode_cosmo with an explicit policy (params may be NULL = defaults);
+ * spp_cosmo_max_encoded_size bounds both policies. */
+spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, int H, int W,
+                               const spp_cosmo_params *params, void *dst, size_t dst_capacity,
+                               size_t *encoded_size);
+
 /* Upper bound of spp_encode_deepcam's output for C x H x W. */
 size_t spp_deepcam_max_encoded_size(int C, int H, int W);
 

@@ -57,6 +57,7 @@ def lib():
         L.orc_cosmo_direct.argtypes = [P, I64, I, I, P]; L.orc_cosmo_direct.restype = I
         L.orc_cosmo_max_encoded_size.argtypes = [I, I, I]; L.orc_cosmo_max_encoded_size.restype = SZ
         L.orc_cosmo_encode.argtypes = [P, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_cosmo_encode.restype = I
+        L.orc_cosmo_encode_ex.argtypes = [P, I, I, I, I, P, SZ, C.POINTER(SZ)]; L.orc_cosmo_encode_ex.restype = I
         L.orc_cosmo_decode.argtypes = [P, SZ, I, I, P, I, I, I, I]; L.orc_cosmo_decode.restype = I
         L.orc_deepcam_code.argtypes = [I]; L.orc_deepcam_code.restype = I
         L.orc_deepcam_decode_line.argtypes = [P, SZ, I, P]; L.orc_deepcam_decode_line.restype = I
@@ -104,14 +105,16 @@ def cosmo_direct(counts: np.ndarray, transform: int = 1, out: str = "f16") -> np
     return o
 
 
-def cosmo_encode(counts: np.ndarray) -> np.ndarray:
+def cosmo_encode(counts: np.ndarray, localize: bool = False) -> np.ndarray:
+    """FORMAT.md 1.3 encoder; `localize` selects the 1.4 localized-table policy."""
     a = np.ascontiguousarray(counts, dtype=np.int16)
     assert a.ndim == 4 and a.shape[0] == 4
     _, D, H, W = a.shape
     cap = lib().orc_cosmo_max_encoded_size(D, H, W)
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
-    _check(lib().orc_cosmo_encode(_p(a), D, H, W, _p(dst), cap, C.byref(size)), "cosmo_encode")
+    _check(lib().orc_cosmo_encode_ex(_p(a), D, H, W, int(localize), _p(dst), cap, C.byref(size)),
+           "cosmo_encode")
     return dst[: size.value].copy()
 
 

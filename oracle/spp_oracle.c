@@ -160,13 +160,52 @@ static void split_slabs(const uint64_t *tup, int64_t plane, int z0, int z1, uint
     (*nout)++;
 }
 
+/* FORMAT.md 1.4 ("localized lookup tables", "multiple lookup
+ * tables", P:106 1-byte keys): bytes of [z0,z1) written as one slab — its
+ * 32-B table entry plus LUT and keys, or the RAW planes (rules of 1.3). */
+static uint64_t slab_bytes(int64_t G, int64_t Nt) {
+    int kw = G == 1 ? 0 : (G <= 256 ? 1 : 2);
+    if (G > 65536 || 8 * G + kw * Nt >= 8 * Nt) return 32 + up16(8 * (uint64_t)Nt);
+    return 32 + up16(8 * (uint64_t)G) + (kw ? up16((uint64_t)kw * (uint64_t)Nt) : 0);
+}
+
+/* FORMAT.md 1.4: among the partitions reachable by halving [z0,z1) at
+ * z0 + (z1-z0)/2, the one with the fewest bytes; the whole slab is kept unless
+ * the halves are strictly smaller.  Appends the slabs in z order. */
+static uint64_t split_localized(const uint64_t *tup, int64_t plane, int z0, int z1, uint64_t *scratch,
+                                zrange_t *out, int *nout) {
+    int64_t g = count_groups(tup, plane, z0, z1, scratch);
+    uint64_t whole = slab_bytes(g, (int64_t)(z1 - z0) * plane);
+    if (z1 - z0 > 1) {
+        int mid = z0 + (z1 - z0) / 2;
+        int n0 = *nout;
+        uint64_t halves = split_localized(tup, plane, z0, mid, scratch, out, nout);
+        halves += split_localized(tup, plane, mid, z1, scratch, out, nout);
+        if (halves < whole) return halves;
+        *nout = n0;                     /* drop the halves, keep the whole slab */
+    }
+    out[*nout].z0 = z0;
+    out[*nout].z1 = z1;
+    (*nout)++;
+    return whole;
+}
+
 size_t orc_cosmo_max_encoded_size(int D, int H, int W) {
     uint64_t N = (uint64_t)D * H * W;
     /* header + U + slab table + worst case per slab: RAW planes (8 B/voxel) */
     return (size_t)(64 + up16(2 * 32768) + up16(32 * (uint64_t)D) + 8 * N + 16 * (uint64_t)D + 64);
 }
 
+int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize, uint8_t *dst, size_t cap,
+                        size_t *size);
 int orc_cosmo_encode(const int16_t *counts, int D, int H, int W, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_cosmo_encode_ex(counts, D, H, W, 0, dst, cap, size);
+}
+
+/* FORMAT.md 1.3 (localize = 0) or 1.4 (localize = 1) */
+int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize, uint8_t *dst, size_t cap,
+                        size_t *size) {
+    if (localize != 0 && localize != 1) return ORC_EINVAL;
     if (!counts || !size || D < 1 || H < 1 || W < 1 || D > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     const int C = 4;
     int64_t plane = (int64_t)H * W, N = (int64_t)D * plane;
@@ -190,7 +229,8 @@ int orc_cosmo_encode(const int16_t *counts, int D, int H, int W, uint8_t *dst, s
     uint64_t *scratch = malloc((size_t)N * 8);
     zrange_t *sl = malloc(sizeof(zrange_t) * (size_t)D);
     int nslab = 0;
-    split_slabs(tup, plane, 0, D, scratch, sl, &nslab);
+    if (localize) split_localized(tup, plane, 0, D, scratch, sl, &nslab);
+    else split_slabs(tup, plane, 0, D, scratch, sl, &nslab);
 
     /* 2. lay out: header, U, slab table, then per slab LUT + keys */
     uint64_t off = 64;

@@ -121,6 +121,39 @@ void split(Ctx &c, int z0, int z1, std::vector<std::pair<int, int>> &out) {
     out.push_back({z0, z1});
 }
 
+// Exact encoded bytes of [z0, z1) as ONE slab (FORMAT.md 1.3 steps 3 and 5):
+// its 32-B slab-table entry + LUT + keys, or the RAW planes of the escape.
+uint64_t slab_cost(int64_t G, int64_t Nt) {
+    const int kw = G == 1 ? 0 : (G <= spp::cosmo::kMaxG1 ? 1 : 2);
+    if (G > spp::cosmo::kMaxG2 || 8 * G + kw * Nt >= 8 * Nt)
+        return spp::cosmo::kSlabBytes + round_up16(8ull * (uint64_t)Nt);
+    return spp::cosmo::kSlabBytes + round_up16(8ull * (uint64_t)G) +
+           (kw ? round_up16((uint64_t)kw * (uint64_t)Nt) : 0);
+}
+
+// FORMAT.md 1.4 localized tables ("localized lookup tables", P:100
+// "multiple lookup tables", P:106 1-byte keys): the z-partition of [z0, z1)
+// into dyadic slabs (same halving as 1.3) with the fewest encoded bytes; a
+// slab is kept whole unless splitting is strictly smaller.  Leaves appended
+// in z order; returns the bytes of the chosen partition.
+uint64_t split_localized(Ctx &c, int z0, int z1, std::vector<std::pair<int, int>> &out) {
+    const int64_t G = count_groups(c, z0, z1);
+    const uint64_t whole = slab_cost(G, (int64_t)(z1 - z0) * c.plane);
+    if (z1 - z0 == 1) {
+        out.push_back({z0, z1});
+        return whole;
+    }
+    const int mid = z0 + (z1 - z0) / 2;
+    std::vector<std::pair<int, int>> parts;
+    const uint64_t halves = split_localized(c, z0, mid, parts) + split_localized(c, mid, z1, parts);
+    if (halves < whole) {
+        out.insert(out.end(), parts.begin(), parts.end());
+        return halves;
+    }
+    out.push_back({z0, z1});
+    return whole;
+}
+
 }  // namespace
 
 extern "C" size_t spp_cosmo_max_encoded_size(int C, int D, int H, int W) {
@@ -132,6 +165,14 @@ extern "C" size_t spp_cosmo_max_encoded_size(int C, int D, int H, int W) {
 
 extern "C" spp_status spp_encode_cosmo(const int16_t *counts, int C, int D, int H, int W, void *dst,
                                        size_t dst_capacity, size_t *encoded_size) {
+    return spp_encode_cosmo_ex(counts, C, D, H, W, nullptr, dst, dst_capacity, encoded_size);
+}
+
+extern "C" spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, int H, int W,
+                                          const spp_cosmo_params *params, void *dst, size_t dst_capacity,
+                                          size_t *encoded_size) {
+    const int localize = params ? params->localize : 0;
+    if (localize != 0 && localize != 1) return SPP_ERR_INVALID_ARG;
     if (!counts || !encoded_size || C != 4 || D < 1 || H < 1 || W < 1 || D > 65535 || H > 65535 ||
         W > 65535)
         return SPP_ERR_INVALID_ARG;
@@ -158,7 +199,10 @@ extern "C" spp_status spp_encode_cosmo(const int16_t *counts, int C, int D, int 
                  ((uint64_t)idx_of[c2[v]] << 16) | (uint64_t)idx_of[c3[v]];
     Ctx ctx{tup.data(), plane, {}, {}};
     std::vector<std::pair<int, int>> ranges;
-    split(ctx, 0, D, ranges);
+    if (localize)
+        split_localized(ctx, 0, D, ranges);
+    else
+        split(ctx, 0, D, ranges);
 
     // 3. per slab: groups ordered by (freq desc, tuple asc), key width, layout
     const int T = (int)ranges.size();

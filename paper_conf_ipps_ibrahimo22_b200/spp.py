@@ -27,7 +27,7 @@ OUT = {"f16": SPP_OUT_F16, "f32": SPP_OUT_F32, "i16": SPP_OUT_I16}
 # every symbol include/spp.h declares (checked by tests/test_host.py)
 EXPORTS = (
     "spp_cosmo_max_encoded_size", "spp_encode_cosmo", "spp_deepcam_max_encoded_size", "spp_encode_deepcam",
-    "spp_encode_deepcam_ex",
+    "spp_encode_deepcam_ex", "spp_encode_cosmo_ex",
     "spp_stream_info", "spp_decode_opts_init", "spp_decode_workspace_size", "spp_decoded_sample_bytes",
     "spp_decode_batch", "spp_decode_launches", "spp_pipeline_create", "spp_pipeline_destroy", "spp_decode_host",
     "spp_pipeline_last_launches", "spp_set_l2_persisting", "spp_status_string", "spp_version",
@@ -38,6 +38,10 @@ class SppError(RuntimeError):
     def __init__(self, code: int, what: str):
         super().__init__(f"{what}: {spp_status_string(code)} ({code})")
         self.code = code
+
+
+class spp_cosmo_params(C.Structure):
+    _fields_ = [("localize", C.c_int)]
 
 
 class spp_deepcam_params(C.Structure):
@@ -67,6 +71,7 @@ def load() -> C.CDLL:
     sig = {
         "spp_cosmo_max_encoded_size": ([I, I, I, I], SZ),
         "spp_encode_cosmo": ([P, I, I, I, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_encode_cosmo_ex": ([P, I, I, I, I, C.POINTER(spp_cosmo_params), P, SZ, C.POINTER(SZ)], I),
         "spp_deepcam_max_encoded_size": ([I, I, I], SZ),
         "spp_encode_deepcam": ([P, I, I, I, P, SZ, C.POINTER(SZ)], I),
         "spp_encode_deepcam_ex": ([P, I, I, I, C.POINTER(spp_deepcam_params), P, SZ, C.POINTER(SZ)], I),
@@ -110,8 +115,9 @@ def spp_cosmo_max_encoded_size(Cc: int, D: int, H: int, W: int) -> int:
     return int(load().spp_cosmo_max_encoded_size(Cc, D, H, W))
 
 
-def spp_encode_cosmo(counts: np.ndarray) -> np.ndarray:
-    """int16 [4, D, H, W] counts -> encoded uint8 stream (FORMAT.md 1)."""
+def spp_encode_cosmo(counts: np.ndarray, localize: bool = False) -> np.ndarray:
+    """int16 [4, D, H, W] counts -> encoded uint8 stream (FORMAT.md 1); with
+    `localize` through spp_encode_cosmo_ex (FORMAT.md 1.4 localized tables)."""
     a = np.ascontiguousarray(counts, dtype=np.int16)
     if a.ndim != 4:
         raise ValueError("counts must be [4, D, H, W]")
@@ -119,8 +125,13 @@ def spp_encode_cosmo(counts: np.ndarray) -> np.ndarray:
     cap = spp_cosmo_max_encoded_size(Cc, D, H, W)
     dst = np.empty(max(cap, 64), dtype=np.uint8)
     size = C.c_size_t(0)
-    _check(load().spp_encode_cosmo(a.ctypes.data, Cc, D, H, W, dst.ctypes.data, dst.size, C.byref(size)),
-           "spp_encode_cosmo")
+    if localize:
+        prm = spp_cosmo_params(1)
+        _check(load().spp_encode_cosmo_ex(a.ctypes.data, Cc, D, H, W, C.byref(prm), dst.ctypes.data, dst.size,
+                                          C.byref(size)), "spp_encode_cosmo_ex")
+    else:
+        _check(load().spp_encode_cosmo(a.ctypes.data, Cc, D, H, W, dst.ctypes.data, dst.size, C.byref(size)),
+               "spp_encode_cosmo")
     return dst[: size.value].copy()
 
 

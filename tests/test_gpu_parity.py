@@ -113,6 +113,36 @@ def test_cosmo_edge_shapes_and_broadcast(dev, orc):
         assert st == 0 and np.array_equal(got[0], x)
 
 
+def test_cosmo_localized_tables(dev, orc):
+    """FORMAT.md 1.4 localized tables (spp_encode_cosmo_ex): many slabs with
+    1-byte keys, mixed kw 0 / 1 / 8 in one stream, a batch mixing both
+    policies; every output bit-exact to the plain definition."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(12)
+    xs = [gen_cosmo(3001, "sparse"), gen_cosmo(3005, "unit", n=64)]
+    v = gen_cosmo(3006, "sparse", n=64)
+    v[:, :16] = 3                                                    # constant slab -> kw 0
+    v[:, 48:] = rng.integers(0, 3000, size=(4, 16, 64, 64))          # dense slab -> RAW escape
+    xs.append(v)
+    for x in xs:
+        b = spp.spp_encode_cosmo(x, localize=True)
+        assert fmt.cosmo_header(b)["T"] > 1 or x.shape[1] < 128
+        for out, tr in (("f16", 1), ("f32", 1), ("i16", 0)):
+            got, st = _decode("cosmo", [b], x.shape, out=out, transform=tr)
+            assert st == 0
+            _same_bits(got[0], orc.cosmo_direct(x, tr, out))
+    kws = {s["kw"] for s in fmt.cosmo_header(spp.spp_encode_cosmo(xs[2], localize=True))["slabs"]}
+    assert {0, 1, 8} <= kws
+    x0 = xs[0]
+    bufs = [spp.spp_encode_cosmo(x0, localize=True), spp.spp_encode_cosmo(x0)] * 3
+    got, st = _decode("cosmo", bufs, x0.shape, out="f16")
+    assert st == 0
+    want = orc.cosmo_direct(x0, 1, "f16")
+    for g in got:
+        _same_bits(g, want)
+
+
 def test_cosmo_oracle_encoded_stream(dev, orc):
     """The GPU decodes a stream written by the oracle's own encoder."""
     from synth import gen_cosmo

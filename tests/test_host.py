@@ -52,6 +52,36 @@ def test_cosmo_encoder_matches_oracle_bytes(spp, orc):
         assert np.array_equal(orc.cosmo_decode(a, x.shape, 0, "i16"), x)
 
 
+def test_cosmo_localized_encoder_matches_oracle_bytes(spp, orc):
+    """FORMAT.md 1.4 (spp_encode_cosmo_ex localize = 1) is byte-identical to
+    the oracle's localized encoder and never larger than the default."""
+    from synth import gen_cosmo
+    rng = np.random.default_rng(6)
+    vols = [gen_cosmo(3001, "sparse"), gen_cosmo(3003, "unit", n=64), gen_cosmo(3002, "dense", n=64),
+            gen_cosmo(3004, "verysparse", n=32), np.zeros((4, 3, 5, 7), dtype=np.int16),
+            rng.integers(0, 9, size=(4, 7, 3, 5)).astype(np.int16)]
+    for x in vols:
+        a = spp.spp_encode_cosmo(x, localize=True)
+        b = orc.cosmo_encode(x, localize=True)
+        assert a.size == b.size and np.array_equal(a, b)
+        assert a.size <= spp.spp_encode_cosmo(x).size
+        assert np.array_equal(orc.cosmo_decode(a, x.shape, 0, "i16"), x)
+
+
+def test_cosmo_params_errors(spp):
+    import ctypes as C
+    x = np.zeros((4, 2, 2, 2), dtype=np.int16)
+    dst = np.zeros(spp.spp_cosmo_max_encoded_size(4, 2, 2, 2), dtype=np.uint8)
+    size = C.c_size_t(0)
+    for bad in (2, -1):
+        prm = spp.spp_cosmo_params(bad)
+        rc = spp.load().spp_encode_cosmo_ex(x.ctypes.data, 4, 2, 2, 2, C.byref(prm), dst.ctypes.data, dst.size,
+                                            C.byref(size))
+        assert rc == 1
+    rc = spp.load().spp_encode_cosmo_ex(x.ctypes.data, 4, 2, 2, 2, None, dst.ctypes.data, dst.size, C.byref(size))
+    assert rc == 0 and size.value == spp.spp_encode_cosmo(x).size
+
+
 def test_deepcam_encoder_matches_oracle_bytes(spp, orc):
     from synth import gen_deepcam
     rng = np.random.default_rng(4)

@@ -173,6 +173,91 @@ def test_cosmo_slab_split_and_raw_escape(orc):
     assert orc.cosmo_decode(hb, y.shape, 1, "f32").tobytes() == orc.cosmo_direct(y, 1, "f32").tobytes()
 
 
+def _localized_volumes():
+    """Tiny volumes whose groups are local in z ("localized lookup
+    tables"): per-block palettes, a constant block, a dense random block,
+    odd depths (unequal halves)."""
+    rng = np.random.default_rng(11)
+    vols = []
+    for D, H, W, blk, pal in [(8, 8, 8, 2, 100), (8, 16, 16, 4, 200), (7, 8, 8, 1, 45), (6, 12, 12, 3, 150),
+                              (16, 8, 8, 2, 90), (8, 16, 16, 8, 300)]:
+        planes = []
+        for z0 in range(0, D, blk):
+            n = min(blk, D - z0) * H * W
+            base = 1000 * (z0 // blk)
+            gid = base + rng.integers(0, pal, size=n)
+            planes.append(np.array([gid % 97, gid % 89, gid // 89, gid % 13], dtype=np.int16)
+                          .reshape(4, min(blk, D - z0), H, W))
+        vols.append(np.concatenate(planes, axis=1))
+    v = vols[1].copy()
+    v[:, :2] = 5                                                     # a constant slab (kw 0)
+    v[:, 6:] = rng.integers(0, 3000, size=(4, 2, 16, 16))            # dense: RAW escape
+    vols.append(v)
+    vols.append(rng.integers(0, 3, size=(4, 5, 4, 4)).astype(np.int16))
+    return vols
+
+
+def _dyadic_partitions(z0, z1):
+    yield [(z0, z1)]
+    if z1 - z0 > 1:
+        mid = z0 + (z1 - z0) // 2
+        for a in _dyadic_partitions(z0, mid):
+            for b in _dyadic_partitions(mid, z1):
+                yield a + b
+
+
+@pytest.mark.parametrize("vi", range(8))
+def test_cosmo_localized_tables_bruteforce(orc, vi):
+    """FORMAT.md 1.4: the localized stream is the
+    byte-smallest of ALL dyadic z-partitions, each slab laid out by FORMAT.md
+    1.1/1.3 (sizes counted here from brute-force group sets), never larger
+    than the default policy, and decodes losslessly."""
+    x = _localized_volumes()[vi]
+    _, D, H, W = x.shape
+    up16 = lambda v: (v + 15) // 16 * 16
+    plane = H * W
+    flat = x.reshape(4, D * plane)
+    Uidx = {v: i for i, v in enumerate(sorted(set(x.ravel().tolist())))}
+    tup = [tuple(Uidx[int(flat[c, v])] for c in range(4)) for v in range(D * plane)]
+
+    def slab_layout(z0, z1):
+        Nt = (z1 - z0) * plane
+        G = len(set(tup[z0 * plane: z1 * plane]))
+        kw = 0 if G == 1 else (1 if G <= 256 else 2)
+        if G > 65536 or 8 * G + kw * Nt >= 8 * Nt:
+            return 32 + up16(8 * Nt), 8
+        return 32 + up16(8 * G) + (up16(kw * Nt) if kw else 0), kw
+
+    head = 64 + up16(2 * len(Uidx))
+    costs = {tuple(p): sum(slab_layout(*r)[0] for r in p) for p in _dyadic_partitions(0, D)}
+    best = min(costs.values())
+    b = orc.cosmo_encode(x, localize=True)
+    h = fmt.cosmo_header(b)
+    part = tuple((s["z0"], s["z1"]) for s in h["slabs"])
+    assert b.size == h["total"] == head + best
+    assert costs[part] == best
+    # the whole slab is kept when splitting does not strictly save bytes
+    assert not (len(part) > 1 and costs[((0, D),)] == best)
+    for s in h["slabs"]:
+        assert s["kw"] == slab_layout(s["z0"], s["z1"])[1]
+    assert b.size <= orc.cosmo_encode(x).size
+    assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
+    assert orc.cosmo_decode(b, x.shape, 1, "f16").tobytes() == orc.cosmo_direct(x, 1, "f16").tobytes()
+
+
+def test_cosmo_localized_tables_take_one_byte_keys(orc):
+    """Sparse paper-like volume (few hundred groups overall, < 256 per 16-plane
+    slab): localized slabs take 1-byte keys and the stream shrinks ~2x."""
+    from synth import gen_cosmo
+    x = gen_cosmo(3001, "sparse")
+    a, b = orc.cosmo_encode(x), orc.cosmo_encode(x, localize=True)
+    ha, hb = fmt.cosmo_header(a), fmt.cosmo_header(b)
+    assert ha["T"] == 1 and ha["slabs"][0]["kw"] == 2
+    assert hb["T"] > 1 and all(s["kw"] in (0, 1) for s in hb["slabs"])
+    assert b.size < 0.55 * a.size
+    assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
+
+
 def test_cosmo_size_closed_form_and_paper_ratio(orc):
     """P:98 'compression factor of roughly 4x' vs gzip 5x; P:219 gzip files are
     'roughly 75%' of ours.  Layout size = 64 + up16(2|U|) + 32 + up16(8G) + 2N."""
