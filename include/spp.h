@@ -110,11 +110,20 @@ spp_status spp_encode_deepcam(const float *x, int C, int H, int W,
  *                errors next to abrupt changes, more segments).  2..65535.
  *   repeat_min : shortest run of bit-identical values that opens a REPEAT
  *                segment (default 16).  2..65535.
+ *   rel_err    : relative-error threshold of the error budget (default 0.1,
+ *                the paper's "larger than 10% error"); > 0 and finite.
+ *   err_budget : FORMAT.md 2.5 error budget (default 0 = off).  k > 0: a line
+ *                whose SEG encoding has k or more values with
+ *                |x̂ - x| > rel_err |x| (S19) is written RAW, i.e.
+ *                kept uncompressed ("areas with abrupt changes are kept
+ *                uncompressed").  Trades bytes for fewer large errors.
  * A zero field selects its default.  Every setting obeys the per-value
  * error bound of DESIGN.md reading S19 and decodes on the unchanged decoders. */
 typedef struct {
     int lookahead;
     int repeat_min;
+    float rel_err;
+    int err_budget;
 } spp_deepcam_params;
 
 /* spp_encode_deepcam with explicit policy knobs (params may be NULL = defaults);

@@ -568,10 +568,45 @@ int orc_deepcam_encode_a(const float *x, int C, int H, int W, int A, uint8_t *ds
 
 /* ... and explicit policy knobs: the emin lookahead window and the shortest
  * REPEAT run (FORMAT.md 2.4 uses 64 and 16) */
+int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, uint8_t *dst, size_t cap, size_t *size);
 int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, uint8_t *dst,
                          size_t cap, size_t *size) {
+    return orc_deepcam_encode_q(x, C, H, W, A, lookahead, repeat_min, 0.1f, 0, dst, cap, size);
+}
+
+/* FORMAT.md 2.5 ("areas with abrupt changes are kept uncompressed";
+ * P:86 "roughly 3% of the values with larger than 10% error"): the number of
+ * values of an encoded SEG line whose relative error exceeds rel (DESIGN.md
+ * S19: |x̂ - x| > rel |x|, so x = 0 counts iff x̂ != 0), x̂ rebuilt from the
+ * segments and codes exactly as the decoder of FORMAT.md 2.3 does. */
+static int line_bad_count(const float *x, const seg_t *segs, int nseg, const uint8_t *deltas, double rel) {
+    int bad = 0, pos = 0;
+    int64_t d = 0;
+    for (int s = 0; s < nseg; s++) {
+        float h = segs[s].head;
+        if (segs[s].kind == 0) {
+            for (int j = 0; j < segs[s].len; j++) if (fabs((double)h - (double)x[pos + j]) > rel * fabs((double)x[pos + j])) bad++;
+        } else {
+            float unit = ldexpf(1.0f, segs[s].emin_b - 150);
+            int64_t S = 0;
+            if (fabs((double)h - (double)x[pos]) > rel * fabs((double)x[pos])) bad++;
+            for (int j = 1; j < segs[s].len; j++) {
+                S += orc_deepcam_code(deltas[d++]);
+                float xh = h + (float)S * unit;
+                if (fabs((double)xh - (double)x[pos + j]) > rel * fabs((double)x[pos + j])) bad++;
+            }
+        }
+        pos += segs[s].len;
+    }
+    return bad;
+}
+
+int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, uint8_t *dst, size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     if (lookahead < 2 || lookahead > 65535 || repeat_min < 2 || repeat_min > 65535) return ORC_EINVAL;
+    if (err_budget < 0 || !(rel_err > 0.0f) || !(rel_err < 1e30f)) return ORC_EINVAL;
     if ((uint64_t)C * H > 0xFFFFFFFFull || A < 1 || W % A != 0) return ORC_EINVAL;
     init_mags();
     uint64_t L = (uint64_t)C * H;
@@ -589,7 +624,9 @@ int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahe
         uint64_t sz = raw_size;
         if (finite) {
             int nseg; int64_t nd;
-            int64_t seg_size = encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, NULL, &nd, run);
+            int64_t seg_size = encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run);
+            if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget)
+                seg_size = -1;                            /* over the error budget: RAW (FORMAT.md 2.5) */
             if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
         }
         pay += sz;
@@ -613,6 +650,8 @@ int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahe
         for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
         int nseg = 0; int64_t nd = 0;
         int64_t seg_size = finite ? encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) : -1;
+        if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget)
+            seg_size = -1;
         if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
             p[0] = 1; wr16(p + 2, (uint16_t)nseg);
             for (int s = 0; s < nseg; s++) {

@@ -141,6 +141,33 @@ struct LineEncoder {
     }
 };
 
+// FORMAT.md 2.5 error budget (P:82 abrupt areas kept uncompressed, P:86 the
+// "> 10% error" statistic): values of the line just encoded whose relative
+// error exceeds rel (S19: |x̂ - x| > rel |x|), x̂ rebuilt from the
+// segments and codes by the decoder's arithmetic (FORMAT.md 2.3).
+int bad_values(const LineEncoder &e, const float *x, double rel) {
+    int bad = 0, pos = 0;
+    size_t d = 0;
+    auto over = [&](float xh, float xv) { return fabs((double)xh - (double)xv) > rel * fabs((double)xv); };
+    for (const Seg &g : e.segs) {
+        if (g.kind == kRepeat) {
+            for (int j = 0; j < g.len; j++) bad += over(g.head, x[pos + j]);
+        } else {
+            const float unit = ldexpf(1.0f, (int)g.emin_b - kEminBias);
+            int64_t S = 0;
+            bad += over(g.head, x[pos]);
+            for (int j = 1; j < g.len; j++) {
+                const uint8_t b = e.deltas[d++];
+                const int mag = kCodes.mag[b & 127];
+                S += (b & 0x80) ? -mag : mag;
+                bad += over(g.head + (float)S * unit, x[pos + j]);
+            }
+        }
+        pos += g.len;
+    }
+    return bad;
+}
+
 inline bool all_finite(const float *x, int W) {
     for (int k = 0; k < W; k++)
         if (!isfinite(x[k])) return false;
@@ -166,7 +193,10 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
         return SPP_ERR_INVALID_ARG;
     const int la = params && params->lookahead ? params->lookahead : kLookahead;
     const int rm = params && params->repeat_min ? params->repeat_min : kRepeatMin;
+    const float rel = params && params->rel_err != 0.0f ? params->rel_err : 0.1f;
+    const int budget = params ? params->err_budget : 0;
     if (la < 2 || la > 65535 || rm < 2 || rm > 65535) return SPP_ERR_INVALID_ARG;
+    if (budget < 0 || !(rel > 0.0f) || !(rel < 1e30f)) return SPP_ERR_INVALID_ARG;
     const uint64_t L = (uint64_t)C * H;
     const uint64_t dir_off = spp::kHeaderBytes;
     const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
@@ -182,7 +212,8 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
         uint64_t sz = raw_size;
         is_seg[l] = 0;
         if (all_finite(xl, W)) {
-            const int64_t seg = enc.encode(xl);
+            int64_t seg = enc.encode(xl);
+            if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) seg = -1;  // FORMAT.md 2.5
             if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
         }
         if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;

@@ -43,13 +43,15 @@ def main():
     precip = [c for c in range(C) if DEEPCAM_CHANNELS[c % len(DEEPCAM_CHANNELS)][0] == "precipitation"]
     dec = Decoder("deepcam", (C, H, W), out="f32")
     rows = []
-    settings = [(la, 0) for la in (4, 8, 16, 36, 64, 128, 256, 1152)] + [(64, 4), (64, 64)]
-    for la, rm in settings:
+    settings = [(la, 0, 0) for la in (4, 8, 16, 36, 64, 128, 256, 1152)] + [(64, 4, 0), (64, 64, 0)]
+    # FORMAT.md 2.5 error budget: a line with >= k values above 10% error stays RAW
+    settings += [(0, 0, k) for k in (256, 64, 16, 4, 1)]
+    for la, rm, budget in settings:
         nbytes, bad, tot, bad_p, tot_p, med = 0, 0, 0, 0, 0, []
         nseg = 0
         nraw = 0
         for x in xs:
-            b = spp.spp_encode_deepcam(x, la, rm)
+            b = spp.spp_encode_deepcam(x, la, rm, err_budget=budget)
             nbytes += b.size
             info = spp.spp_stream_info("deepcam", b)
             nraw += info[0]
@@ -65,7 +67,8 @@ def main():
             tot_p += r[precip].size
             med.append(float(np.median(r)))
         vals = args.samples * C * H * W
-        rows.append({"lookahead": la, "repeat_min": rm or 16, "bytes_per_value": nbytes / vals,
+        rows.append({"lookahead": la or 64, "repeat_min": rm or 16, "err_budget": budget,
+                     "bytes_per_value": nbytes / vals,
                      "ratio_vs_fp32": 4.0 * vals / nbytes, "frac_rel_err_gt_10pct": bad / tot,
                      "frac_rel_err_gt_10pct_precip_channel": bad_p / max(1, tot_p),
                      "frac_rel_err_gt_10pct_other_channels": (bad - bad_p) / max(1, tot - tot_p),
@@ -73,7 +76,7 @@ def main():
                      "raw_lines": nraw})
         print(json.dumps(rows[-1]), file=sys.stderr, flush=True)
     print(json.dumps({"what": "DeepCAM ratio vs error over encoder knobs (FORMAT.md 2.4 defaults: lookahead 64, "
-                      "repeat_min 16); decoded by libspp on the GPU (fp32 x-hat)",
+                      "repeat_min 16; FORMAT.md 2.5 err_budget k at rel_err 0.1, 0 = off); decoded by libspp on the GPU (fp32 x-hat)",
                       "samples": args.samples, "shape": [C, H, W], "paper": "about 3% of values > 10% error (P:86)",
                       "rows": rows}, indent=1))
 

@@ -232,6 +232,25 @@ def test_deepcam_c3_paper_sample(dev, orc):
     _same_bits(got[0], _dc_ref(orc, b, x.shape, None, None, "f32"))
 
 
+@pytest.mark.parametrize("budget", [1, 16])
+def test_deepcam_error_budget_streams(dev, orc, budget):
+    """FORMAT.md 2.5 error-budget streams (many RAW lines interleaved with SEG
+    lines) on the full-size C3 shape: bit-exact, and RAW lines are x itself."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2006)
+    mean, rstd = deepcam_stats(x)
+    b = spp.spp_encode_deepcam(x, err_budget=budget)
+    raw, seg, _, _ = spp.spp_stream_info("deepcam", b)
+    assert raw > 100 and seg > 100
+    got, st = _decode("deepcam", [b, spp.spp_encode_deepcam(x)], x.shape, out="f16", shift=mean, scale=rstd)
+    assert st == 0
+    _same_bits(got[0], _dc_ref(orc, b, x.shape, mean, rstd, "f16"))
+    got, st = _decode("deepcam", [b], x.shape, out="f32")
+    assert st == 0
+    _same_bits(got[0], _dc_ref(orc, b, x.shape, None, None, "f32"))
+
+
 def test_deepcam_oracle_encoded_stream(dev, orc):
     from synth import gen_deepcam
     x = gen_deepcam(2002, H=64)

@@ -174,11 +174,24 @@ def test_deepcam_encoder_knobs_match_oracle_and_bound(spp, orc, lookahead, repea
             _check_bound(x.reshape(-1, x.shape[-1])[l], orc.deepcam_decode_line(a, l, x.shape[-1]), info["segs"])
 
 
+@pytest.mark.parametrize("rel,budget", [(0.1, 1), (0.1, 32), (0.05, 4), (0.5, 200)])
+def test_deepcam_error_budget_matches_oracle(spp, orc, rel, budget):
+    """FORMAT.md 2.5 error budget: product == oracle bytes."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2005, H=16)
+    a = spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget)
+    b = orc.deepcam_encode(x, rel_err=rel, err_budget=budget)
+    assert a.size == b.size and np.array_equal(a, b)
+
+
 def test_deepcam_encoder_knob_errors(spp):
     x = np.zeros((1, 1, 8), np.float32)
     for la, rm in ((1, 16), (64, 1), (70000, 16), (64, -3)):
         with pytest.raises(spp.SppError):
             spp.spp_encode_deepcam(x, la, rm)
+    for rel, budget in ((-0.1, 1), (float("nan"), 1), (float("inf"), 1), (0.1, -1)):
+        with pytest.raises(spp.SppError):
+            spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget)
 
 
 def test_cosmo_ratio_vs_gzip_matches_paper(spp):

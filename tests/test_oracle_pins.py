@@ -489,6 +489,42 @@ def test_deepcam_paper_statistic(orc):
     assert x.nbytes / b.size > 3.0                     # it compresses
 
 
+@pytest.mark.parametrize("rel,budget", [(0.1, 1), (0.1, 8), (0.1, 64), (0.01, 16)])
+def test_deepcam_error_budget(orc, rel, budget):
+    """FORMAT.md 2.5 (P:82 abrupt areas kept uncompressed, P:86 the "> 10%
+    error" statistic): exactly the lines whose default SEG encoding has
+    `budget` or more values with |x̂ - x| > rel |x| (counted here with numpy
+    on the oracle's decode) become RAW, and no other line changes."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2004, H=24)
+    C, H, W = x.shape
+    b0 = orc.deepcam_encode(x)
+    b1 = orc.deepcam_encode(x, rel_err=rel, err_budget=budget)
+    h0, h1 = fmt.deepcam_header(b0), fmt.deepcam_header(b1)
+    x64 = x.astype(np.float64)
+    switched = 0
+    for l in range(C * H):
+        c, y = divmod(l, H)
+        i0, i1 = fmt.deepcam_line(b0, h0, l), fmt.deepcam_line(b1, h1, l)
+        xh0 = orc.deepcam_decode_line(b0, l, W).astype(np.float64)
+        nbad = int((np.abs(xh0 - x64[c, y]) > np.float64(np.float32(rel)) * np.abs(x64[c, y])).sum())
+        if i0["mode"] == 1 and nbad >= budget:
+            assert i1["mode"] == 0                                          # kept uncompressed
+            assert np.array_equal(orc.deepcam_decode_line(b1, l, W).view(np.uint32), x[c, y].view(np.uint32))
+            switched += 1
+        else:
+            assert i1 == i0                                                 # untouched
+    assert switched > 0 and b1.size > b0.size
+    # the statistic falls: values above 10% error in the budgeted stream
+    xh1 = orc.deepcam_decode(b1, x.shape, out="f32").astype(np.float64)
+    xh0 = orc.deepcam_decode(b0, x.shape, out="f32").astype(np.float64)
+    bad1 = (np.abs(xh1 - x64) > 0.1 * np.abs(x64)).mean()
+    bad0 = (np.abs(xh0 - x64) > 0.1 * np.abs(x64)).mean()
+    assert bad1 < bad0
+    if rel == 0.1:
+        assert bad1 <= budget / W + 1e-12                                   # per-line cap holds on average
+
+
 def test_deepcam_special_shapes(orc):
     for (C, H, W) in ((1, 1, 1), (1, 3, 2), (2, 2, 17), (1, 1, 16)):
         x = np.random.default_rng(C * 100 + W).standard_normal((C, H, W)).astype(np.float32)
