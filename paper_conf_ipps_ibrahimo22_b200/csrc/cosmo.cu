@@ -79,7 +79,11 @@ constexpr int kStageBytes = kTileVox * 2;
 #define SPP_KC_LA 1
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
-constexpr int kColdSlotBytes = (kColdLA + 1) * kConsumers * 16;  // 2 rows per thread per tile in flight
+#ifndef SPP_KC_COLD_SLOTS
+#define SPP_KC_COLD_SLOTS 2
+#endif
+constexpr int kColdSlots = SPP_KC_COLD_SLOTS;             // LUT rows per thread per tile fetched ahead
+constexpr int kColdSlotBytes = (kColdLA + 1) * kConsumers * kColdSlots * 8;
 constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes + 2 * kKeyStages * 8;
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
@@ -362,40 +366,40 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         return ring.buf + (gt % kKeyStages) * kStageBytes;
     };
     // Cold rows: while tile t is expanded, the thread classifies its keys of
-    // tile t + kColdLA and starts LDGSTS copies (cp.async) of up to two cold LUT
-    // rows into its own shared-memory slots; one copy group per tile, so the
-    // rows of tile t are waited for (per thread, no barrier) kColdLA tiles later.
-    // cj[t % (kColdLA+1)] = (j0 | j1 << 8) cold positions of that tile (8 = none).
+    // tile t + kColdLA and starts LDGSTS copies (cp.async) of its first
+    // kColdSlots cold LUT rows into its own shared-memory slots; one copy group
+    // per tile, so the rows of tile t are waited for (per thread, no barrier)
+    // kColdLA tiles later.  cj[] = the 8-bit cold mask of each tile in flight;
+    // the i-th cold position of a tile reads slot i (i < kColdSlots).
     uint32_t cj[kColdLA + 1];
 #pragma unroll
-    for (int i = 0; i <= kColdLA; i++) cj[i] = 0x0808u;
-    auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k (0/1) of this thread for tile t
-        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * 2 + k) * 8;
+    for (int i = 0; i <= kColdLA; i++) cj[i] = 0u;
+    auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k of this thread for tile t
+        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * kColdSlots + k) * 8;
     };
     auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
-        uint32_t j0 = 8, j1 = 8;
+        uint32_t cold = 0;
         if (q < b) {
             const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
             const Keys8 k = keys_from_smem(stage, kwb);
-            uint32_t cold = 0;
 #pragma unroll
             for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
 #if SPP_KC_DIAG_NOCOLD
             cold = 0;
 #endif
-            if (cold) {
-                j0 = __ffs(cold) - 1;
-                cp_async8(slot_addr(t, 0), sv.lut + 8ull * min(k.get_dyn(j0), Gm1));
-                cold &= cold - 1;
-                if (cold) {
-                    j1 = __ffs(cold) - 1;
-                    cp_async8(slot_addr(t, 1), sv.lut + 8ull * min(k.get_dyn(j1), Gm1));
+            uint32_t m = cold;
+#pragma unroll
+            for (int i = 0; i < kColdSlots; i++) {
+                if (m) {
+                    const uint32_t j = __ffs(m) - 1;
+                    cp_async8(slot_addr(t, i), sv.lut + 8ull * min(k.get_dyn(j), Gm1));
+                    m &= m - 1;
                 }
             }
         }
         cp_async_commit();
-        return j0 | (j1 << 8);
+        return cold;
     };
     if constexpr (kProducerWarp) {
         // The producer warp keeps the ring full for the whole call: it refills a
@@ -430,10 +434,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             cp_async_commit();  // keep one group per iteration
         }
         cp_async_wait<kColdLA>();  // the copies of tile t have landed (this thread's)
-        const uint32_t cjt = cj[0];
+        const uint32_t cmask = cj[0];
 #pragma unroll
         for (int i = 0; i < kColdLA; i++) cj[i] = cj[i + 1];  // rotate (compile-time indices)
-        const uint32_t cj0 = cjt & 0xFFu, cj1 = cjt >> 8;
         const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         if (q < b) {
@@ -450,9 +453,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     e[j] = lds_entry<OUT>(hot_base + g * EB);
                 } else {
                     bad |= g > Gm1;
-                    const uint2 lv = (uint32_t)j == cj0 ? lds_u2(slot_addr(t, 0))
-                                     : (uint32_t)j == cj1 ? lds_u2(slot_addr(t, 1))
-                                                          : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // 3rd+: rare
+                    const uint32_t si = __popc(cmask & ((1u << j) - 1u));  // rank among the tile's cold keys
+                    const uint2 lv = si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
+                                                               : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }
             }

@@ -27,6 +27,7 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--policies", default="default,localized",
                     help="encoder policies per preset: default (FORMAT.md 1.3), localized (1.4)")
+    ap.add_argument("--only", default="", help="comma-separated preset names to run (default: all)")
     a = ap.parse_args()
     grid = [(lam, rho) for lam in (0.01, 0.05, 1.0, 2.0, 16.0, 64.0) for rho in (0.9, 0.7, 0.0)]
     rows = []
@@ -34,6 +35,8 @@ def main():
         if (Path(__file__).resolve().parent.parent / "MEASURED_PEAKS.json").exists() else 6650.0
     cases = [("zeros", None, None)] + [(f"lam{lam}_rho{rho}", lam, rho) for lam, rho in grid]
     policies = a.policies.split(",")
+    if a.only:
+        cases = [c for c in cases if c[0] in a.only.split(",")]
     for name, lam, rho in cases:
         if lam is None:
             xs = [np.zeros((4, 128, 128, 128), dtype=np.int16)]

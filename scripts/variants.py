@@ -10,11 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kd_ns3": ["SPP_KD_WS_NS=3"],
-    "kd_ns3_s2304": ["SPP_KD_WS_NS=3", "SPP_KD_WS_SLOT=2304"],
-    "kd_ns4_s2304": ["SPP_KD_WS_NS=4", "SPP_KD_WS_SLOT=2304"],
-    "kd_ns3_s3072": ["SPP_KD_WS_NS=3", "SPP_KD_WS_SLOT=3072"],
-    "kd_ns3b": ["SPP_KD_WS_NS=3", "SPP_KD_TAG=1"],
+    "kc_conv": [],
+    "kc_noconv": ["SPP_KC_COLD_CONVERT=0"],
+    "kc_conv_k3": ["SPP_KC_COLD_SLOTS=3", "SPP_KC_HOT_KB=120"],
+    "kc_conv_k4": ["SPP_KC_COLD_SLOTS=4", "SPP_KC_HOT_KB=108"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
@@ -55,6 +54,14 @@ def run():
                 res[name].update({"deepcam": d["value"], "dfrac": d["roofline"]["frac"]})
             except Exception as ex:
                 res[name]["derror"] = str(ex)
+        if os.environ.get("VARIANT_SWEEP"):
+            out = subprocess.run([sys.executable, str(ROOT / "scripts" / "sweep.py"), "--pool", "2", "--steps", "10",
+                                  "--only", os.environ["VARIANT_SWEEP"]], env=env, capture_output=True, text=True)
+            try:
+                rows = json.loads(out.stdout)["rows"]
+                res[name]["sweep"] = {f'{r["preset"]}/{r["policy"]}': round(r["frac_of_measured_hbm"], 3) for r in rows}
+            except Exception as ex:
+                res[name]["serror"] = str(ex) + out.stderr[-300:]
         print(name, res[name], flush=True)
     print(json.dumps(res))
 
