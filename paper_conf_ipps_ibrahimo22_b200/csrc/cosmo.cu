@@ -229,15 +229,18 @@ struct SlabView {
     const uint8_t *keys;
 };
 
-__device__ __forceinline__ SlabView read_slab(const uint8_t *b, int t) {
-    const uint8_t *sl = b + ld_le64(b + kSlabOff) + (uint64_t)kSlabBytes * t;
+// slab table entry t (32 B, 16-B aligned and bounds-checked by KC0; the
+// stream is little-endian like the device): two 16-B read-only loads
+__device__ __forceinline__ SlabView read_slab(const uint8_t *b, uint64_t slab_off, int t) {
+    const uint8_t *sl = b + slab_off + (uint64_t)kSlabBytes * t;
+    const uint4 w0 = ld_ro_u4(sl), w1 = ld_ro_u4(sl + 16);
     SlabView v;
-    v.z0 = ld_le32(sl);
-    v.z1 = ld_le32(sl + 4);
-    v.G = ld_le32(sl + 8);
-    v.kw = sl[12];
-    v.lut = b + ld_le64(sl + 16);
-    v.keys = b + ld_le64(sl + 24);
+    v.z0 = w0.x;
+    v.z1 = w0.y;
+    v.G = w0.z;
+    v.kw = (int)(w0.w & 0xFFu);
+    v.lut = b + ((uint64_t)w1.y << 32 | w1.x);
+    v.keys = b + ((uint64_t)w1.w << 32 | w1.z);
     return v;
 }
 
@@ -401,18 +404,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         cp_async_commit();
         return cold;
     };
-    if constexpr (kProducerWarp) {
-        // The producer warp keeps the ring full for the whole call: it refills a
-        // stage as soon as the last consumer warp releases it, independent of
-        // any consumer's own progress (an issuing consumer would lag the others).
-        if (threadIdx.x >= (uint32_t)kConsumers) {
-            if (threadIdx.x == (uint32_t)kConsumers)
-                for (uint32_t t = 0; t < ntiles; t++) issue(t);
-            __syncwarp();
-            ring.count += ntiles;
-            return;
-        }
-    } else if (threadIdx.x == 0) {
+    // (with kProducerWarp the key tiles are issued by kc_produce, which runs
+    // ahead of the consumers across segments, items and samples)
+    if (!kProducerWarp && threadIdx.x == 0) {
         for (uint32_t t = 0; t < ntiles && t < (uint32_t)(kKeyStages - 1); t++) issue(t);
     }
 #pragma unroll
@@ -468,6 +462,59 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     ring.count += ntiles;
 }
 
+// The producer warp's whole life (VEC kernel with kProducerWarp): walk the
+// same (item, slab) segments as the consumers, in the same order, and stream
+// every key tile they will expand through the ring, refilling a stage the
+// moment the last consumer warp releases it.  It never waits on the consumers'
+// hot-prefix rebuilds, so the next segment's first tiles are already in shared
+// memory when the consumers get there (no ring drain between segments).
+// (Inlined: as a __noinline__ call the kernel ran 13% slower on C2.)
+__device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, const CosmoMeta *__restrict__ meta,
+                                           KeyRing ring, uint64_t i0, uint64_t i1, uint32_t items_per_sample,
+                                           uint64_t chunk, uint64_t N, uint64_t plane) {
+    uint32_t gt = 0;  // CTA-global tile index, same sequence as the consumers' ring.count
+#pragma unroll 1
+    for (uint64_t it = i0; it < i1; it++) {
+        const int s = (int)(it / items_per_sample);
+        const uint64_t v0 = (it % items_per_sample) * chunk;
+        const uint64_t v1 = min(N, v0 + chunk);
+        const CosmoMeta m = meta[s];
+        if (!m.valid || 4u * m.nU > (uint32_t)kRegionBytes / 2) continue;  // consumers take the scalar path
+        const uint8_t *b = static_cast<const uint8_t *>(src[s]);
+        const uint64_t slab_off = ld_le64(b + kSlabOff);
+#pragma unroll 1
+        for (uint32_t t = 0; t < m.nslab; t++) {
+            const SlabView sv = read_slab(b, slab_off, t);
+            const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
+            const uint64_t a = max(v0, sa), e = min(v1, sb);
+            if (a >= e || (sv.kw != 1 && sv.kw != 2)) continue;
+            const uint32_t kwb = (uint32_t)sv.kw;
+            const uint64_t ra = a - sa, rb = e - sa;
+            const uint32_t ntiles = (uint32_t)((rb - ra + kTileVox - 1) / kTileVox);
+#pragma unroll 1
+            for (uint32_t k = 0; k < ntiles; k++, gt++) {
+                const uint32_t stg = gt % kKeyStages;
+                if (gt >= (uint32_t)kKeyStages) mbar_wait(&ring.empty[stg], ((gt / kKeyStages) - 1) & 1u);
+                const uint64_t st = ra + (uint64_t)k * kTileVox;
+                const uint64_t rem = rb - st;
+                const uint32_t nvox = rem < (uint64_t)kTileVox ? (uint32_t)rem : (uint32_t)kTileVox;
+                const uint32_t bytes = (nvox * kwb + 15u) & ~15u;
+                fence_proxy_async_smem();
+                mbar_arrive_expect_tx(&ring.full[stg], bytes);
+                bulk_g2s(ring.buf + stg * kStageBytes, sv.keys + st * kwb, bytes, &ring.full[stg]);
+            }
+        }
+    }
+}
+
+// CTA-wide barrier of the threads that run the item loop: all of them, or the
+// consumer warps only when the producer warp has split off (named barrier 1)
+template <bool SPLIT>
+__device__ __forceinline__ void loop_sync() {
+    if constexpr (SPLIT) asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory");
+    else __syncthreads();
+}
+
 template <int OUT, bool VEC>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *const *__restrict__ src, int n,
                                                          const float *__restrict__ fU_ws,
@@ -498,6 +545,15 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     const uint64_t per = (total_items + gridDim.x - 1) / gridDim.x;
     const uint64_t i0 = (uint64_t)blockIdx.x * per;
     const uint64_t i1 = min(total_items, i0 + per);
+    constexpr bool kSplit = VEC && kProducerWarp;        // producer warp streams keys, consumers expand
+    constexpr uint32_t kLoopThreads = kSplit ? (uint32_t)kConsumers : (uint32_t)kThreads;
+    if constexpr (kSplit) {
+        if (threadIdx.x >= (uint32_t)kConsumers) {
+            if (threadIdx.x == (uint32_t)kConsumers)
+                kc_produce(src, meta, ring, i0, i1, items_per_sample, chunk, N, plane);
+            return;
+        }
+    }
     const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
     int cached_s = -1, cached_t = -1;
     uint32_t n_hot = 0;
@@ -514,9 +570,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
         const FuView fu_g{fu_base, fu.global, m.nU, false};
         uint8_t *out_s = dst + (uint64_t)s * 4 * N * ob;
         uint32_t bad = 0;  // corrupt key / index seen by this thread in this item
+        const uint64_t slab_off = ld_le64(b + kSlabOff);
 #pragma unroll 1
         for (uint32_t t = 0; t < m.nslab; t++) {
-            const SlabView sv = read_slab(b, t);
+            const SlabView sv = read_slab(b, slab_off, t);
             const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
             const uint64_t a = max(v0, sa), e = min(v1, sb);
             if (a >= e) continue;
@@ -524,7 +581,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                 if (cached_s != s || cached_t != (int)t) {
                     // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples;
                     // the LUT tail (cold groups) is prefetched into L2 for the cold lookups
-                    __syncthreads();
+                    loop_sync<kSplit>();
 #if SPP_KC_PREFETCH_TAIL
                     if (threadIdx.x == 0 && sv.G > hot_cap) {  // (hot_cap: nominal prefix size)
                         const uint64_t off = 8ull * hot_cap, end = 8ull * sv.G;
@@ -536,8 +593,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     }
 #endif
                     if (cached_s != s && fu.in_smem)
-                        for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
-                    __syncthreads();
+                        for (uint32_t i = threadIdx.x; i < m.nU; i += kLoopThreads) sts_f32(fu_base + 4 * i, fu.global[i]);
+                    loop_sync<kSplit>();
                     const uint32_t fu_bytes = fu.in_smem ? (4u * m.nU + 15u) & ~15u : 0u;
                     hot_base = region + fu_bytes;
                     // hot prefix: as many tuples as fit, but not more than this CTA's
@@ -547,29 +604,29 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     const uint32_t amort = span / 8 > 4096 ? (uint32_t)min(span / 8, (uint64_t)0xFFFFFFFFu) : 4096u;
                     n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes) / EB), amort);
 #pragma unroll 1
-                    for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * blockDim.x) {
+                    for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * kLoopThreads) {
                         uint2 lv[4];
 #pragma unroll
                         for (int u = 0; u < 4; u++) {
-                            const uint32_t g = g0 + u * blockDim.x;
+                            const uint32_t g = g0 + u * kLoopThreads;
                             if (g < n_hot) lv[u] = ld_ro_u2(sv.lut + 8ull * g);
                         }
 #pragma unroll
                         for (int u = 0; u < 4; u++) {
-                            const uint32_t g = g0 + u * blockDim.x;
+                            const uint32_t g = g0 + u * kLoopThreads;
                             if (g < n_hot)
                                 sts_entry<OUT>(hot_base + g * EB, fu.in_smem ? make_entry<OUT, true>(lv[u], fu, bad)
                                                                              : make_entry<OUT, false>(lv[u], fu, bad));
                         }
                     }
-                    __syncthreads();
+                    loop_sync<kSplit>();
                     cached_s = s;
                     cached_t = (int)t;
                 }
                 if (VEC && fu.in_smem) {
                     if constexpr (VEC) expand_keys_vec<OUT>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad, ring);
                 } else {  // scalar path: odd shapes, or |U| too large for shared memory
-                    for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
+                    for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) {
                         const uint64_t rel = v - sa;
                         uint32_t g = sv.kw == 2 ? ld_le16(sv.keys + 2 * rel) : sv.keys[rel];
                         bad |= g >= sv.G;
@@ -586,22 +643,22 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     E e8[8];
 #pragma unroll
                     for (int j = 0; j < 8; j++) e8[j] = en;
-                    for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)blockDim.x * 8)
+                    for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)kLoopThreads * 8)
                         store8<OUT>(out_s, N, q, e8);
                 } else {
-                    for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) store1<OUT>(out_s, N, v, en);
+                    for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) store1<OUT>(out_s, N, v, en);
                 }
             } else if (VEC && fu.in_smem) {
                 // RAW escape slab: four planes of U indices (FORMAT.md 1.1, kw = 8), 8 voxels per thread
                 if (cached_s != s) {
-                    __syncthreads();
-                    for (uint32_t i = threadIdx.x; i < m.nU; i += blockDim.x) sts_f32(fu_base + 4 * i, fu.global[i]);
-                    __syncthreads();
+                    loop_sync<kSplit>();
+                    for (uint32_t i = threadIdx.x; i < m.nU; i += kLoopThreads) sts_f32(fu_base + 4 * i, fu.global[i]);
+                    loop_sync<kSplit>();
                     cached_s = s;
                     cached_t = -1;
                 }
                 const uint64_t Nt = sb - sa;
-                for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)blockDim.x * 8) {
+                for (uint64_t q = a + (uint64_t)threadIdx.x * 8; q < e; q += (uint64_t)kLoopThreads * 8) {
                     const uint64_t rel = q - sa;
                     uint4 pc[4];
 #pragma unroll
@@ -622,7 +679,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
             } else {
                 // RAW escape slab: four planes of U indices (FORMAT.md 1.1, kw = 8)
                 const uint64_t Nt = sb - sa;
-                for (uint64_t v = a + threadIdx.x; v < e; v += blockDim.x) {
+                for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) {
                     const uint64_t rel = v - sa;
                     uint2 ent;
                     ent.x = (uint32_t)ld_le16(sv.keys + 2 * rel) | ((uint32_t)ld_le16(sv.keys + 2 * (Nt + rel)) << 16);

@@ -10,10 +10,7 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_conv": [],
-    "kc_noconv": ["SPP_KC_COLD_CONVERT=0"],
-    "kc_conv_k3": ["SPP_KC_COLD_SLOTS=3", "SPP_KC_HOT_KB=120"],
-    "kc_conv_k4": ["SPP_KC_COLD_SLOTS=4", "SPP_KC_HOT_KB=108"],
+    "kc_whole": [],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
