@@ -345,8 +345,16 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as td
+        # one process per GPU over NCCL.  SPP_DIST_BACKEND=gloo (tests only) lets
+        # several ranks share one GPU: the device is local_rank modulo the count
+        backend = os.environ.get("SPP_DIST_BACKEND", "nccl")
+        if backend != "nccl":
+            local_rank %= max(1, torch.cuda.device_count())
         torch.cuda.set_device(local_rank)
-        td.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if backend == "nccl":
+            td.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            td.init_process_group(backend)
         dist = td
     res, bufs, stats = run_gpu(args, rank, world, local_rank, dist)
     sec = None

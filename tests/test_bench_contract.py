@@ -50,3 +50,26 @@ def test_gpu_arm_contract():
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["gpu_launches"] == 2 * d["steps"]
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+
+
+@pytest.mark.gpu
+def test_gpu_arm_two_ranks():
+    """The multi-rank path of bench.py (torchrun, one process per rank, barrier +
+    MAX over ranks, whole-job throughput) with two ranks sharing this GPU over
+    gloo (the driver's scaling run uses NCCL, one GPU per rank)."""
+    import os
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    env = dict(os.environ, SPP_DIST_BACKEND="gloo")
+    out = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                          "--master-addr=127.0.0.1", "--master-port=29731", str(ROOT / "bench.py"), "--gpus", "2",
+                          "--batch", "32", "--pool", "2", "--steps", "3", "--warmup", "3", "--e2e-steps", "1"],
+                         capture_output=True, text=True, timeout=900, cwd=str(ROOT), env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["value"] > 0 and d["cpu_baseline"] is None
+    assert d["value"] == pytest.approx(2 * 32 * 3 / (d["ms_per_step"] * 3 / 1e3), rel=1e-6)
+    assert d["e2e"]["value"] > 0 and d["gpu_launches"] == 2 * 3
