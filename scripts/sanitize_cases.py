@@ -34,6 +34,14 @@ print("cosmo ok", run("cosmo", [b, b], x.shape))
 print("cosmo bad keys", run("cosmo", [b, bad], x.shape))
 print("cosmo bad lut", run("cosmo", [lut, b], x.shape, out="f32"))
 print("cosmo truncated", run("cosmo", [b, trunc], x.shape))
+# many slabs (FORMAT.md 1.4 localized tables; kw 0 / 1 / 8 in one stream): the
+# producer warp streams key tiles across slab and sample boundaries
+v = gen_cosmo(3006, "sparse", n=64)
+v[:, :16] = 3
+v[:, 48:] = np.random.default_rng(1).integers(0, 3000, size=(4, 16, 64, 64))
+loc = spp.spp_encode_cosmo(v, localize=True)
+print("cosmo localized", run("cosmo", [loc, spp.spp_encode_cosmo(gen_cosmo(3001, "sparse", n=64), localize=True), loc],
+                             v.shape))
 y = gen_deepcam(2001, H=16)
 d = spp.spp_encode_deepcam(y)
 hd = fmt.deepcam_header(d)
