@@ -10,7 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_whole": [],
+    "kc_base": [],
+    "kc_notail": ["SPP_KC_PREFETCH_TAIL=0"],
+    "kc_hint": ["SPP_KC_COLD_HINT=1"],
+    "kc_hint_notail": ["SPP_KC_COLD_HINT=1", "SPP_KC_PREFETCH_TAIL=0"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
