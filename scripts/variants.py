@@ -10,10 +10,9 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_base": [],
-    "kc_notail": ["SPP_KC_PREFETCH_TAIL=0"],
-    "kc_hint": ["SPP_KC_COLD_HINT=1"],
-    "kc_hint_notail": ["SPP_KC_COLD_HINT=1", "SPP_KC_PREFETCH_TAIL=0"],
+    "kd_rowbuf": [],
+    "kd_rowbuf_s2048": ["SPP_KD_WS_SLOT=2048"],
+    "kd_old": ["SPP_KD_WS_ROWBUF=0", "SPP_KD_WS_SLOT=2560"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
