@@ -194,6 +194,37 @@ def test_cosmo_256_multi_lut(dev, orc):
     _same_bits(got[1], want)
 
 
+def test_cosmo_512_full_simulation_volume(dev, orc):
+    """The paper's full 512^3 simulation histogram (before the 128^3
+    decomposition; "for larger than 128^3 decompositions, multiple lookup
+    tables are required"): 4x512^3 counts (1 GiB) built from 64
+    offset copies of a paper-shaped 128^3 sample, so groups do not repeat
+    across tiles.  Identity output equals the input counts bit for bit over
+    the whole volume; fp16 ln(1+c) equals the oracle's plain definition on
+    every voxel of sampled planes."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    base = gen_cosmo(1001)
+    off = np.arange(64, dtype=np.int16).reshape(4, 4, 4)
+    x = np.empty((4, 512, 512, 512), dtype=np.int16)
+    for tz in range(4):
+        for ty in range(4):
+            for tx in range(4):
+                x[:, tz * 128:(tz + 1) * 128, ty * 128:(ty + 1) * 128, tx * 128:(tx + 1) * 128] = \
+                    base + 7 * off[tz, ty, tx]
+    b = spp.spp_encode_cosmo(x)
+    nU, T, G, kw = spp.spp_stream_info("cosmo", b)
+    assert T > 1
+    got, st = _decode("cosmo", [b], x.shape, out="i16", transform=0)
+    assert st == 0 and np.array_equal(got[0], x)
+    del got
+    got, st = _decode("cosmo", [b], x.shape, out="f16")
+    assert st == 0
+    for z in (0, 127, 128, 255, 300, 511):
+        plane = np.ascontiguousarray(x[:, z:z + 1])
+        _same_bits(got[0][:, z:z + 1], orc.cosmo_direct(plane, 1, "f16"))
+
+
 def test_cosmo_corruption_detected(dev):
     from synth import gen_cosmo
     from paper_conf_ipps_ibrahimo22_b200 import spp
