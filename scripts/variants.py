@@ -10,9 +10,9 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kd_rowbuf": [],
-    "kd_rowbuf_s2048": ["SPP_KD_WS_SLOT=2048"],
-    "kd_old": ["SPP_KD_WS_ROWBUF=0", "SPP_KD_WS_SLOT=2560"],
+    "kc_nored_r80": ["SPP_KC_REDIRECT=0", "SPP_KC_MAXNREG=80"],
+    "kc_red_r80": ["SPP_KC_MAXNREG=80"],
+    "kc_nored": ["SPP_KC_REDIRECT=0"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
