@@ -154,6 +154,13 @@ def cpu_baseline(workload: str, bufs, dims, stats, seconds: float = 12.0):
         return 1
 
     oracle.lib()
+    # (i) one core, one sample at a time, briefly
+    one, t1 = 0, time.perf_counter()
+    while one < 2 or time.perf_counter() - t1 < min(2.0, seconds / 4):
+        work(one)
+        one += 1
+    one_rate = one / (time.perf_counter() - t1)
+    # (ii) every host core, one sample per thread (PAPER.md P:106's CPU assignment)
     done = 0
     t0 = time.perf_counter()
     with ThreadPoolExecutor(max_workers=cores) as ex:
@@ -161,8 +168,10 @@ def cpu_baseline(workload: str, bufs, dims, stats, seconds: float = 12.0):
             done += sum(ex.map(work, range(done, done + cores)))
     dt = time.perf_counter() - t0
     return {"value": done / dt, "unit": "samples/s", "cores": cores, "kind": "oracle",
+            "value_1core": one_rate,
             "sample": f"{done} {workload} samples (oracle/spp_oracle.c sequential decoder, fp16 out), "
-                      f"one per thread on {cores} threads, {dt:.1f} s wall"}
+                      f"one per thread on {cores} threads, {dt:.1f} s wall; value_1core: {one} samples on one "
+                      "thread"}
 
 
 # ----------------------------------------------------------------------------- GPU arm

@@ -10,9 +10,10 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_nored_r80": ["SPP_KC_REDIRECT=0", "SPP_KC_MAXNREG=80"],
-    "kc_red_r80": ["SPP_KC_MAXNREG=80"],
-    "kc_nored": ["SPP_KC_REDIRECT=0"],
+    "kc_t704": ["SPP_KC_THREADS=704"],
+    "kc_t704_h138": ["SPP_KC_THREADS=704", "SPP_KC_HOT_KB=138"],
+    "kc_t640_h144": ["SPP_KC_THREADS=640", "SPP_KC_HOT_KB=144"],
+    "kc_t768": [],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
