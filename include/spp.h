@@ -84,9 +84,14 @@ spp_status spp_encode_cosmo(const int16_t *counts, int C, int D, int H, int W,
  * Both policies write FORMAT.md v1 streams; the decoders are unchanged. */
 typedef struct {
     int localize;
+    int escape_keys;  /* 1 = FORMAT.md 1.5: a slab that would take 2-byte keys stores
+                         1-byte keys with the 255 most frequent groups inline and an
+                         escape list of the rest, when that is smaller (beyond the
+                         paper's 1/2-byte keys); 0 (default) = off */
 } spp_cosmo_params;
 
-/* spp_encode_cosmo with an explicit policy (params may be NULL = defaults);
+/* spp_encode_cosmo with an explicit policy (params may be NULL = defaults;
+ * escape_keys other than 0/1 -> SPP_ERR_INVALID_ARG);
  * spp_cosmo_max_encoded_size bounds both policies. */
 spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, int H, int W,
                                const spp_cosmo_params *params, void *dst, size_t dst_capacity,
@@ -156,6 +161,11 @@ typedef struct {
     void *const *timing_events; /* optional host array of 3 cudaEvent_t, recorded on `stream`
                                    before the prologue kernel, between the prologue and the main
                                    kernel, and after the main kernel (live per-kernel timing) */
+    int escape_keys;         /* CosmoFlow: 1 = the batch may hold FORMAT.md 1.5 escaped-key slabs
+                                (spp_encode_cosmo_ex escape_keys = 1): use the kernel variant that
+                                stages them.  0 (default): the paper-format kernel, which reports
+                                such samples as SPP_ERR_UNSUPPORTED in `status` (odd shapes that
+                                take the scalar kernel decode them either way). */
 } spp_decode_opts;
 
 /* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */

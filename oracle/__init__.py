@@ -107,15 +107,17 @@ def cosmo_direct(counts: np.ndarray, transform: int = 1, out: str = "f16") -> np
     return o
 
 
-def cosmo_encode(counts: np.ndarray, localize: bool = False) -> np.ndarray:
-    """FORMAT.md 1.3 encoder; `localize` selects the 1.4 localized-table policy."""
+def cosmo_encode(counts: np.ndarray, localize: bool = False, escape: bool = False) -> np.ndarray:
+    """FORMAT.md 1.3 encoder; `localize` selects the 1.4 localized-table
+    policy, `escape` the 1.5 escaped 1-byte keys."""
     a = np.ascontiguousarray(counts, dtype=np.int16)
     assert a.ndim == 4 and a.shape[0] == 4
     _, D, H, W = a.shape
     cap = lib().orc_cosmo_max_encoded_size(D, H, W)
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
-    _check(lib().orc_cosmo_encode_ex(_p(a), D, H, W, int(localize), _p(dst), cap, C.byref(size)),
+    _check(lib().orc_cosmo_encode_ex(_p(a), D, H, W, int(localize) | (2 if escape else 0), _p(dst), cap,
+                                     C.byref(size)),
            "cosmo_encode")
     return dst[: size.value].copy()
 

@@ -136,6 +136,30 @@ static int64_t find_u64(const uint64_t *arr, int64_t n, uint64_t key) {
 
 typedef struct { int z0, z1; } zrange_t;
 
+static int cmp_i64_desc(const void *a, const void *b) {
+    int64_t x = *(const int64_t *)a, y = *(const int64_t *)b;
+    return (x < y) - (x > y);
+}
+/* FORMAT.md 1.5: voxels of a slab whose key would be >= 255 (escaped) = all
+ * voxels minus those of the 255 most frequent groups; `sorted` holds the
+ * slab's tuples in ascending order */
+static int64_t escaped_count(const uint64_t *sorted, int64_t Nt, int64_t G) {
+    int64_t *f = malloc(8 * (size_t)G), g = -1, top = 0;
+    for (int64_t i = 0; i < Nt; i++) {
+        if (i == 0 || sorted[i] != sorted[i - 1]) f[++g] = 0;
+        f[g]++;
+    }
+    qsort(f, (size_t)G, 8, cmp_i64_desc);
+    for (int64_t k = 0; k < G && k < 255; k++) top += f[k];
+    free(f);
+    return Nt - top;
+}
+/* FORMAT.md 1.5 key bytes of an escaped-key slab: eidx, low bytes, escapes */
+static uint64_t escaped_bytes(int64_t Nt, int64_t n_esc) {
+    uint64_t nb = ((uint64_t)Nt + 255) / 256;
+    return up16(4 * (nb + 1)) + up16((uint64_t)Nt) + up16(2 * (uint64_t)n_esc);
+}
+
 /* count distinct 4-tuples over planes [z0,z1) */
 static int64_t count_groups(const uint64_t *tup, int64_t plane, int z0, int z1, uint64_t *scratch) {
     int64_t n = (int64_t)(z1 - z0) * plane;
@@ -196,16 +220,17 @@ size_t orc_cosmo_max_encoded_size(int D, int H, int W) {
     return (size_t)(64 + up16(2 * 32768) + up16(32 * (uint64_t)D) + 8 * N + 16 * (uint64_t)D + 64);
 }
 
-int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize, uint8_t *dst, size_t cap,
+int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int policy, uint8_t *dst, size_t cap,
                         size_t *size);
 int orc_cosmo_encode(const int16_t *counts, int D, int H, int W, uint8_t *dst, size_t cap, size_t *size) {
     return orc_cosmo_encode_ex(counts, D, H, W, 0, dst, cap, size);
 }
 
-/* FORMAT.md 1.3 (localize = 0) or 1.4 (localize = 1) */
-int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize, uint8_t *dst, size_t cap,
+/* FORMAT.md 1.3; policy bit 0: 1.4 localized tables, bit 1: 1.5 escaped keys */
+int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int policy, uint8_t *dst, size_t cap,
                         size_t *size) {
-    if (localize != 0 && localize != 1) return ORC_EINVAL;
+    if (policy < 0 || policy > 3) return ORC_EINVAL;
+    const int localize = policy & 1, escape = (policy >> 1) & 1;
     if (!counts || !size || D < 1 || H < 1 || W < 1 || D > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     const int C = 4;
     int64_t plane = (int64_t)H * W, N = (int64_t)D * plane;
@@ -250,9 +275,15 @@ int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize
             for (int64_t i = 0; i < Nt; i++) if (i == 0 || scratch[i] != scratch[i - 1]) G++;
             int kw = G == 1 ? 0 : (G <= 256 ? 1 : 2);
             if (G > 65536 || 8 * G + kw * Nt >= 8 * Nt) { kw = 8; }
+            int64_t n_esc = 0;
+            if (escape && kw == 2) {                     /* FORMAT.md 1.5: escaped 1-byte keys if smaller */
+                n_esc = escaped_count(scratch, Nt, G);
+                if (escaped_bytes(Nt, n_esc) < up16(2 * (uint64_t)Nt)) kw = 3;
+            }
             uint64_t lut_off = 0, keys_off = 0;
             if (kw != 8) { lut_off = cur; cur = up16(cur + 8 * (uint64_t)G); }
-            if (kw != 0) { keys_off = cur; cur = up16(cur + (uint64_t)(kw == 8 ? 8 : kw) * (uint64_t)Nt); }
+            if (kw == 3) { keys_off = cur; cur += escaped_bytes(Nt, n_esc); }
+            else if (kw != 0) { keys_off = cur; cur = up16(cur + (uint64_t)(kw == 8 ? 8 : kw) * (uint64_t)Nt); }
             if (pass == 1) {
                 uint8_t *s = out + slab_off + 32 * (uint64_t)t;
                 wr32(s, (uint32_t)sl[t].z0); wr32(s + 4, (uint32_t)sl[t].z1);
@@ -283,11 +314,20 @@ int orc_cosmo_encode_ex(const int16_t *counts, int D, int H, int W, int localize
                         for (int c = 0; c < C; c++)
                             wr16(out + lut_off + 8 * (uint64_t)k + 2 * (uint64_t)c,
                                  (uint16_t)((grp[k].tup >> (16 * (3 - c))) & 0xFFFFu));
+                    uint64_t nb = ((uint64_t)Nt + 255) / 256;
+                    uint64_t low_off = keys_off + up16(4 * (nb + 1)), esc_off = low_off + up16((uint64_t)Nt);
+                    int64_t seen = 0;
                     for (int64_t v = 0; v < Nt && kw != 0; v++) {
                         int64_t k = key_of[find_u64(uniq, G, tt[v])];
                         if (kw == 1) out[keys_off + (uint64_t)v] = (uint8_t)k;
-                        else wr16(out + keys_off + 2 * (uint64_t)v, (uint16_t)k);
+                        else if (kw == 2) wr16(out + keys_off + 2 * (uint64_t)v, (uint16_t)k);
+                        else {                           /* kw = 3: escape keys >= 255 */
+                            if (v % 256 == 0) wr32(out + keys_off + 4 * ((uint64_t)v / 256), (uint32_t)seen);
+                            out[low_off + (uint64_t)v] = (uint8_t)(k < 255 ? k : 255);
+                            if (k >= 255) wr16(out + esc_off + 2 * (uint64_t)seen++, (uint16_t)k);
+                        }
                     }
+                    if (kw == 3) wr32(out + keys_off + 4 * nb, (uint32_t)seen);
                     free(grp); free(uniq); free(key_of);
                 }
             }
@@ -334,17 +374,38 @@ int orc_cosmo_decode(const uint8_t *src, size_t size, int transform, int out_kin
         if (kw == 0 && G != 1) return ORC_ECORRUPT;
         if (kw == 1 && (G < 1 || G > 256)) return ORC_ECORRUPT;
         if (kw == 2 && (G < 1 || G > 65536)) return ORC_ECORRUPT;
+        if (kw == 3 && (G < 1 || G > 65536)) return ORC_ECORRUPT;
         if (kw == 8 && G != 0) return ORC_ECORRUPT;
-        if (kw != 0 && kw != 1 && kw != 2 && kw != 8) return ORC_ECORRUPT;
+        if (kw != 0 && kw != 1 && kw != 2 && kw != 3 && kw != 8) return ORC_ECORRUPT;
         if (kw != 8 && lut_off + 8 * (uint64_t)G > total) return ORC_ECORRUPT;
-        if (kw != 0 && keys_off + (uint64_t)(kw == 8 ? 8 : kw) * (uint64_t)Nt > total) return ORC_ECORRUPT;
+        /* kw = 3 (FORMAT.md 1.5): eidx u32[nb+1], low u8[Nt], esc u16[eidx[nb]] */
+        uint64_t nb = ((uint64_t)Nt + 255) / 256, low_off = 0, esc_off = 0, n_esc = 0, seen = 0;
+        if (kw == 3) {
+            low_off = keys_off + up16(4 * (nb + 1));
+            esc_off = low_off + up16((uint64_t)Nt);
+            if (esc_off > total || rd32(src + keys_off) != 0) return ORC_ECORRUPT;
+            n_esc = rd32(src + keys_off + 4 * nb);
+            if (esc_off + 2 * n_esc > total) return ORC_ECORRUPT;
+        } else if (kw != 0 && keys_off + (uint64_t)(kw == 8 ? 8 : kw) * (uint64_t)Nt > total) {
+            return ORC_ECORRUPT;
+        }
         for (int64_t v = 0; v < Nt; v++) {
+            uint32_t g = 0;
+            if (kw == 3) {                               /* escaped 1-byte keys, voxel order */
+                if (v % 256 == 0 && rd32(src + keys_off + 4 * ((uint64_t)v / 256)) != seen) return ORC_ECORRUPT;
+                g = src[low_off + (uint64_t)v];
+                if (g == 255) {
+                    if (seen >= n_esc) return ORC_ECORRUPT;
+                    g = rd16(src + esc_off + 2 * seen++);
+                }
+            }
             for (int c = 0; c < C; c++) {
                 uint32_t e;
                 if (kw == 8) {
                     e = rd16(src + keys_off + 2 * ((uint64_t)c * Nt + v));
                 } else {
-                    uint32_t g = kw == 0 ? 0 : (kw == 1 ? src[keys_off + v] : rd16(src + keys_off + 2 * (uint64_t)v));
+                    if (kw != 3)
+                        g = kw == 0 ? 0 : (kw == 1 ? src[keys_off + v] : rd16(src + keys_off + 2 * (uint64_t)v));
                     if (g >= G) return ORC_ECORRUPT;
                     e = rd16(src + lut_off + 8 * (uint64_t)g + 2 * (uint64_t)c);
                 }
@@ -355,6 +416,7 @@ int orc_cosmo_decode(const uint8_t *src, size_t size, int transform, int out_kin
                 if (rc) return rc;
             }
         }
+        if (kw == 3 && seen != n_esc) return ORC_ECORRUPT;
     }
     if (zexp != (uint32_t)D) return ORC_ECORRUPT;
     return ORC_OK;

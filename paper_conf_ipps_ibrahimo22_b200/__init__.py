@@ -35,7 +35,8 @@ class Decoder:
     across calls.
     """
 
-    def __init__(self, fmt: str, dims, out: str = "f16", transform: int | None = None, device=None):
+    def __init__(self, fmt: str, dims, out: str = "f16", transform: int | None = None, device=None,
+                 escape_keys: bool = False):
         import torch
         self.torch = torch
         spp.load()
@@ -44,6 +45,7 @@ class Decoder:
         Cc, D, H, W = (self.dims if fmt == "cosmo" else (self.dims[0], 1, self.dims[1], self.dims[2]))
         self.out = out
         self.opts = spp_decode_opts_init(fmt, Cc, D, H, W, out=out, transform=transform)
+        self.opts.escape_keys = int(bool(escape_keys))  # FORMAT.md 1.5 streams: the staging kernel
         self.device = torch.device(device or "cuda")
         self.status = torch.zeros(1, dtype=torch.int32, device=self.device)
         self._ws = None

@@ -129,10 +129,18 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
                 if (kw == 0) ok = ok && G == 1;
                 else if (kw == 1) ok = ok && G >= 1 && G <= (uint32_t)kMaxG1;
                 else if (kw == 2) ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
+                else if (kw == kEscaped) ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
                 else if (kw == kRawSlab) ok = ok && G == 0;
                 else ok = 0;
                 if (kw != kRawSlab) ok = ok && (lut_off & 15) == 0 && lut_off + 8ull * G <= total;
-                if (kw != 0) ok = ok && (keys_off & 15) == 0 && keys_off + (uint64_t)(kw == kRawSlab ? 8 : kw) * Nt <= total;
+                if (kw == kEscaped) {  // FORMAT.md 1.5: eidx[0] = 0, the escape list inside the stream
+                    const uint64_t nb = (Nt + kEscBlock - 1) / kEscBlock;
+                    const uint64_t esc_off = keys_off + ((4 * (nb + 1) + 15) & ~15ull) + ((Nt + 15) & ~15ull);
+                    ok = ok && (keys_off & 15) == 0 && esc_off <= total && ld_le32(b + keys_off) == 0 &&
+                         esc_off + 2ull * ld_le32(b + keys_off + 4 * nb) <= total;
+                } else if (kw != 0) {
+                    ok = ok && (keys_off & 15) == 0 && keys_off + (uint64_t)(kw == kRawSlab ? 8 : kw) * Nt <= total;
+                }
                 zexp = z1;
             }
             ok = ok && zexp == (uint32_t)D;
@@ -244,6 +252,53 @@ __device__ __forceinline__ SlabView read_slab(const uint8_t *b, uint64_t slab_of
     return v;
 }
 
+__host__ __device__ __forceinline__ uint64_t up16(uint64_t x) { return (x + 15) & ~uint64_t(15); }
+
+// FORMAT.md 1.5 escaped-key slab of Nt voxels: eidx u32[nb+1] at keys, then
+// the low bytes, then the u16 escape list (each section 16-B aligned)
+struct EscView {
+    const uint32_t *eidx;
+    const uint8_t *low;
+    const uint16_t *esc;
+    uint32_t nb, n_esc;
+};
+__device__ __forceinline__ EscView esc_view(const SlabView &sv, uint64_t Nt) {
+    EscView e;
+    e.nb = (uint32_t)((Nt + kEscBlock - 1) / kEscBlock);
+    e.eidx = reinterpret_cast<const uint32_t *>(sv.keys);
+    e.low = sv.keys + up16(4ull * (e.nb + 1));
+    e.esc = reinterpret_cast<const uint16_t *>(e.low + up16(Nt));
+    e.n_esc = ld_le32(sv.keys + 4ull * e.nb);
+    return e;
+}
+// key of voxel `rel` of an escaped-key slab, sequentially (scalar path)
+__device__ __forceinline__ uint32_t esc_key_scalar(const EscView &ev, uint64_t rel) {
+    const uint32_t lo = ev.low[rel];
+    if (lo != 255u) return lo;
+    const uint64_t b0 = rel / kEscBlock * kEscBlock;
+    uint32_t r = ev.eidx[rel / kEscBlock];
+    for (uint64_t v = b0; v < rel; v++) r += ev.low[v] == 255u;
+    return ev.n_esc ? ev.esc[min(r, ev.n_esc - 1)] : 0xFFFFFFFFu;
+}
+// eidx[blk + 1] - eidx[blk] equals the escapes in block blk (scalar-path check)
+__device__ __forceinline__ bool esc_block_ok(const EscView &ev, uint64_t blk, uint64_t Nt) {
+    uint32_t c = 0;
+    const uint64_t v1 = min(Nt, (blk + 1) * kEscBlock);
+    for (uint64_t v = blk * kEscBlock; v < v1; v++) c += ev.low[v] == 255u;
+    return ev.eidx[blk + 1] - ev.eidx[blk] == c;
+}
+
+// Key stage layout of an escaped-key tile (FORMAT.md 1.5 staged by the producer):
+// low bytes at 0, the tile's eidx entries from entry (b0 & ~3) at kIdxOff, and its
+// escape entries from entry (e0 & ~7) at kEscOff when they fit kEscCap
+constexpr uint32_t kIdxOff = kTileVox;          // after the low bytes (1 per voxel)
+constexpr uint32_t kEscOff = kIdxOff + 160;      // eidx slice: <= 4 * (kTileVox / 256 + 4) bytes
+constexpr uint32_t kEscCap = kStageBytes - kEscOff;
+static_assert(4 * (kTileVox / kEscBlock + 4) <= 160 && kEscCap >= 1024, "escaped-key stage layout");
+__device__ __forceinline__ uint32_t esc_copy_bytes(uint32_t e0, uint32_t e1) {
+    return ((2u * e1 + 15u) & ~15u) - ((2u * e0) & ~15u);
+}
+
 // store the 4 planes of 8 consecutive voxels (vector path): plane c of voxel v
 // is out_s[(c*N + v)]; one 16-B (fp16/int16) or 32-B (fp32) store per plane
 template <int OUT>
@@ -300,6 +355,14 @@ struct Keys8 {
         const uint32_t w = (j & 4) ? ((j & 2) ? v.w : v.z) : ((j & 2) ? v.y : v.x);
         return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
     }
+    __device__ __forceinline__ void set_dyn(uint32_t j, uint32_t key) {  // j runtime, key < 2^16
+        const uint32_t sh = (j & 1u) * 16u, keep = ~(0xFFFFu << sh), nv = (key & 0xFFFFu) << sh;
+        const uint32_t w = j >> 1;
+        v.x = w == 0 ? (v.x & keep) | nv : v.x;
+        v.y = w == 1 ? (v.y & keep) | nv : v.y;
+        v.z = w == 2 ? (v.z & keep) | nv : v.z;
+        v.w = w == 3 ? (v.w & keep) | nv : v.w;
+    }
 };
 
 // The key stream of the CTA's current range is staged into shared memory by
@@ -340,17 +403,74 @@ __device__ __forceinline__ Keys8 keys_from_smem(const uint8_t *stage, uint32_t k
 // and requested their LUT rows (up to two per thread; more are fetched in
 // place, rarely), so every group is stored once, complete, and no warp waits
 // on an L2 round trip.  A key >= G (corrupt) can only be cold: clamped, flagged.
-template <int OUT>
+template <int OUT, bool ESC>
 __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
                                                 uint32_t hot_base, uint32_t n_hot, const FuView &fu, uint8_t *out_s,
-                                                uint64_t N, uint32_t &bad, KeyRing &ring) {
+                                                uint64_t N, uint32_t &bad, KeyRing &ring, uint64_t Nt) {
     using E = typename Entry<OUT>::T;
     constexpr uint32_t EB = sizeof(E);
-    const uint32_t kwb = (uint32_t)sv.kw;
+    const bool escd = ESC && sv.kw == kEscaped;     // FORMAT.md 1.5 tile (staged by kc_produce)
+    const uint32_t kwb = escd ? 1u : (uint32_t)sv.kw;  // key bytes per voxel in the stage
+    EscView ev{};
+    if (escd) ev = esc_view(sv, Nt);
     const uint32_t Gm1 = sv.G - 1;
     const uint32_t ntiles = (uint32_t)((b - a + kTileVox - 1) / kTileVox);
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t pol = l2_policy_evict_last();  // keep this sample's LUT in L2 against the output stream
+    // kw = 3 (FORMAT.md 1.5) tile t: where this warp's escaped keys are.  The stage
+    // holds the tile's eidx entries (from entry b0 & ~3) and, when they fit, its
+    // escape entries (from entry e0 & ~7); otherwise they are read from global
+    // memory.  Returns esp with esp[i] = esc[e0 + i], and the warp's escape offset.
+    struct EscTile {
+        const uint16_t *esp;
+        uint32_t n;      // escapes of the tile (esp[0..n) valid)
+        uint32_t wbase;  // this warp's first escape, relative to e0
+        uint32_t wcnt;   // this warp's escapes per the index
+        bool wact;       // the warp has voxels in the tile
+    };
+    auto esc_tile = [&](uint32_t t) {
+        const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
+        const uint64_t st = a + (uint64_t)t * kTileVox;
+        const uint64_t rem = b - st;
+        const uint32_t nvox = rem < (uint64_t)kTileVox ? (uint32_t)rem : (uint32_t)kTileVox;
+        const uint32_t b0 = (uint32_t)(st / kEscBlock), b1 = (uint32_t)((st + nvox + kEscBlock - 1) / kEscBlock);
+        const uint32_t bw = min(b0 + (threadIdx.x >> 5), b1 - 1);
+        const uint32_t *ix = reinterpret_cast<const uint32_t *>(stage + kIdxOff) - (b0 & ~3u);  // ix[b] = eidx[b]
+        const uint32_t e0 = ix[b0], e1 = ix[b1];
+        EscTile et;
+        et.wact = b0 + (threadIdx.x >> 5) < b1;
+        const bool sane = e1 >= e0 && ix[bw] >= e0 && ix[bw + 1] >= ix[bw] && ix[bw + 1] <= e1;
+        et.n = sane ? e1 - e0 : 0u;
+        et.wbase = sane ? ix[bw] - e0 : 0u;
+        et.wcnt = sane ? ix[bw + 1] - ix[bw] : 0xFFFFFFFFu;
+        const bool staged = sane && esc_copy_bytes(e0, e1) <= kEscCap;
+        if (!staged) et.n = sane ? min(et.n, ev.n_esc > e0 ? ev.n_esc - e0 : 0u) : 0u;
+        et.esp = staged ? reinterpret_cast<const uint16_t *>(stage + kEscOff) + (e0 & 7u) : ev.esc + min(e0, ev.n_esc);
+        return et;
+    };
+    // 8-bit mask of the escaped voxels (low byte 255) among a thread's 8 low bytes
+    auto esc_mask8 = [](uint2 raw) {
+        const uint32_t a0 = __vcmpeq4(raw.x, 0xFFFFFFFFu) & 0x01010101u, a1 = __vcmpeq4(raw.y, 0xFFFFFFFFu) & 0x01010101u;
+        return ((a0 * 0x01020408u) >> 24) | (((a1 * 0x01020408u) >> 24) << 4);
+    };
+    // the keys of a thread's 8 voxels: low bytes widened, escaped ones from esp
+    auto esc_keys = [&](uint2 raw, uint32_t m, uint32_t r0, const EscTile &et) {
+        Keys8 k;
+        k.v.x = __byte_perm(raw.x, 0u, 0x4140);
+        k.v.y = __byte_perm(raw.x, 0u, 0x4342);
+        k.v.z = __byte_perm(raw.y, 0u, 0x4140);
+        k.v.w = __byte_perm(raw.y, 0u, 0x4342);
+#pragma unroll
+        for (int j = 0; j < 8; j++) {
+            if ((m >> j) & 1u) {
+                const uint32_t i = r0 + __popc(m & ((1u << j) - 1u));
+                const uint32_t key = i < et.n ? (uint32_t)et.esp[i] : 0xFFFFu;  // past the list: corrupt
+                uint32_t &w = j < 2 ? k.v.x : j < 4 ? k.v.y : j < 6 ? k.v.z : k.v.w;
+                w = (j & 1) ? (w & 0xFFFFu) | (key << 16) : (w & 0xFFFF0000u) | key;
+            }
+        }
+        return k;
+    };
     auto issue = [&](uint32_t t) {  // thread 0: bulk copy of tile t's keys once its stage is free
         const uint32_t gt = ring.count + t;
         const uint32_t stg = gt % kKeyStages;
@@ -383,9 +503,24 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         uint32_t cold = 0;
+        Keys8 kres;
+        uint32_t escw = 0;  // escaped tile: escape mask << 8 | first escape (tile-relative) << 16
+        if (escd) {         // warp-collective (scan): inactive lanes take part with no keys
+            const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
+            const uint2 raw = q < b ? lds_u2(smem_u32(stage) + threadIdx.x * 8u) : make_uint2(0u, 0u);
+            const uint32_t m = q < b ? esc_mask8(raw) : 0u;
+            const uint32_t c = __popc(m);
+            const uint32_t incl = warp_incl_scan(c, (int)lane);
+            const EscTile et = esc_tile(t);
+            const uint32_t wtot = __shfl_sync(0xffffffffu, incl, 31);
+            if (lane == 0 && et.wact && wtot != et.wcnt) bad = 1u;  // the index disagrees with the low bytes
+            const uint32_t r0 = et.wbase + incl - c;
+            kres = esc_keys(raw, m, r0, et);
+            escw = (m << 8) | (min(r0, 0xFFFFu) << 16);
+        }
         if (q < b) {
             const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
-            const Keys8 k = keys_from_smem(stage, kwb);
+            const Keys8 k = escd ? kres : keys_from_smem(stage, kwb);
 #pragma unroll
             for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
 #if SPP_KC_DIAG_NOCOLD
@@ -402,7 +537,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             }
         }
         cp_async_commit();
-        return cold;
+        return cold | escw;
     };
     // (with kProducerWarp the key tiles are issued by kc_produce, which runs
     // ahead of the consumers across segments, items and samples)
@@ -428,13 +563,19 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             cp_async_commit();  // keep one group per iteration
         }
         cp_async_wait<kColdLA>();  // the copies of tile t have landed (this thread's)
-        const uint32_t cmask = cj[0];
+        const uint32_t cmask_all = cj[0], cmask = cmask_all & 0xFFu;  // cold mask (+ escapes, kw = 3)
 #pragma unroll
         for (int i = 0; i < kColdLA; i++) cj[i] = cj[i + 1];  // rotate (compile-time indices)
         const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         if (q < b) {
-            const Keys8 k0 = keys_from_smem(stage, kwb);
+            Keys8 k0;
+            if (escd) {  // the escapes located at classify time (mask, first index) from cj
+                const EscTile et = esc_tile(t);
+                k0 = esc_keys(lds_u2(smem_u32(stage) + threadIdx.x * 8u), (cmask_all >> 8) & 0xFFu, cmask_all >> 16, et);
+            } else {
+                k0 = keys_from_smem(stage, kwb);
+            }
             E e[8];
 #pragma unroll
             for (int j = 0; j < 8; j++) {
@@ -469,6 +610,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
 // hot-prefix rebuilds, so the next segment's first tiles are already in shared
 // memory when the consumers get there (no ring drain between segments).
 // (Inlined: as a __noinline__ call the kernel ran 13% slower on C2.)
+template <bool ESC>
 __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, const CosmoMeta *__restrict__ meta,
                                            KeyRing ring, uint64_t i0, uint64_t i1, uint32_t items_per_sample,
                                            uint64_t chunk, uint64_t N, uint64_t plane) {
@@ -487,8 +629,11 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
             const SlabView sv = read_slab(b, slab_off, t);
             const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
             const uint64_t a = max(v0, sa), e = min(v1, sb);
-            if (a >= e || (sv.kw != 1 && sv.kw != 2)) continue;
-            const uint32_t kwb = (uint32_t)sv.kw;
+            const bool escd = ESC && sv.kw == kEscaped && plane % kEscBlock == 0;
+            if (a >= e || (sv.kw != 1 && sv.kw != 2 && !escd)) continue;
+            const uint32_t kwb = escd ? 1u : (uint32_t)sv.kw;
+            EscView ev{};
+            if (escd) ev = esc_view(sv, sb - sa);
             const uint64_t ra = a - sa, rb = e - sa;
             const uint32_t ntiles = (uint32_t)((rb - ra + kTileVox - 1) / kTileVox);
 #pragma unroll 1
@@ -499,9 +644,28 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
                 const uint64_t rem = rb - st;
                 const uint32_t nvox = rem < (uint64_t)kTileVox ? (uint32_t)rem : (uint32_t)kTileVox;
                 const uint32_t bytes = (nvox * kwb + 15u) & ~15u;
+                uint8_t *stage = ring.buf + stg * kStageBytes;
+                if (!escd) {
+                    fence_proxy_async_smem();
+                    mbar_arrive_expect_tx(&ring.full[stg], bytes);
+                    bulk_g2s(stage, sv.keys + st * kwb, bytes, &ring.full[stg]);
+                    continue;
+                }
+                // FORMAT.md 1.5 tile: low bytes, the eidx entries of its blocks (from an
+                // aligned entry b0 & ~3) and, when they fit, its escape entries
+                const uint32_t b0 = (uint32_t)(st / kEscBlock), b1 = (uint32_t)((st + nvox + kEscBlock - 1) / kEscBlock);
+                const uint32_t i_lo = 4u * (b0 & ~3u), i_hi = (4u * (b1 + 1) + 15u) & ~15u;
+                const uint32_t e0r = __ldg(ev.eidx + b0), e1r = __ldg(ev.eidx + b1);
+                const uint32_t e1 = min(e1r, ev.n_esc), e0 = min(e0r, e1);
+                const uint32_t ebytes = e1r >= e0r && e1r <= ev.n_esc && e1 > e0 && esc_copy_bytes(e0, e1) <= kEscCap
+                                            ? esc_copy_bytes(e0, e1) : 0u;
                 fence_proxy_async_smem();
-                mbar_arrive_expect_tx(&ring.full[stg], bytes);
-                bulk_g2s(ring.buf + stg * kStageBytes, sv.keys + st * kwb, bytes, &ring.full[stg]);
+                mbar_arrive_expect_tx(&ring.full[stg], bytes + (i_hi - i_lo) + ebytes);
+                bulk_g2s(stage, ev.low + st, bytes, &ring.full[stg]);
+                bulk_g2s(stage + kIdxOff, reinterpret_cast<const uint8_t *>(ev.eidx) + i_lo, i_hi - i_lo, &ring.full[stg]);
+                if (ebytes)
+                    bulk_g2s(stage + kEscOff, reinterpret_cast<const uint8_t *>(ev.esc) + ((2u * e0) & ~15u), ebytes,
+                             &ring.full[stg]);
             }
         }
     }
@@ -515,7 +679,7 @@ __device__ __forceinline__ void loop_sync() {
     else __syncthreads();
 }
 
-template <int OUT, bool VEC>
+template <int OUT, bool VEC, bool ESC>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *const *__restrict__ src, int n,
                                                          const float *__restrict__ fU_ws,
                                                          const CosmoMeta *__restrict__ meta, uint8_t *__restrict__ dst,
@@ -550,7 +714,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     if constexpr (kSplit) {
         if (threadIdx.x >= (uint32_t)kConsumers) {
             if (threadIdx.x == (uint32_t)kConsumers)
-                kc_produce(src, meta, ring, i0, i1, items_per_sample, chunk, N, plane);
+                kc_produce<ESC>(src, meta, ring, i0, i1, items_per_sample, chunk, N, plane);
             return;
         }
     }
@@ -577,7 +741,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
             const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
             const uint64_t a = max(v0, sa), e = min(v1, sb);
             if (a >= e) continue;
-            if (sv.kw == 1 || sv.kw == 2) {
+            if (sv.kw == 1 || sv.kw == 2 || sv.kw == kEscaped) {
                 if (cached_s != s || cached_t != (int)t) {
                     // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples;
                     // the LUT tail (cold groups) is prefetched into L2 for the cold lookups
@@ -623,8 +787,31 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     cached_s = s;
                     cached_t = (int)t;
                 }
-                if (VEC && fu.in_smem) {
-                    if constexpr (VEC) expand_keys_vec<OUT>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad, ring);
+                // escaped-key slabs (FORMAT.md 1.5) take the vector path in the ESC instance
+                // (the caller's opts.escape_keys) when blocks align with planes, else the scalar one
+                if (VEC && fu.in_smem && (sv.kw != kEscaped || (ESC && plane % kEscBlock == 0))) {
+                    if constexpr (VEC)
+                        expand_keys_vec<OUT, ESC>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad, ring,
+                                                  sb - sa);
+                } else if (sv.kw == kEscaped) {
+                    // escaped keys off the vector path: scalar, each key resolved by counting the
+                    // escapes before it in its block; the thread ending a block checks its eidx
+                    if constexpr (ESC || !VEC) {
+                        const EscView ev = esc_view(sv, sb - sa);
+                        for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) {
+                            const uint64_t rel = v - sa;
+                            uint32_t g = esc_key_scalar(ev, rel);
+                            if ((rel & (kEscBlock - 1)) == kEscBlock - 1 || rel + 1 == sb - sa)
+                                bad |= !esc_block_ok(ev, rel / kEscBlock, sb - sa);
+                            bad |= g >= sv.G;
+                            g = g < sv.G ? g : 0u;
+                            const E en = g < n_hot ? lds_entry<OUT>(hot_base + g * EB)
+                                                   : make_entry<OUT, false>(ld_ro_u2(sv.lut + 8ull * g), fu_g, bad);
+                            store1<OUT>(out_s, N, v, en);
+                        }
+                    } else {
+                        if (threadIdx.x == 0) report(status, SPP_ERR_UNSUPPORTED, s);  // needs opts.escape_keys
+                    }
                 } else {  // scalar path: odd shapes, or |U| too large for shared memory
                     for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) {
                         const uint64_t rel = v - sa;
@@ -693,14 +880,14 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     }
 }
 
-template <int OUT, bool VEC>
+template <int OUT, bool VEC, bool ESC = false>
 spp_status launch_expand(const void *const *d_src, int n, const float *fU, const CosmoMeta *meta, uint8_t *dst,
                          const spp_decode_opts &o, uint64_t N, cudaStream_t stream, const DeviceProps &dp) {
-    auto kern = kc_expand<OUT, VEC>;
+    auto kern = kc_expand<OUT, VEC, ESC>;
     const int entry_bytes = OUT == SPP_OUT_F32 ? 16 : 8;
     const int smem = kSmemBytes;
-    static int attr_done[8] = {0};  // per template instance (device-agnostic attribute)
-    const int key = (OUT - 1) * 2 + (VEC ? 1 : 0);
+    static int attr_done[16] = {0};  // per template instance (device-agnostic attribute)
+    const int key = ((OUT - 1) * 2 + (VEC ? 1 : 0)) * 2 + (ESC ? 1 : 0);
     if (!attr_done[key]) {
         if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
             return SPP_ERR_CUDA;
@@ -758,16 +945,21 @@ static spp_status cosmo_expand(const void *const *d_src, int n, void *d_dst, con
     const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
     const bool vec = plane % 16 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;  // 16-B key tiles
     uint8_t *dst = static_cast<uint8_t *>(d_dst);
+    // opts.escape_keys selects the instance that stages FORMAT.md 1.5 escaped keys
+    const bool esc = vec && o.escape_keys && kProducerWarp;
     switch (o.out) {
         case SPP_OUT_F16:
-            return vec ? launch_expand<SPP_OUT_F16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
-                       : launch_expand<SPP_OUT_F16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+            return esc   ? launch_expand<SPP_OUT_F16, true, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                   : vec ? launch_expand<SPP_OUT_F16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                         : launch_expand<SPP_OUT_F16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
         case SPP_OUT_F32:
-            return vec ? launch_expand<SPP_OUT_F32, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
-                       : launch_expand<SPP_OUT_F32, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+            return esc   ? launch_expand<SPP_OUT_F32, true, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                   : vec ? launch_expand<SPP_OUT_F32, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                         : launch_expand<SPP_OUT_F32, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
         case SPP_OUT_I16:
-            return vec ? launch_expand<SPP_OUT_I16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
-                       : launch_expand<SPP_OUT_I16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
+            return esc   ? launch_expand<SPP_OUT_I16, true, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                   : vec ? launch_expand<SPP_OUT_I16, true>(d_src, n, fU, meta, dst, o, N, stream, dp)
+                         : launch_expand<SPP_OUT_I16, false>(d_src, n, fU, meta, dst, o, N, stream, dp);
         default:
             return SPP_ERR_INVALID_ARG;
     }

@@ -11,6 +11,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <functional>
 #include <vector>
 
 #include "spp.h"
@@ -86,9 +87,15 @@ struct GroupTable {
     }
 };
 
+// FORMAT.md 1.5: eidx u32[nb+1] + low u8[Nt] + escaped u16[n_esc], 16-B sections
+uint64_t escaped_key_bytes(int64_t Nt, int64_t n_esc) {
+    const uint64_t nb = ((uint64_t)Nt + 255) / 256;
+    return round_up16(4 * (nb + 1)) + round_up16((uint64_t)Nt) + round_up16(2 * (uint64_t)n_esc);
+}
+
 struct Slab {
     int z0, z1;
-    int64_t G;
+    int64_t G, n_esc;
     int kw;
     uint64_t lut_off, keys_off;
     std::vector<uint64_t> lut;       // ordered 4-tuples (hot first)
@@ -172,7 +179,8 @@ extern "C" spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, i
                                           const spp_cosmo_params *params, void *dst, size_t dst_capacity,
                                           size_t *encoded_size) {
     const int localize = params ? params->localize : 0;
-    if (localize != 0 && localize != 1) return SPP_ERR_INVALID_ARG;
+    const int escape = params ? params->escape_keys : 0;
+    if ((localize != 0 && localize != 1) || (escape != 0 && escape != 1)) return SPP_ERR_INVALID_ARG;
     if (!counts || !encoded_size || C != 4 || D < 1 || H < 1 || W < 1 || D > 65535 || H > 65535 ||
         W > 65535)
         return SPP_ERR_INVALID_ARG;
@@ -222,6 +230,17 @@ extern "C" spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, i
         s.G = (int64_t)tab.tuple_of.size();
         s.kw = s.G == 1 ? 0 : (s.G <= spp::cosmo::kMaxG1 ? 1 : 2);
         if (s.G > spp::cosmo::kMaxG2 || 8 * s.G + s.kw * Nt >= 8 * Nt) s.kw = spp::cosmo::kRawSlab;
+        s.n_esc = 0;
+        if (escape && s.kw == 2) {
+            // FORMAT.md 1.5: escaped 1-byte keys when smaller (keys >= 255 go to a u16 list)
+            std::vector<int64_t> f(tab.freq.begin(), tab.freq.end());
+            const size_t top = std::min<size_t>(255, f.size());
+            std::partial_sort(f.begin(), f.begin() + top, f.end(), std::greater<int64_t>());
+            int64_t hot = 0;
+            for (size_t k = 0; k < top; k++) hot += f[k];
+            s.n_esc = Nt - hot;
+            if (escaped_key_bytes(Nt, s.n_esc) < round_up16(2ull * (uint64_t)Nt)) s.kw = spp::cosmo::kEscaped;
+        }
         if (s.kw != spp::cosmo::kRawSlab) {
             std::vector<uint32_t> order((size_t)s.G);
             for (uint32_t i = 0; i < (uint32_t)s.G; i++) order[i] = i;
@@ -241,7 +260,10 @@ extern "C" spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, i
             s.G = 0;
             s.lut_off = 0;
         }
-        if (s.kw != 0) {
+        if (s.kw == spp::cosmo::kEscaped) {
+            s.keys_off = off;
+            off += escaped_key_bytes(Nt, s.n_esc);
+        } else if (s.kw != 0) {
             s.keys_off = off;
             off = round_up16(off + (uint64_t)(s.kw == spp::cosmo::kRawSlab ? 8 : s.kw) * (uint64_t)Nt);
         } else {
@@ -302,13 +324,28 @@ extern "C" spp_status spp_encode_cosmo_ex(const int16_t *counts, int C, int D, i
                 while (tab.keys[h] != tt[v]) h = (h + 1) & tab.mask;
                 keys[v] = (uint8_t)s.key_of_slot[tab.slot[h] - 1];
             }
-        } else {
+        } else if (s.kw == 2) {
             uint16_t *keys = (uint16_t *)(out + s.keys_off);
             for (int64_t v = 0; v < Nt; v++) {
                 uint64_t h = GroupTable::hash(tt[v]) & tab.mask;
                 while (tab.keys[h] != tt[v]) h = (h + 1) & tab.mask;
                 keys[v] = (uint16_t)s.key_of_slot[tab.slot[h] - 1];
             }
+        } else {  // FORMAT.md 1.5 escaped keys
+            const uint64_t nb = ((uint64_t)Nt + 255) / 256;
+            uint32_t *eidx = (uint32_t *)(out + s.keys_off);
+            uint8_t *low = out + s.keys_off + round_up16(4 * (nb + 1));
+            uint16_t *esc = (uint16_t *)(low + round_up16((uint64_t)Nt));
+            uint32_t seen = 0;
+            for (int64_t v = 0; v < Nt; v++) {
+                if ((v & 255) == 0) eidx[v >> 8] = seen;
+                uint64_t h = GroupTable::hash(tt[v]) & tab.mask;
+                while (tab.keys[h] != tt[v]) h = (h + 1) & tab.mask;
+                const uint32_t k = s.key_of_slot[tab.slot[h] - 1];
+                low[v] = (uint8_t)(k < 255 ? k : 255);
+                if (k >= 255) esc[seen++] = (uint16_t)k;
+            }
+            eidx[nb] = seen;
         }
     }
     return SPP_OK;

@@ -20,6 +20,8 @@ constexpr int kMaxU = 32768;
 constexpr int kMaxG2 = 65536;                    // 16-bit keys
 constexpr int kMaxG1 = 256;                      // 8-bit keys
 constexpr int kRawSlab = 8;                      // RAW escape key width
+constexpr int kEscaped = 3;                      // escaped 1-byte keys (FORMAT.md 1.5)
+constexpr int kEscBlock = 256;                   // voxels per eidx entry
 }  // namespace cosmo
 
 // DeepCAM header field offsets (FORMAT.md 2.1)

@@ -41,7 +41,7 @@ class SppError(RuntimeError):
 
 
 class spp_cosmo_params(C.Structure):
-    _fields_ = [("localize", C.c_int)]
+    _fields_ = [("localize", C.c_int), ("escape_keys", C.c_int)]
 
 
 class spp_deepcam_params(C.Structure):
@@ -52,7 +52,7 @@ class spp_decode_opts(C.Structure):
     _fields_ = [("out", C.c_int), ("transform", C.c_int), ("shift", C.c_void_p), ("scale", C.c_void_p),
                 ("status", C.c_void_p), ("src_bytes", C.c_void_p), ("workspace", C.c_void_p),
                 ("workspace_size", C.c_size_t), ("C", C.c_int), ("D", C.c_int), ("H", C.c_int), ("W", C.c_int),
-                ("timing_events", C.c_void_p)]
+                ("timing_events", C.c_void_p), ("escape_keys", C.c_int)]
 
 
 _lib = None
@@ -115,7 +115,7 @@ def spp_cosmo_max_encoded_size(Cc: int, D: int, H: int, W: int) -> int:
     return int(load().spp_cosmo_max_encoded_size(Cc, D, H, W))
 
 
-def spp_encode_cosmo(counts: np.ndarray, localize: bool = False) -> np.ndarray:
+def spp_encode_cosmo(counts: np.ndarray, localize: bool = False, escape: bool = False) -> np.ndarray:
     """int16 [4, D, H, W] counts -> encoded uint8 stream (FORMAT.md 1); with
     `localize` through spp_encode_cosmo_ex (FORMAT.md 1.4 localized tables)."""
     a = np.ascontiguousarray(counts, dtype=np.int16)
@@ -125,8 +125,8 @@ def spp_encode_cosmo(counts: np.ndarray, localize: bool = False) -> np.ndarray:
     cap = spp_cosmo_max_encoded_size(Cc, D, H, W)
     dst = np.empty(max(cap, 64), dtype=np.uint8)
     size = C.c_size_t(0)
-    if localize:
-        prm = spp_cosmo_params(1)
+    if localize or escape:
+        prm = spp_cosmo_params(int(localize), int(escape))
         _check(load().spp_encode_cosmo_ex(a.ctypes.data, Cc, D, H, W, C.byref(prm), dst.ctypes.data, dst.size,
                                           C.byref(size)), "spp_encode_cosmo_ex")
     else:

@@ -44,9 +44,9 @@ def _same_bits(got: np.ndarray, want: np.ndarray):
         assert np.array_equal(got, want)
 
 
-def _decode(fmt_name, bufs, dims, out="f16", transform=None, shift=None, scale=None):
+def _decode(fmt_name, bufs, dims, out="f16", transform=None, shift=None, scale=None, escape_keys=False):
     from paper_conf_ipps_ibrahimo22_b200 import Decoder
-    dec = Decoder(fmt_name, dims, out=out, transform=transform)
+    dec = Decoder(fmt_name, dims, out=out, transform=transform, escape_keys=escape_keys)
     if shift is not None or scale is not None:
         dec.set_normalisation(shift, scale)
     srcs = [_to_dev(b) for b in bufs]
@@ -141,6 +141,59 @@ def test_cosmo_localized_tables(dev, orc):
     want = orc.cosmo_direct(x0, 1, "f16")
     for g in got:
         _same_bits(g, want)
+
+
+def test_cosmo_escaped_keys(dev, orc):
+    """FORMAT.md 1.5 escaped 1-byte keys decode bit-exactly with
+    opts.escape_keys = 1 (the staging kernel; its scalar path when a plane is
+    not a multiple of the 256-voxel escape block): paper sample, 4x256^3
+    multi-table, localized + escaped volume, a 48x40-plane volume, a batch
+    mixing formats; all outputs.  Without the flag the vector kernel reports
+    SPP_ERR_UNSUPPORTED for such samples."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    cases = [(gen_cosmo(1001), False), (gen_cosmo(1002, n=256), False), (gen_cosmo(3005, "unit", n=64), True),
+             (np.ascontiguousarray(gen_cosmo(1003, n=64)[:, :, :48, :40]), False)]
+    for x, loc in cases:
+        b = spp.spp_encode_cosmo(x, localize=loc, escape=True)
+        assert any(s["kw"] == 3 for s in fmt.cosmo_header(b)["slabs"])
+        for out, tr in (("f16", 1), ("i16", 0), ("f32", 1)):
+            got, st = _decode("cosmo", [b], x.shape, out=out, transform=tr, escape_keys=True)
+            assert st == 0
+            _same_bits(got[0], orc.cosmo_direct(x, tr, out))
+        _, st = _decode("cosmo", [b], x.shape, out="f16", escape_keys=False)
+        assert st == 4                                          # SPP_ERR_UNSUPPORTED, sample 0
+    x = gen_cosmo(1004)
+    bufs = [spp.spp_encode_cosmo(x, escape=True), spp.spp_encode_cosmo(x), spp.spp_encode_cosmo(x, escape=True)]
+    got, st = _decode("cosmo", bufs, x.shape, out="f16", escape_keys=True)
+    assert st == 0
+    want = orc.cosmo_direct(x, 1, "f16")
+    for g in got:
+        _same_bits(g, want)
+
+
+def test_cosmo_escaped_keys_corruption(dev):
+    """A wrong escape-block index is reported (status), on both kernels."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_cosmo(1001, n=64)
+    b = spp.spp_encode_cosmo(x, escape=True)
+    s = fmt.cosmo_header(b)["slabs"][0]
+    assert s["kw"] == 3
+    bad = b.copy()
+    o = s["keys_off"] + 4 * 40
+    v = int(np.frombuffer(bytes(bad[o:o + 4]), "<u4")[0]) + 3
+    bad[o:o + 4] = np.frombuffer(np.uint32(v).tobytes(), np.uint8)
+    _, st = _decode("cosmo", [b, bad], x.shape, out="f16", escape_keys=True)
+    assert st == (1 << 8 | 3)                                   # SPP_ERR_CORRUPT, sample 1
+    y = np.ascontiguousarray(x[:, :, :48, :40])                 # scalar path of the staging kernel
+    by = spp.spp_encode_cosmo(y, escape=True)
+    sy = fmt.cosmo_header(by)["slabs"][0]
+    bady = by.copy()
+    o = sy["keys_off"] + 4 * 20
+    bady[o:o + 4] = np.frombuffer(np.uint32(int(np.frombuffer(bytes(by[o:o + 4]), "<u4")[0]) + 3).tobytes(), np.uint8)
+    _, st = _decode("cosmo", [by, bady], y.shape, out="f16", escape_keys=True)
+    assert st == (1 << 8 | 3)
 
 
 def test_cosmo_oracle_encoded_stream(dev, orc):

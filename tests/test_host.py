@@ -68,13 +68,27 @@ def test_cosmo_localized_encoder_matches_oracle_bytes(spp, orc):
         assert np.array_equal(orc.cosmo_decode(a, x.shape, 0, "i16"), x)
 
 
+def test_cosmo_escaped_encoder_matches_oracle_bytes(spp, orc):
+    """FORMAT.md 1.5 escaped keys (spp_encode_cosmo_ex escape_keys = 1), alone
+    and with localized tables: product == oracle bytes."""
+    from synth import gen_cosmo
+    vols = [gen_cosmo(1001), gen_cosmo(3003, "unit", n=64), gen_cosmo(3002, "dense", n=64),
+            gen_cosmo(3001, "sparse", n=64), np.zeros((4, 3, 5, 7), dtype=np.int16)]
+    for x in vols:
+        for loc in (False, True):
+            a = spp.spp_encode_cosmo(x, localize=loc, escape=True)
+            b = orc.cosmo_encode(x, localize=loc, escape=True)
+            assert a.size == b.size and np.array_equal(a, b)
+            assert a.size <= spp.spp_encode_cosmo(x, localize=loc).size
+
+
 def test_cosmo_params_errors(spp):
     import ctypes as C
     x = np.zeros((4, 2, 2, 2), dtype=np.int16)
     dst = np.zeros(spp.spp_cosmo_max_encoded_size(4, 2, 2, 2), dtype=np.uint8)
     size = C.c_size_t(0)
-    for bad in (2, -1):
-        prm = spp.spp_cosmo_params(bad)
+    for bad in ((2, 0), (-1, 0), (0, 2), (0, -1)):
+        prm = spp.spp_cosmo_params(*bad)
         rc = spp.load().spp_encode_cosmo_ex(x.ctypes.data, 4, 2, 2, 2, C.byref(prm), dst.ctypes.data, dst.size,
                                             C.byref(size))
         assert rc == 1

@@ -258,6 +258,72 @@ def test_cosmo_localized_tables_take_one_byte_keys(orc):
     assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
 
 
+@pytest.mark.parametrize("vi", [0, 1, 3, 5, 6])
+def test_cosmo_escaped_keys_layout_bruteforce(orc, vi):
+    """FORMAT.md 1.5 escaped keys, pinned by brute force: on volumes with more
+    than 256 groups the slab's keys are the frequency ranks of FORMAT.md 1.3
+    step 4; ranks < 255 sit in the low bytes, the rest (low byte 255) in the
+    escape list in voxel order, eidx[b] counts the escapes before block b; the
+    layout is chosen only when smaller than 2-byte keys; decoding is lossless."""
+    rng = np.random.default_rng(20 + vi)
+    D, H, W = (8, 16, 16) if vi < 5 else (6, 16, 24)      # 2304 voxels: a partial last block
+    n = D * H * W
+    # a hot set of ~100 groups and a uniform tail (vi 6: mostly tail, so 2-byte keys win)
+    hot_frac = 0.15 if vi == 6 else 0.5 + 0.08 * vi
+    tail = 1000 if vi == 6 else 3000
+    gid = np.where(rng.random(n) < hot_frac, rng.integers(0, 100, size=n), rng.integers(100, 100 + tail, size=n))
+    x = np.array([gid % 31, gid // 31, (gid * 7) % 13, gid % 5], dtype=np.int16).reshape(4, D, H, W)
+    b = orc.cosmo_encode(x, escape=True)
+    h = fmt.cosmo_header(b)
+    assert h["T"] == 1
+    s = h["slabs"][0]
+    Uidx = {v: i for i, v in enumerate(h["U"].tolist())}
+    flat = x.reshape(4, n)
+    tuples = [tuple(Uidx[int(flat[c, v])] for c in range(4)) for v in range(n)]
+    freq = {t: tuples.count(t) for t in set(tuples)}
+    order = sorted(freq, key=lambda t: (-freq[t], t))
+    rank = {t: i for i, t in enumerate(order)}
+    keys = [rank[t] for t in tuples]
+    up16 = lambda v: (v + 15) // 16 * 16
+    nb = (n + 255) // 256
+    n_esc = sum(k >= 255 for k in keys)
+    esc_bytes = up16(4 * (nb + 1)) + up16(n) + up16(2 * n_esc)
+    assert len(order) > 256
+    if esc_bytes < up16(2 * n):
+        assert s["kw"] == 3
+        raw = bytes(b[s["keys_off"]:])
+        eidx = np.frombuffer(raw[:4 * (nb + 1)], dtype="<u4")
+        low = np.frombuffer(raw[up16(4 * (nb + 1)):][:n], dtype=np.uint8)
+        esc = np.frombuffer(raw[up16(4 * (nb + 1)) + up16(n):][:2 * n_esc], dtype="<u2")
+        assert low.tolist() == [min(k, 255) for k in keys]
+        assert esc.tolist() == [k for k in keys if k >= 255]
+        assert eidx.tolist() == [sum(k >= 255 for k in keys[:256 * i]) for i in range(nb)] + [n_esc]
+        lut = [tuple(int(t) for t in row) for row in fmt.cosmo_lut(b, s)]
+        assert lut == order
+    else:
+        assert s["kw"] == 2
+    assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
+    assert orc.cosmo_decode(b, x.shape, 1, "f16").tobytes() == orc.cosmo_direct(x, 1, "f16").tobytes()
+    # a wrong block count is corruption
+    if s["kw"] == 3 and nb > 1:
+        bad = b.copy()
+        o = s["keys_off"] + 4
+        bad[o:o + 4] = np.frombuffer(np.uint32(int(np.frombuffer(bytes(b[o:o + 4]), "<u4")[0]) + 1).tobytes(), np.uint8)
+        with pytest.raises(Exception):
+            orc.cosmo_decode(bad, x.shape, 0, "i16")
+
+
+def test_cosmo_escaped_keys_paper_ratio(orc):
+    """On the paper-shaped generator the escaped layout beats gzip's ~5x
+     where the paper's 2-byte keys give ~3.7x; lossless."""
+    from synth import gen_cosmo
+    x = gen_cosmo(1001)
+    a, b = orc.cosmo_encode(x), orc.cosmo_encode(x, escape=True)
+    assert 3.6 < x.nbytes / a.size < 3.8 and x.nbytes / b.size > 5.0
+    assert fmt.cosmo_header(b)["slabs"][0]["kw"] == 3
+    assert np.array_equal(orc.cosmo_decode(b, x.shape, 0, "i16"), x)
+
+
 def test_cosmo_size_closed_form_and_paper_ratio(orc):
     """P:98 'compression factor of roughly 4x' vs gzip 5x; P:219 gzip files are
     'roughly 75%' of ours.  Layout size = 64 + up16(2|U|) + 32 + up16(8G) + 2N."""
