@@ -79,6 +79,10 @@ constexpr int kStageBytes = kTileVox * 2;
 #define SPP_KC_LA 1
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
+#ifndef SPP_KC_ESC_PREFETCH
+#define SPP_KC_ESC_PREFETCH 0
+#endif
+constexpr bool kEscPrefetch = SPP_KC_ESC_PREFETCH;  // escaped tiles: resolve keys at classify to prefetch cold rows
 #ifndef SPP_KC_COLD_SLOTS
 #define SPP_KC_COLD_SLOTS 2
 #endif
@@ -515,8 +519,12 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             const uint32_t wtot = __shfl_sync(0xffffffffu, incl, 31);
             if (lane == 0 && et.wact && wtot != et.wcnt) bad = 1u;  // the index disagrees with the low bytes
             const uint32_t r0 = et.wbase + incl - c;
-            kres = esc_keys(raw, m, r0, et);
             escw = (m << 8) | (min(r0, 0xFFFFu) << 16);
+            if constexpr (!kEscPrefetch) {  // cold rows of escaped tiles are fetched at expansion
+                cp_async_commit();
+                return escw;
+            }
+            kres = esc_keys(raw, m, r0, et);
         }
         if (q < b) {
             const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
@@ -589,7 +597,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 } else {
                     bad |= g > Gm1;
                     const uint32_t si = __popc(cmask & ((1u << j) - 1u));  // rank among the tile's cold keys
-                    const uint2 lv = si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
+                    const bool pre = kEscPrefetch || ((cmask >> j) & 1u);  // fetched ahead at classify
+                    const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
                                                                : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }

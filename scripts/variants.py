@@ -10,10 +10,8 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_t704": ["SPP_KC_THREADS=704"],
-    "kc_t704_h138": ["SPP_KC_THREADS=704", "SPP_KC_HOT_KB=138"],
-    "kc_t640_h144": ["SPP_KC_THREADS=640", "SPP_KC_HOT_KB=144"],
-    "kc_t768": [],
+    "kc_esc_pf": [],
+    "kc_esc_nopf": ["SPP_KC_ESC_PREFETCH=0"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
@@ -40,7 +38,9 @@ def run():
         res[name] = {}
         if os.environ.get("VARIANT_COSMO", "1") == "1":
             out = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--secondary", "none", "--cpu-seconds", "0.5",
-                                  "--e2e-steps", "1", "--steps", "100"], env=env, capture_output=True, text=True)
+                                  "--e2e-steps", "1", "--steps", "100",
+                                  *os.environ.get("VARIANT_BENCH_ARGS", "").split()], env=env, capture_output=True,
+                                 text=True)
             try:
                 d = json.loads(out.stdout.strip().splitlines()[-1])
                 res[name] = {"cosmo": d["value"], "frac": d["roofline"]["frac"]}
