@@ -17,3 +17,7 @@ ncu --set full --clock-control none --import-source on -k regex:kd_decode -s 3 -
     python bench.py --workload deepcam --steps 2 --warmup 3 --e2e-steps 1 --cpu-seconds 0.2 \
     > gpurun_out/${R}_kd_ncu.log 2>&1
 echo done
+ncu --set full --clock-control none --import-source on -k regex:kc_expand -s 3 -c 1 -o gpurun_out/${R}_kc_esc \
+    python bench.py --steps 2 --warmup 3 --e2e-steps 1 --cpu-seconds 0.2 --secondary none --escape-keys \
+    > gpurun_out/${R}_kc_esc_ncu.log 2>&1
+echo done-esc
