@@ -597,7 +597,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 } else {
                     bad |= g > Gm1;
                     const uint32_t si = __popc(cmask & ((1u << j) - 1u));  // rank among the tile's cold keys
-                    const bool pre = kEscPrefetch || ((cmask >> j) & 1u);  // fetched ahead at classify
+                    const bool pre = !ESC || kEscPrefetch || ((cmask >> j) & 1u);  // fetched ahead at classify
                     const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
                                                                : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
