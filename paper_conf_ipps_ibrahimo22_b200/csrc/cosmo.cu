@@ -98,13 +98,13 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
                                                          const uint64_t *__restrict__ src_bytes, int transform,
                                                          int D, int H, int W, float *__restrict__ fU_ws,
                                                          CosmoMeta *__restrict__ meta,
-                                                         uint32_t *__restrict__ status) {
+                                                         uint32_t *__restrict__ status, int esc_ok) {
     const int s = blockIdx.x;
     const uint8_t *b = static_cast<const uint8_t *>(src[s]);
     __shared__ uint32_t sh_ok, sh_nU;
     __shared__ uint64_t sh_Uoff;
     if (threadIdx.x == 0) {
-        uint32_t ok = b != nullptr && (reinterpret_cast<uintptr_t>(b) & 15) == 0;
+        uint32_t ok = b != nullptr && (reinterpret_cast<uintptr_t>(b) & 15) == 0, unsupported = 0;
         uint64_t limit = src_bytes ? src_bytes[s] : ~0ull;
         uint32_t nU = 0, T = 0;
         uint64_t U_off = 0;
@@ -133,7 +133,10 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
                 if (kw == 0) ok = ok && G == 1;
                 else if (kw == 1) ok = ok && G >= 1 && G <= (uint32_t)kMaxG1;
                 else if (kw == 2) ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
-                else if (kw == kEscaped) ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
+                else if (kw == kEscaped) {
+                    if (!esc_ok) unsupported = 1;
+                    ok = ok && G >= 1 && G <= (uint32_t)kMaxG2;
+                }
                 else if (kw == kRawSlab) ok = ok && G == 0;
                 else ok = 0;
                 if (kw != kRawSlab) ok = ok && (lut_off & 15) == 0 && lut_off + 8ull * G <= total;
@@ -150,6 +153,8 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
             ok = ok && zexp == (uint32_t)D;
         }
         if (!ok) report(status, SPP_ERR_CORRUPT, s);
+        else if (unsupported) report(status, SPP_ERR_UNSUPPORTED, s);  // needs opts.escape_keys
+        ok = ok && !unsupported;
         sh_ok = ok;
         sh_nU = nU;
         sh_Uoff = U_off;
@@ -750,7 +755,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
             const uint64_t sa = (uint64_t)sv.z0 * plane, sb = (uint64_t)sv.z1 * plane;
             const uint64_t a = max(v0, sa), e = min(v1, sb);
             if (a >= e) continue;
-            if (sv.kw == 1 || sv.kw == 2 || sv.kw == kEscaped) {
+            if (sv.kw == 1 || sv.kw == 2 || ((ESC || !VEC) && sv.kw == kEscaped)) {
                 if (cached_s != s || cached_t != (int)t) {
                     // stage f(U) and the hottest groups (keys are frequency-ordered) as output tuples;
                     // the LUT tail (cold groups) is prefetched into L2 for the cold lookups
@@ -818,8 +823,6 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                                                    : make_entry<OUT, false>(ld_ro_u2(sv.lut + 8ull * g), fu_g, bad);
                             store1<OUT>(out_s, N, v, en);
                         }
-                    } else {
-                        if (threadIdx.x == 0) report(status, SPP_ERR_UNSUPPORTED, s);  // needs opts.escape_keys
                     }
                 } else {  // scalar path: odd shapes, or |U| too large for shared memory
                     for (uint64_t v = a + threadIdx.x; v < e; v += kLoopThreads) {
@@ -939,7 +942,14 @@ spp_status cosmo_decode(const void *const *d_src, int n, void *d_dst, const spp_
     CosmoMeta *meta = reinterpret_cast<CosmoMeta *>(ws + meta_offset(n));
     cudaEvent_t const *ev = reinterpret_cast<cudaEvent_t const *>(o.timing_events);
     if (ev && cudaEventRecord(ev[0], stream) != cudaSuccess) return SPP_ERR_CUDA;
-    kc0_prologue<<<n, kPrologueThreads, 0, stream>>>(d_src, o.src_bytes, o.transform, o.D, o.H, o.W, fU, meta, o.status);
+    // escaped-key slabs (FORMAT.md 1.5) decode on the instance selected by opts.escape_keys or on
+    // the scalar kernel (shapes off the vector path); the paper-format vector kernel never sees them
+    const uint64_t plane = (uint64_t)o.H * o.W;
+    const size_t align = o.out == SPP_OUT_F32 ? 32 : 16;
+    const bool vec = plane % 16 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
+    const int esc_ok = !vec || o.escape_keys;
+    kc0_prologue<<<n, kPrologueThreads, 0, stream>>>(d_src, o.src_bytes, o.transform, o.D, o.H, o.W, fU, meta, o.status,
+                                                     esc_ok);
     if (cudaGetLastError() != cudaSuccess) return SPP_ERR_CUDA;
     if (ev && cudaEventRecord(ev[1], stream) != cudaSuccess) return SPP_ERR_CUDA;
     spp_status r = cosmo_expand(d_src, n, d_dst, o, stream, dp, fU, meta);
