@@ -56,12 +56,15 @@ def _setup(fmt_name, n_samples):
     if fmt_name == "cosmo":
         xs = [gen_cosmo(4100 + i, n=16) for i in range(n_samples)]
         return xs, [spp.spp_encode_cosmo(x) for x in xs], xs[0].shape, None
+    if fmt_name == "cosmo_escaped":  # FORMAT.md 1.5 streams (32^3: more than 256 groups)
+        xs = [gen_cosmo(4100 + i, n=32) for i in range(n_samples)]
+        return xs, [spp.spp_encode_cosmo(x, escape=True) for x in xs], xs[0].shape, None
     xs = [gen_deepcam(4200 + i, H=8, W=1152) for i in range(n_samples)]
     return xs, [spp.spp_encode_deepcam(x) for x in xs], xs[0].shape, deepcam_stats(xs[0])
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("fmt_name", ["cosmo", "deepcam"])
+@pytest.mark.parametrize("fmt_name", ["cosmo", "deepcam", "cosmo_escaped"])
 @pytest.mark.parametrize("source,graph", [("device", True), ("device", False), ("host", False)])
 def test_loader_batches_match_oracle(fmt_name, source, graph, orc):
     if not torch.cuda.is_available():
@@ -69,9 +72,12 @@ def test_loader_batches_match_oracle(fmt_name, source, graph, orc):
     from paper_conf_ipps_ibrahimo22_b200 import Decoder
     from paper_conf_ipps_ibrahimo22_b200.loader import DecodeLoader, EncodedShard, EpochSampler
     xs, bufs, dims, stats = _setup(fmt_name, 11)
-    want = [orc.cosmo_direct(x, 1, "f16") if fmt_name == "cosmo"
+    want = [orc.cosmo_direct(x, 1, "f16") if fmt_name.startswith("cosmo")
             else orc.deepcam_decode(b, dims, stats[0], stats[1], "f16") for x, b in zip(xs, bufs)]
-    dec = Decoder(fmt_name, dims, out="f16")
+    dec = Decoder(fmt_name.split("_")[0], dims, out="f16", escape_keys=fmt_name == "cosmo_escaped")
+    if fmt_name == "cosmo_escaped":
+        from tests import fmt
+        assert all(fmt.cosmo_header(b)["slabs"][0]["kw"] == 3 for b in bufs)
     if stats is not None:
         dec.set_normalisation(stats[0], stats[1])
     shard = EncodedShard(bufs, device_resident=(source == "device"))
