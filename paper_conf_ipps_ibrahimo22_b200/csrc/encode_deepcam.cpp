@@ -13,6 +13,9 @@
 #include <stdint.h>
 #include <string.h>
 
+#include <algorithm>
+#include <cstdlib>
+#include <thread>
 #include <vector>
 
 #include "spp.h"
@@ -202,23 +205,45 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
     const uint64_t raw_size = round_up16(16 + 4 * (uint64_t)W);
     const int A = alignment_for(W);
-    LineEncoder enc(W, A, la, rm);
+    // Lines encode independently, so both passes run over contiguous
+    // line ranges on host threads (SPP_ENCODE_THREADS, default: the hardware
+    // concurrency); the output is identical for any thread count.
+    unsigned nthr = std::thread::hardware_concurrency();
+    if (const char *e = getenv("SPP_ENCODE_THREADS")) nthr = (unsigned)atoi(e);
+    nthr = std::max(1u, std::min<unsigned>(nthr ? nthr : 1u, (unsigned)((L + 63) / 64)));
+    auto parallel_lines = [&](auto &&body) {  // body(l0, l1) on [l0, l1)
+        if (nthr == 1) {
+            body((uint64_t)0, L);
+            return;
+        }
+        std::vector<std::thread> th;
+        for (unsigned i = 0; i < nthr; i++)
+            th.emplace_back([&, i]() { body(L * i / nthr, L * (i + 1) / nthr); });
+        for (auto &t : th) t.join();
+    };
     // pass 1: per-line size (SEG vs RAW)
     std::vector<uint8_t> is_seg(L);
     std::vector<uint32_t> dir(L + 1);
+    std::vector<uint64_t> line_size(L);
+    parallel_lines([&](uint64_t l0, uint64_t l1) {
+        LineEncoder enc(W, A, la, rm);
+        for (uint64_t l = l0; l < l1; l++) {
+            const float *xl = x + l * (uint64_t)W;
+            uint64_t sz = raw_size;
+            is_seg[l] = 0;
+            if (all_finite(xl, W)) {
+                int64_t seg = enc.encode(xl);
+                if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) seg = -1;  // FORMAT.md 2.5
+                if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
+            }
+            line_size[l] = sz;
+        }
+    });
     uint64_t cur = 0;
     for (uint64_t l = 0; l < L; l++) {
-        const float *xl = x + l * (uint64_t)W;
-        uint64_t sz = raw_size;
-        is_seg[l] = 0;
-        if (all_finite(xl, W)) {
-            int64_t seg = enc.encode(xl);
-            if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) seg = -1;  // FORMAT.md 2.5
-            if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
-        }
         if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;
         dir[l] = (uint32_t)cur;
-        cur += sz;
+        cur += line_size[l];
     }
     if (cur > 0xFFFFFFFFull) return SPP_ERR_UNSUPPORTED;
     dir[L] = (uint32_t)cur;
@@ -241,7 +266,9 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     memcpy(out + kTotal, &total, 8);
     memcpy(out + dir_off, dir.data(), 4 * (L + 1));
     // pass 2: payloads
-    for (uint64_t l = 0; l < L; l++) {
+    parallel_lines([&](uint64_t l0, uint64_t l1) {
+    LineEncoder enc(W, A, la, rm);
+    for (uint64_t l = l0; l < l1; l++) {
         const float *xl = x + l * (uint64_t)W;
         uint8_t *p = out + payload_off + dir[l];
         if (!is_seg[l]) {
@@ -262,5 +289,6 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
         }
         memcpy(p + 4 + 8 * (size_t)nseg, enc.deltas.data(), enc.deltas.size());
     }
+    });
     return SPP_OK;
 }
