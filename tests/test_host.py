@@ -221,3 +221,14 @@ def test_cosmo_ratio_vs_gzip_matches_paper(spp):
     assert 3.3 < x.nbytes / ours < 4.5          # "roughly 4x"
     assert 4.5 < x.nbytes / gz < 5.5            # gzip "5x"
     assert 0.65 < gz / ours < 0.85              # "roughly 75%"
+
+
+def test_deepcam_encoder_thread_count_invariant(spp, monkeypatch):
+    """Lines are encoded on host threads; the bytes do not depend on how many."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2007, H=40)
+    outs = []
+    for n in ("1", "3", "8"):
+        monkeypatch.setenv("SPP_ENCODE_THREADS", n)
+        outs.append(spp.spp_encode_deepcam(x, err_budget=8))
+    assert all(o.size == outs[0].size and np.array_equal(o, outs[0]) for o in outs)
