@@ -80,9 +80,13 @@ constexpr int kStageBytes = kTileVox * 2;
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
 #ifndef SPP_KC_ESC_PREFETCH
-#define SPP_KC_ESC_PREFETCH 0
+#define SPP_KC_ESC_PREFETCH 2
 #endif
-constexpr bool kEscPrefetch = SPP_KC_ESC_PREFETCH;  // escaped tiles: resolve keys at classify to prefetch cold rows
+// escaped tiles: 0 = keys resolved at expansion, cold rows fetched there; 1 = resolved at
+// classify (to prefetch cold rows) and again at expansion; 2 = resolved once, at classify,
+// into a buffer carved from the end of the hot region, cold rows prefetched
+constexpr int kEscPrefetch = SPP_KC_ESC_PREFETCH;
+constexpr uint32_t kRkBytes = (kColdLA + 1) * kConsumers * 16;  // resolved keys, 16 B per thread per tile
 #ifndef SPP_KC_COLD_SLOTS
 #define SPP_KC_COLD_SLOTS 2
 #endif
@@ -415,7 +419,8 @@ __device__ __forceinline__ Keys8 keys_from_smem(const uint8_t *stage, uint32_t k
 template <int OUT, bool ESC>
 __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t slab_v0, uint64_t a, uint64_t b,
                                                 uint32_t hot_base, uint32_t n_hot, const FuView &fu, uint8_t *out_s,
-                                                uint64_t N, uint32_t &bad, KeyRing &ring, uint64_t Nt) {
+                                                uint64_t N, uint32_t &bad, KeyRing &ring, uint64_t Nt,
+                                                uint32_t rk_base) {
     using E = typename Entry<OUT>::T;
     constexpr uint32_t EB = sizeof(E);
     const bool escd = ESC && sv.kw == kEscaped;     // FORMAT.md 1.5 tile (staged by kc_produce)
@@ -525,11 +530,14 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             if (lane == 0 && et.wact && wtot != et.wcnt) bad = 1u;  // the index disagrees with the low bytes
             const uint32_t r0 = et.wbase + incl - c;
             escw = (m << 8) | (min(r0, 0xFFFFu) << 16);
-            if constexpr (!kEscPrefetch) {  // cold rows of escaped tiles are fetched at expansion
+            if constexpr (kEscPrefetch == 0) {  // cold rows of escaped tiles are fetched at expansion
                 cp_async_commit();
                 return escw;
             }
             kres = esc_keys(raw, m, r0, et);
+            if constexpr (kEscPrefetch == 2) {  // the expansion reads these resolved keys back
+                if (q < b) sts_u4(rk_base + (((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * 16u, kres.v);
+            }
         }
         if (q < b) {
             const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
@@ -584,8 +592,13 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         if (q < b) {
             Keys8 k0;
             if (escd) {  // the escapes located at classify time (mask, first index) from cj
-                const EscTile et = esc_tile(t);
-                k0 = esc_keys(lds_u2(smem_u32(stage) + threadIdx.x * 8u), (cmask_all >> 8) & 0xFFu, cmask_all >> 16, et);
+                if constexpr (kEscPrefetch == 2) {
+                    k0.v = lds_u4(rk_base + (((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * 16u);
+                } else {
+                    const EscTile et = esc_tile(t);
+                    k0 = esc_keys(lds_u2(smem_u32(stage) + threadIdx.x * 8u), (cmask_all >> 8) & 0xFFu,
+                                  cmask_all >> 16, et);
+                }
             } else {
                 k0 = keys_from_smem(stage, kwb);
             }
@@ -602,7 +615,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 } else {
                     bad |= g > Gm1;
                     const uint32_t si = __popc(cmask & ((1u << j) - 1u));  // rank among the tile's cold keys
-                    const bool pre = !ESC || kEscPrefetch || ((cmask >> j) & 1u);  // fetched ahead at classify
+                    const bool pre = !ESC || kEscPrefetch != 0 || ((cmask >> j) & 1u);  // fetched ahead at classify
                     const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
                                                                : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
@@ -780,7 +793,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     const uint64_t cta_end = v0 + (i1 - it) * chunk;  // this CTA's remaining voxels of the sample
                     const uint64_t span = (sb < cta_end ? sb : cta_end) - a;
                     const uint32_t amort = span / 8 > 4096 ? (uint32_t)min(span / 8, (uint64_t)0xFFFFFFFFu) : 4096u;
-                    n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes) / EB), amort);
+                    // (an escaped slab on the staging instance keeps the region's last kRkBytes
+                    // for its resolved keys)
+                    const uint32_t rk = ESC && kEscPrefetch == 2 && sv.kw == kEscaped ? kRkBytes : 0u;
+                    n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes - rk) / EB), amort);
 #pragma unroll 1
                     for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * kLoopThreads) {
                         uint2 lv[4];
@@ -806,7 +822,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                 if (VEC && fu.in_smem && (sv.kw != kEscaped || (ESC && plane % kEscBlock == 0))) {
                     if constexpr (VEC)
                         expand_keys_vec<OUT, ESC>(sv, sa, a - sa, e - sa, hot_base, n_hot, fu, out_s, N, bad, ring,
-                                                  sb - sa);
+                                                  sb - sa, region + (uint32_t)kRegionBytes - kRkBytes);
                 } else if (sv.kw == kEscaped) {
                     // escaped keys off the vector path: scalar, each key resolved by counting the
                     // escapes before it in its block; the thread ending a block checks its eidx
