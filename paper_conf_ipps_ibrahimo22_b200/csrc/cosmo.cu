@@ -87,6 +87,10 @@ constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row l
 // into a buffer carved from the end of the hot region, cold rows prefetched
 constexpr int kEscPrefetch = SPP_KC_ESC_PREFETCH;
 constexpr uint32_t kRkBytes = (kColdLA + 1) * kConsumers * 16;  // resolved keys, 16 B per thread per tile
+#ifndef SPP_KC_ALL_LANES_RELEASE
+#define SPP_KC_ALL_LANES_RELEASE 1
+#endif
+constexpr bool kAllLanesRelease = SPP_KC_ALL_LANES_RELEASE;  // every consumer lane arrives on a stage's empty barrier
 #ifndef SPP_KC_COLD_SLOTS
 #define SPP_KC_COLD_SLOTS 2
 #endif
@@ -624,7 +628,9 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             store8<OUT>(out_s, N, slab_v0 + q, e);
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);  // this warp is done with the stage
+        // this warp is done with the stage: every lane releases its own reads (kAllLanesRelease), or
+        // lane 0 for the warp after __syncwarp (bar.warp.sync orders the other lanes' reads)
+        if (kAllLanesRelease || lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);
     }
     cp_async_wait<0>();
     ring.count += ntiles;
@@ -726,7 +732,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     if (VEC && threadIdx.x == 0) {
         for (int i = 0; i < kKeyStages; i++) {
             mbar_init(&ring.full[i], 1);
-            mbar_init(&ring.empty[i], kConsumers / kWarp);  // one arrival per consumer warp
+            mbar_init(&ring.empty[i], kAllLanesRelease ? kConsumers : kConsumers / kWarp);
         }
         fence_mbar_init();
     }

@@ -10,8 +10,8 @@ from pathlib import Path
 ROOT = Path(__file__).resolve().parent.parent
 sys.path.insert(0, str(ROOT))
 VARIANTS = {
-    "kc_esc2": [],
-    "kc_esc0": ["SPP_KC_ESC_PREFETCH=0"],
+    "kc_alllanes": [],
+    "kc_lane0": ["SPP_KC_ALL_LANES_RELEASE=0"],
 }
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
