@@ -172,6 +172,30 @@ def test_cosmo_escaped_keys(dev, orc):
         _same_bits(g, want)
 
 
+def test_cosmo_escaped_keys_edge_layouts(dev, orc):
+    """Escaped-key slabs whose tiles hold more escapes than a key stage can
+    stage (escapes clustered in z: the global-memory path of the staging
+    kernel), and a slab whose last 256-voxel block is partial (scalar path)."""
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(31)
+    vols = []
+    n = 32 * 32 * 32                                  # 22 planes of 100 hot groups, 10 of a 3000-group tail
+    gid = np.concatenate([rng.integers(0, 100, size=22 * 1024), rng.integers(100, 3100, size=10 * 1024)])
+    vols.append(np.array([gid % 31, gid // 31, (gid * 7) % 13, gid % 5], dtype=np.int16).reshape(4, 32, 32, 32))
+    n = 5 * 12 * 20                                   # 1200 voxels: 4 full blocks and a partial one
+    gid = np.where(rng.random(n) < 0.6, rng.integers(0, 100, size=n), rng.integers(100, 3100, size=n))
+    vols.append(np.array([gid % 31, gid // 31, (gid * 7) % 13, gid % 5], dtype=np.int16).reshape(4, 5, 12, 20))
+    for x in vols:
+        b = spp.spp_encode_cosmo(x, escape=True)
+        assert fmt.cosmo_header(b)["slabs"][0]["kw"] == 3
+        for out, tr in (("f16", 1), ("i16", 0)):
+            got, st = _decode("cosmo", [b, b], x.shape, out=out, transform=tr, escape_keys=True)
+            assert st == 0
+            want = orc.cosmo_direct(x, tr, out)
+            _same_bits(got[0], want)
+            _same_bits(got[1], want)
+
+
 def test_cosmo_escaped_keys_corruption(dev):
     """A wrong escape-block index is reported (status), on both kernels."""
     from synth import gen_cosmo
