@@ -122,13 +122,20 @@ spp_status spp_encode_deepcam(const float *x, int C, int H, int W,
  *                |x̂ - x| > rel_err |x| (S19) is written RAW, i.e.
  *                kept uncompressed ("areas with abrupt changes are kept
  *                uncompressed").  Trades bytes for fewer large errors.
+ *   raw16      : 1 = a line the error budget keeps uncompressed is stored as
+ *                binary16 (FORMAT.md 2.6, half the bytes) when every value is
+ *                finite and its fp16 rounding is within rel_err of it; else
+ *                fp32 RAW.  0 (default) = fp32 RAW only.  Other values ->
+ *                SPP_ERR_INVALID_ARG.
  * A zero field selects its default.  Every setting obeys the per-value
- * error bound of DESIGN.md reading S19 and decodes on the unchanged decoders. */
+ * error bound of DESIGN.md reading S19 (RAW16 lines: within rel_err) and
+ * decodes on the same decoders. */
 typedef struct {
     int lookahead;
     int repeat_min;
     float rel_err;
     int err_budget;
+    int raw16;
 } spp_deepcam_params;
 
 /* spp_encode_deepcam with explicit policy knobs (params may be NULL = defaults);

@@ -69,6 +69,9 @@ def lib():
         L.orc_deepcam_encode_p.restype = I
         L.orc_deepcam_encode_q.argtypes = [P, I, I, I, I, I, I, C.c_float, I, P, SZ, C.POINTER(SZ)]
         L.orc_deepcam_encode_q.restype = I
+        L.orc_deepcam_encode_r.argtypes = [P, I, I, I, I, I, I, C.c_float, I, I, P, SZ, C.POINTER(SZ)]
+        L.orc_deepcam_encode_r.restype = I
+        L.orc_f16_to_f32.argtypes = [C.c_uint16]; L.orc_f16_to_f32.restype = C.c_float
         L.orc_deepcam_align.argtypes = [I]; L.orc_deepcam_align.restype = I
         _lib = L
     return _lib
@@ -134,8 +137,12 @@ def deepcam_code(b: int) -> int:
     return int(lib().orc_deepcam_code(int(b)))
 
 
+def f16_to_f32(h: int) -> float:
+    return float(lib().orc_f16_to_f32(int(h)))
+
+
 def deepcam_encode(x: np.ndarray, align: int | None = None, lookahead: int = 64, repeat_min: int = 16,
-                   rel_err: float = 0.1, err_budget: int = 0) -> np.ndarray:
+                   rel_err: float = 0.1, err_budget: int = 0, raw16: bool = False) -> np.ndarray:
     """FORMAT.md 2.4 encoder; `align` overrides the default alignment rule,
     `lookahead` / `repeat_min` the policy knobs (defaults 64 / 16);
     `err_budget` > 0 applies the FORMAT.md 2.5 error budget (a SEG line with
@@ -147,8 +154,9 @@ def deepcam_encode(x: np.ndarray, align: int | None = None, lookahead: int = 64,
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
     A = lib().orc_deepcam_align(W) if align is None else int(align)
-    _check(lib().orc_deepcam_encode_q(_p(a), Cc, H, W, A, int(lookahead), int(repeat_min), float(rel_err),
-                                      int(err_budget), _p(dst), cap, C.byref(size)), "deepcam_encode")
+    _check(lib().orc_deepcam_encode_r(_p(a), Cc, H, W, A, int(lookahead), int(repeat_min), float(rel_err),
+                                      int(err_budget), int(bool(raw16)), _p(dst), cap, C.byref(size)),
+           "deepcam_encode")
     return dst[: size.value].copy()
 
 

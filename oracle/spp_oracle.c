@@ -50,6 +50,16 @@ static uint64_t up16(uint64_t x) { return (x + 15) & ~(uint64_t)15; }
 /* ------------------------------------------------------------------ */
 /* IEEE binary32 -> binary16, round to nearest, ties to even.
  * Pinned against numpy's float16 conversion (library routine). */
+/* binary16 -> binary32 (exact: every half is a float), FORMAT.md 2.6 */
+float orc_f16_to_f32(uint16_t h) {
+    int sgn = h >> 15, E = (h >> 10) & 31, M = h & 1023;
+    float v;
+    if (E == 0) v = ldexpf((float)M, -24);                       /* zero / subnormal */
+    else if (E == 31) v = M ? NAN : INFINITY;
+    else v = ldexpf((float)(1024 + M), E - 25);
+    return sgn ? -v : v;
+}
+
 uint16_t orc_f32_to_f16(float f) {
     uint32_t x = bits_of_f32(f);
     uint32_t sign = (x >> 16) & 0x8000u;
@@ -451,6 +461,11 @@ int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat)
         for (int x = 0; x < W; x++) xhat[x] = f32_of_bits(rd32(p + 16 + 4 * (uint64_t)x));
         return ORC_OK;
     }
+    if (mode == 2) {                                     /* RAW16 (FORMAT.md 2.6) */
+        if (16 + 2 * (uint64_t)W > len_line) return ORC_ECORRUPT;
+        for (int x = 0; x < W; x++) xhat[x] = orc_f16_to_f32(rd16(p + 16 + 2 * (uint64_t)x));
+        return ORC_OK;
+    }
     if (mode != 1) return ORC_ECORRUPT;
     int nseg = rd16(p + 2);
     if (nseg < 1 || nseg > W || 4 + 8 * (uint64_t)nseg > len_line) return ORC_ECORRUPT;
@@ -636,6 +651,24 @@ int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahe
                          size_t cap, size_t *size) {
     return orc_deepcam_encode_q(x, C, H, W, A, lookahead, repeat_min, 0.1f, 0, dst, cap, size);
 }
+int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, uint8_t *dst, size_t cap, size_t *size);
+int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_deepcam_encode_r(x, C, H, W, A, lookahead, repeat_min, rel_err, err_budget, 0, dst, cap, size);
+}
+
+/* FORMAT.md 2.6: a line the error budget keeps uncompressed may be stored as
+ * binary16 when every value is finite and its RNE binary16 rounding is within
+ * rel of it (same metric as line_bad_count) */
+static int raw16_ok(const float *x, int W, double rel) {
+    for (int k = 0; k < W; k++) {
+        if (!isfinite(x[k])) return 0;
+        float h = orc_f16_to_f32(orc_f32_to_f16(x[k]));
+        if (!isfinite(h) || fabs((double)h - (double)x[k]) > rel * fabs((double)x[k])) return 0;
+    }
+    return 1;
+}
 
 /* FORMAT.md 2.5 ("areas with abrupt changes are kept uncompressed";
  * P:86 "roughly 3% of the values with larger than 10% error"): the number of
@@ -664,9 +697,11 @@ static int line_bad_count(const float *x, const seg_t *segs, int nseg, const uin
     return bad;
 }
 
-int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
-                         int err_budget, uint8_t *dst, size_t cap, size_t *size) {
+int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, uint8_t *dst, size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
+    if (raw16 != 0 && raw16 != 1) return ORC_EINVAL;
+    uint64_t raw16_size = up16(16 + 2 * (uint64_t)W);
     if (lookahead < 2 || lookahead > 65535 || repeat_min < 2 || repeat_min > 65535) return ORC_EINVAL;
     if (err_budget < 0 || !(rel_err > 0.0f) || !(rel_err < 1e30f)) return ORC_EINVAL;
     if ((uint64_t)C * H > 0xFFFFFFFFull || A < 1 || W % A != 0) return ORC_EINVAL;
@@ -687,8 +722,10 @@ int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahe
         if (finite) {
             int nseg; int64_t nd;
             int64_t seg_size = encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run);
-            if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget)
+            if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
                 seg_size = -1;                            /* over the error budget: RAW (FORMAT.md 2.5) */
+                if (raw16 && raw16_ok(xl, W, rel_err)) sz = raw16_size;   /* ... in binary16 (2.6) */
+            }
             if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
         }
         pay += sz;
@@ -712,9 +749,16 @@ int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahe
         for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
         int nseg = 0; int64_t nd = 0;
         int64_t seg_size = finite ? encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) : -1;
-        if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget)
+        int use16 = 0;
+        if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
             seg_size = -1;
-        if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
+            use16 = raw16 && raw16_ok(xl, W, rel_err);
+        }
+        if (use16) {
+            p[0] = 2;
+            for (int k = 0; k < W; k++) wr16(p + 16 + 2 * (uint64_t)k, orc_f32_to_f16(xl[k]));
+            cur += raw16_size;
+        } else if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
             p[0] = 1; wr16(p + 2, (uint16_t)nseg);
             for (int s = 0; s < nseg; s++) {
                 wr16(p + 4 + 4 * s, (uint16_t)segs[s].len);

@@ -126,7 +126,7 @@ spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, in
             const uint64_t a = r32(dir_off + 4ull * l), e = r32(dir_off + 4ull * l + 4);
             if (pay + e > src_bytes || e < a + 16) return SPP_ERR_CORRUPT;
             const uint8_t *p = b + pay + a;
-            if (p[0] == deepcam::kModeRaw) { raw++; continue; }
+            if (p[0] == deepcam::kModeRaw || p[0] == deepcam::kModeRaw16) { raw++; continue; }
             seg++;
             uint16_t ns;
             memcpy(&ns, p + 2, 2);

@@ -196,6 +196,31 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
         }
         return true;
     }
+    if (mode == kModeRaw16) {  // FORMAT.md 2.6: binary16 values, widened exactly
+        if (16u + 2u * W > bytes) return false;
+        const __half *x = reinterpret_cast<const __half *>(buf + 16);
+        for (uint32_t c0 = 0; c0 < W; c0 += 256) {
+            const uint32_t p0 = c0 + 8 * lane;
+            if (p0 >= W) continue;
+            float y[8];
+            if constexpr (VEC) {
+                const uint4 v = *reinterpret_cast<const uint4 *>(x + p0);
+                const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                for (int j = 0; j < 8; j++) {
+                    const float xv = __half2float(__ushort_as_half((unsigned short)((w[j >> 1] >> (16 * (j & 1))) & 0xFFFFu)));
+                    y[j] = __fmul_rn(__fsub_rn(xv, shv), scv);
+                }
+                emit8<OUT>(row, p0, W, y);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 8; j++)
+                    y[j] = p0 + j < W ? __fmul_rn(__fsub_rn(__half2float(x[p0 + j]), shv), scv) : 0.f;
+                emit_scalar<OUT>(row, p0, W, y);
+            }
+        }
+        return true;
+    }
     if (mode != kModeSeg) return false;
     const uint32_t nseg = hdr >> 16;
     if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;

@@ -171,6 +171,28 @@ int bad_values(const LineEncoder &e, const float *x, double rel) {
     return bad;
 }
 
+// binary32 -> binary16, round to nearest even (FORMAT.md 2.6 RAW16 lines)
+inline uint16_t f32_to_f16(float f) {
+    _Float16 h = (_Float16)f;
+    uint16_t u;
+    memcpy(&u, &h, 2);
+    return u;
+}
+inline float f16_to_f32(uint16_t u) {
+    _Float16 h;
+    memcpy(&h, &u, 2);
+    return (float)h;
+}
+// FORMAT.md 2.6: every value finite and its binary16 rounding within rel of it
+bool raw16_ok(const float *x, int W, double rel) {
+    for (int k = 0; k < W; k++) {
+        if (!isfinite(x[k])) return false;
+        const float h = f16_to_f32(f32_to_f16(x[k]));
+        if (!isfinite(h) || fabs((double)h - (double)x[k]) > rel * fabs((double)x[k])) return false;
+    }
+    return true;
+}
+
 inline bool all_finite(const float *x, int W) {
     for (int k = 0; k < W; k++)
         if (!isfinite(x[k])) return false;
@@ -198,6 +220,9 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     const int rm = params && params->repeat_min ? params->repeat_min : kRepeatMin;
     const float rel = params && params->rel_err != 0.0f ? params->rel_err : 0.1f;
     const int budget = params ? params->err_budget : 0;
+    const int raw16 = params ? params->raw16 : 0;
+    if (raw16 != 0 && raw16 != 1) return SPP_ERR_INVALID_ARG;
+    const uint64_t raw16_size = round_up16(16 + 2 * (uint64_t)W);
     if (la < 2 || la > 65535 || rm < 2 || rm > 65535) return SPP_ERR_INVALID_ARG;
     if (budget < 0 || !(rel > 0.0f) || !(rel < 1e30f)) return SPP_ERR_INVALID_ARG;
     const uint64_t L = (uint64_t)C * H;
@@ -233,7 +258,10 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
             is_seg[l] = 0;
             if (all_finite(xl, W)) {
                 int64_t seg = enc.encode(xl);
-                if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) seg = -1;  // FORMAT.md 2.5
+                if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) {  // FORMAT.md 2.5
+                    seg = -1;
+                    if (raw16 && raw16_ok(xl, W, rel)) { sz = raw16_size; is_seg[l] = 2; }  // 2.6
+                }
                 if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
             }
             line_size[l] = sz;
@@ -274,6 +302,14 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
         if (!is_seg[l]) {
             p[0] = kModeRaw;
             memcpy(p + 16, xl, 4 * (size_t)W);
+            continue;
+        }
+        if (is_seg[l] == 2) {
+            p[0] = kModeRaw16;
+            for (int k = 0; k < W; k++) {
+                const uint16_t h = f32_to_f16(xl[k]);
+                memcpy(p + 16 + 2 * (size_t)k, &h, 2);
+            }
             continue;
         }
         enc.encode(xl);

@@ -48,8 +48,8 @@ def deepcam_header(b: np.ndarray):
 def deepcam_line(b, hdr, l):
     a, e = int(hdr["dir"][l]), int(hdr["dir"][l + 1])
     p = bytes(b[hdr["payload_off"] + a: hdr["payload_off"] + e])
-    if p[0] == 0:
-        return dict(mode=0, size=len(p))
+    if p[0] in (0, 2):                 # RAW (fp32) / RAW16 (FORMAT.md 2.6)
+        return dict(mode=int(p[0]), size=len(p))
     nseg = struct.unpack_from("<H", p, 2)[0]
     segs = []
     for s in range(nseg):

@@ -359,6 +359,26 @@ def test_deepcam_error_budget_streams(dev, orc, budget):
     _same_bits(got[0], _dc_ref(orc, b, x.shape, None, None, "f32"))
 
 
+@pytest.mark.parametrize("budget", [1, 16])
+def test_deepcam_raw16_streams(dev, orc, budget):
+    """FORMAT.md 2.6 RAW16 lines (error budget + raw16) on the full C3 shape,
+    mixed with SEG and fp32 RAW lines: bit-exact, fp16 / fp32 / x-hat."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2009)
+    mean, rstd = deepcam_stats(x)
+    b = spp.spp_encode_deepcam(x, err_budget=budget, raw16=True)
+    h = fmt.deepcam_header(b)
+    modes = {fmt.deepcam_line(b, h, l)["mode"] for l in range(0, h["L"], 5)}
+    assert {1, 2} <= modes
+    for out, sh, sc in (("f16", mean, rstd), ("f32", mean, rstd), ("f32", None, None)):
+        got, st = _decode("deepcam", [b, b], x.shape, out=out, shift=sh, scale=sc)
+        assert st == 0
+        want = _dc_ref(orc, b, x.shape, sh, sc, out)
+        _same_bits(got[0], want)
+        _same_bits(got[1], want)
+
+
 def test_deepcam_oracle_encoded_stream(dev, orc):
     from synth import gen_deepcam
     x = gen_deepcam(2002, H=64)

@@ -190,12 +190,13 @@ def test_deepcam_encoder_knobs_match_oracle_and_bound(spp, orc, lookahead, repea
 
 @pytest.mark.parametrize("rel,budget", [(0.1, 1), (0.1, 32), (0.05, 4), (0.5, 200)])
 def test_deepcam_error_budget_matches_oracle(spp, orc, rel, budget):
-    """FORMAT.md 2.5 error budget: product == oracle bytes."""
+    """FORMAT.md 2.5 error budget (and 2.6 RAW16 lines): product == oracle bytes."""
     from synth import gen_deepcam
     x = gen_deepcam(2005, H=16)
-    a = spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget)
-    b = orc.deepcam_encode(x, rel_err=rel, err_budget=budget)
-    assert a.size == b.size and np.array_equal(a, b)
+    for raw16 in (False, True):
+        a = spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget, raw16=raw16)
+        b = orc.deepcam_encode(x, rel_err=rel, err_budget=budget, raw16=raw16)
+        assert a.size == b.size and np.array_equal(a, b)
 
 
 def test_deepcam_encoder_knob_errors(spp):

@@ -591,6 +591,48 @@ def test_deepcam_error_budget(orc, rel, budget):
         assert bad1 <= budget / W + 1e-12                                   # per-line cap holds on average
 
 
+def test_f16_to_f32_exhaustive(orc):
+    """FORMAT.md 2.6 widening: all 65,536 binary16 patterns against numpy."""
+    h = np.arange(65536, dtype=np.uint16)
+    want = h.view(np.float16).astype(np.float32)
+    got = np.array([orc.f16_to_f32(int(v)) for v in h], dtype=np.float32)
+    nan = np.isnan(want)
+    assert np.array_equal(np.isnan(got), nan)
+    assert np.array_equal(got[~nan].view(np.uint32), want[~nan].view(np.uint32))
+
+
+@pytest.mark.parametrize("budget", [1, 16])
+def test_deepcam_raw16_lines(orc, budget):
+    """FORMAT.md 2.6: with raw16, exactly the budget's RAW lines whose values
+    all round to finite binary16 within rel_err (checked with numpy) become
+    RAW16 and decode to numpy's float16 rounding; nothing else changes."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2008, H=24)
+    C, H, W = x.shape
+    b0 = orc.deepcam_encode(x, err_budget=budget)
+    b1 = orc.deepcam_encode(x, err_budget=budget, raw16=True)
+    h0, h1 = fmt.deepcam_header(b0), fmt.deepcam_header(b1)
+    n16 = 0
+    for l in range(C * H):
+        c, y = divmod(l, H)
+        i0, i1 = fmt.deepcam_line(b0, h0, l), fmt.deepcam_line(b1, h1, l)
+        xs = x[c, y]
+        with np.errstate(over="ignore"):
+            r16 = xs.astype(np.float16).astype(np.float32)
+        ok16 = bool(np.all(np.isfinite(xs)) and np.all(np.isfinite(r16)) and
+                    np.all(np.abs(r16.astype(np.float64) - xs) <= np.float64(np.float32(0.1)) * np.abs(xs.astype(np.float64))))
+        seg_budget = i0["mode"] == 0 and fmt.deepcam_line(orc.deepcam_encode(x[c:c + 1, y:y + 1]),
+                                                           fmt.deepcam_header(orc.deepcam_encode(x[c:c + 1, y:y + 1])),
+                                                           0)["mode"] == 1
+        if seg_budget and ok16:
+            assert i1["mode"] == 2 and i1["size"] == (16 + 2 * W + 15) // 16 * 16
+            assert np.array_equal(orc.deepcam_decode_line(b1, l, W).view(np.uint32), r16.view(np.uint32))
+            n16 += 1
+        else:
+            assert i1 == i0
+    assert n16 > 0 and b1.size < b0.size
+
+
 def test_deepcam_special_shapes(orc):
     for (C, H, W) in ((1, 1, 1), (1, 3, 2), (2, 2, 17), (1, 1, 16)):
         x = np.random.default_rng(C * 100 + W).standard_normal((C, H, W)).astype(np.float32)
