@@ -104,6 +104,12 @@ int cpu_deepcam_decode_f16(const uint8_t *s, size_t size, const float *shift, co
             const uint8_t *p = s + payload_off + dir[l];
             if (p[0] == 0) {
                 memcpy(xh, p + 16, 4 * (size_t)W);
+            } else if (p[0] == 2) {  /* RAW16 (FORMAT.md 2.6) */
+                for (int x = 0; x < W; x++) {
+                    _Float16 h;
+                    memcpy(&h, p + 16 + 2 * (size_t)x, 2);
+                    xh[x] = (float)h;
+                }
             } else {
                 const int nseg = RD(uint16_t, p + 2);
                 const uint8_t *desc = p + 4, *heads = p + 4 + 4 * nseg, *d = p + 4 + 8 * nseg;

@@ -23,7 +23,8 @@ def test_cpu_plugin_matches_oracle(orc):
     y = gen_deepcam(2001, H=24)
     y[3, 5, 7] = np.nan                                    # a RAW line
     mean, rstd = deepcam_stats(np.nan_to_num(y))
-    for d in (spp.spp_encode_deepcam(y), spp.spp_encode_deepcam(y, err_budget=4)):
+    for d in (spp.spp_encode_deepcam(y), spp.spp_encode_deepcam(y, err_budget=4),
+              spp.spp_encode_deepcam(y, err_budget=4, raw16=True)):
         got = cpu_plugin.deepcam_decode(L, d, y.shape, mean, rstd)
         want = orc.deepcam_decode(d, y.shape, mean, rstd, "f16")
         nan = np.isnan(want)
