@@ -79,6 +79,9 @@ constexpr int kStageBytes = kTileVox * 2;
 #define SPP_KC_LA 1
 #endif
 constexpr int kColdLA = SPP_KC_LA;                        // tiles of cold-row lookahead
+#ifndef SPP_KC_ESC_IMPL
+#define SPP_KC_ESC_IMPL 1  // escaped-key resolution: 0 predicated generic loads, 1 shared loads + PRMT, 2 loop
+#endif
 #ifndef SPP_KC_ESC_PREFETCH
 #define SPP_KC_ESC_PREFETCH 2
 #endif
@@ -373,12 +376,11 @@ struct Keys8 {
         return (j & 1) ? (w >> 16) : (w & 0xFFFFu);
     }
     __device__ __forceinline__ void set_dyn(uint32_t j, uint32_t key) {  // j runtime, key < 2^16
-        const uint32_t sh = (j & 1u) * 16u, keep = ~(0xFFFFu << sh), nv = (key & 0xFFFFu) << sh;
-        const uint32_t w = j >> 1;
-        v.x = w == 0 ? (v.x & keep) | nv : v.x;
-        v.y = w == 1 ? (v.y & keep) | nv : v.y;
-        v.z = w == 2 ? (v.z & keep) | nv : v.z;
-        v.w = w == 3 ? (v.w & keep) | nv : v.w;
+        const uint32_t sel = (j & 1) ? 0x5410u : 0x3254u, w = j >> 1;
+        v.x = w == 0 ? __byte_perm(v.x, key, sel) : v.x;
+        v.y = w == 1 ? __byte_perm(v.y, key, sel) : v.y;
+        v.z = w == 2 ? __byte_perm(v.z, key, sel) : v.z;
+        v.w = w == 3 ? __byte_perm(v.w, key, sel) : v.w;
     }
 };
 
@@ -445,6 +447,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         uint32_t wbase;  // this warp's first escape, relative to e0
         uint32_t wcnt;   // this warp's escapes per the index
         bool wact;       // the warp has voxels in the tile
+        bool staged;     // esp is in shared memory (at ssh)
+        uint32_t ssh;
     };
     auto esc_tile = [&](uint32_t t) {
         const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
@@ -464,6 +468,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         const bool staged = sane && esc_copy_bytes(e0, e1) <= kEscCap;
         if (!staged) et.n = sane ? min(et.n, ev.n_esc > e0 ? ev.n_esc - e0 : 0u) : 0u;
         et.esp = staged ? reinterpret_cast<const uint16_t *>(stage + kEscOff) + (e0 & 7u) : ev.esc + min(e0, ev.n_esc);
+        et.staged = staged;
+        et.ssh = smem_u32(stage + kEscOff) + 2u * (e0 & 7u);  // shared address of esp[0] when staged
         return et;
     };
     // 8-bit mask of the escaped voxels (low byte 255) among a thread's 8 low bytes
@@ -478,6 +484,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         k.v.y = __byte_perm(raw.x, 0u, 0x4342);
         k.v.z = __byte_perm(raw.y, 0u, 0x4140);
         k.v.w = __byte_perm(raw.y, 0u, 0x4342);
+#if SPP_KC_ESC_IMPL == 0
 #pragma unroll
         for (int j = 0; j < 8; j++) {
             if ((m >> j) & 1u) {
@@ -487,6 +494,41 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 w = (j & 1) ? (w & 0xFFFFu) | (key << 16) : (w & 0xFFFF0000u) | key;
             }
         }
+#elif SPP_KC_ESC_IMPL == 1
+        // the warp's escapes are staged (the common case): shared loads; one PRMT per insert
+        if (et.staged) {
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                if ((m >> j) & 1u) {
+                    const uint32_t i = r0 + __popc(m & ((1u << j) - 1u));
+                    const uint32_t key = i < et.n ? lds_u16(et.ssh + 2u * i) : 0xFFFFu;  // past the list: corrupt
+                    uint32_t &w = j < 2 ? k.v.x : j < 4 ? k.v.y : j < 6 ? k.v.z : k.v.w;
+                    w = __byte_perm(w, key, (j & 1) ? 0x5410u : 0x3254u);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                if ((m >> j) & 1u) {
+                    const uint32_t i = r0 + __popc(m & ((1u << j) - 1u));
+                    const uint32_t key = i < et.n ? (uint32_t)__ldg(et.esp + i) : 0xFFFFu;
+                    uint32_t &w = j < 2 ? k.v.x : j < 4 ? k.v.y : j < 6 ? k.v.z : k.v.w;
+                    w = __byte_perm(w, key, (j & 1) ? 0x5410u : 0x3254u);
+                }
+            }
+        }
+#else
+        // a loop over this lane's escapes only (consecutive in the list)
+        uint32_t i = r0;
+#pragma unroll 1
+        while (m) {
+            const uint32_t j = __ffs(m) - 1;
+            m &= m - 1;
+            const uint32_t key = i < et.n ? (et.staged ? lds_u16(et.ssh + 2u * i) : (uint32_t)__ldg(et.esp + i)) : 0xFFFFu;
+            k.set_dyn(j, key);
+            i++;
+        }
+#endif
         return k;
     };
     auto issue = [&](uint32_t t) {  // thread 0: bulk copy of tile t's keys once its stage is free
