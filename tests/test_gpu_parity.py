@@ -379,6 +379,23 @@ def test_deepcam_raw16_streams(dev, orc, budget):
         _same_bits(got[1], want)
 
 
+@pytest.mark.parametrize("W", [37, 64])
+def test_deepcam_raw16_narrow_lines(dev, orc, W):
+    """RAW16, RAW and SEG lines on the scalar (W = 37) and 8-wide (W = 64)
+    decode paths, normalised fp16 / fp32."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2010, H=16, W=W)
+    mean, rstd = deepcam_stats(x)
+    b = spp.spp_encode_deepcam(x, err_budget=1, raw16=True)
+    h = fmt.deepcam_header(b)
+    assert {0, 1, 2} <= {fmt.deepcam_line(b, h, l)["mode"] for l in range(h["L"])}
+    for out in ("f16", "f32"):
+        got, st = _decode("deepcam", [b], x.shape, out=out, shift=mean, scale=rstd)
+        assert st == 0
+        _same_bits(got[0], _dc_ref(orc, b, x.shape, mean, rstd, out))
+
+
 def test_deepcam_oracle_encoded_stream(dev, orc):
     from synth import gen_deepcam
     x = gen_deepcam(2002, H=64)
