@@ -19,7 +19,16 @@
 //                        keys rebuild the tuple from the L1/L2-resident LUT.
 //                        Each thread handles 8 consecutive voxels: one 16-B key
 //                        load, 8 smem gathers, four 16-B (fp16) streaming
-//                        stores, one per redshift plane.
+//                        stores, one per redshift plane.  One producer warp
+//                        streams the key tiles of every segment the CTA will
+//                        expand through a 5-stage TMA ring (kc_produce); the
+//                        768 consumer threads classify cold keys one tile
+//                        ahead and fetch their LUT rows by cp.async.
+//   KC (ESC instance, opts.escape_keys) also decodes FORMAT.md 1.5 escaped
+//                        1-byte keys: the producer stages each tile's low
+//                        bytes, escape-block index and escape entries; the
+//                        consumers resolve keys once per tile (warp scan of
+//                        escape counts) into a buffer carved from the hot region.
 // HBM traffic per sample = keys + LUT + U + outputs; everything else is
 // on-chip or L2.
 #include <cuda_fp16.h>
