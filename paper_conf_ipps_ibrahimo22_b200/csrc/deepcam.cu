@@ -26,6 +26,13 @@
 //                         (one rounding; FORMAT.md 2.3 reading S13);
 //                      3. y = (x̂ - shift) * scale (two roundings), RNE to fp16,
 //                         one 16-B streaming store per lane (512 B per warp).
+//   KD   kd_decode_ws  (the default) the same decode, warp-specialised: one
+//                    producer warp per CTA streams each consumer warp's lines
+//                    (line record by st.async + bytes by TMA) into a 3-slot
+//                    ring; W = 1152 lines with 36-aligned segments decode in
+//                    one warp pass (decode_line_onepass) and leave as one TMA
+//                    bulk store of the staged row.  RAW and RAW16 lines
+//                    (FORMAT.md 2.6) take the general line path.
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
