@@ -858,6 +858,9 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
 #define SPP_KD_WS_MINB 2
 #endif
 constexpr int kWsWarps = SPP_KD_WS_WPC + 1;
+#ifndef SPP_KD_PROD_SLEEP_NS
+#define SPP_KD_PROD_SLEEP_NS 100  // producer back-off when no slot was free this round
+#endif
 #ifndef SPP_KD_WS_NS
 #define SPP_KD_WS_NS 3  // input slots per consumer warp (a ring)
 #endif
@@ -1002,7 +1005,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
                     }
                 }
             }
-            if (!__any_sync(0xffffffffu, did)) __nanosleep(100);
+            if (!__any_sync(0xffffffffu, did) && SPP_KD_PROD_SLEEP_NS) __nanosleep(SPP_KD_PROD_SLEEP_NS);
         }
         return;
     }
