@@ -589,6 +589,29 @@ def test_deepcam_corruption_detected(dev):
     c = b.copy(); c[0] = 0
     _, st = _decode("deepcam", [b, c], (1, 2, W), out="f16")
     assert st == (3 | (1 << 8))
+    # a RAW16 line (FORMAT.md 2.6) shorter than 16 + 2 W bytes, and an unknown line mode
+    short16 = bytes([2]) + b"\0" * 15 + b"\0" * (2 * W - 16)
+    mode9 = bytes([9]) + b"\0" * 15 + b"\0" * (2 * W)
+    for bad in (short16, mode9):
+        b = fmt.build_deepcam_stream(1, 2, W, [good, bad])
+        _, st = _decode("deepcam", [b, b], (1, 2, W), out="f16")
+        assert st & 0xFF == 3
+
+
+def test_deepcam_mixed_line_modes_batch(dev, orc):
+    """One batch mixing streams of every line mode the encoders write: the
+    default SEG stream, an error-budget stream (fp32 RAW lines), a RAW16
+    stream, a knob-tuned stream; every output bit-exact."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2011, H=96)
+    mean, rstd = deepcam_stats(x)
+    bufs = [spp.spp_encode_deepcam(x), spp.spp_encode_deepcam(x, err_budget=4),
+            spp.spp_encode_deepcam(x, err_budget=4, raw16=True), spp.spp_encode_deepcam(x, lookahead=8, repeat_min=4)]
+    got, st = _decode("deepcam", bufs, x.shape, out="f16", shift=mean, scale=rstd)
+    assert st == 0
+    for g, b in zip(got, bufs):
+        _same_bits(g, _dc_ref(orc, b, x.shape, mean, rstd, "f16"))
 
 
 # ------------------------------------------------------------------ streamed (b.4 + b.5)
