@@ -466,7 +466,7 @@ int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat)
         for (int x = 0; x < W; x++) xhat[x] = orc_f16_to_f32(rd16(p + 16 + 2 * (uint64_t)x));
         return ORC_OK;
     }
-    if (mode != 1) return ORC_ECORRUPT;
+    if (mode != 1 && mode != 3) return ORC_ECORRUPT;        /* 3: SEG with RAW segments (FORMAT.md 2.7) */
     int nseg = rd16(p + 2);
     if (nseg < 1 || nseg > W || 4 + 8 * (uint64_t)nseg > len_line) return ORC_ECORRUPT;
     uint64_t dpos = 4 + 8 * (uint64_t)nseg;             /* next delta byte */
@@ -490,6 +490,10 @@ int orc_deepcam_decode_line(const uint8_t *src, size_t size, int l, float *xhat)
                 xhat[pos + j] = h + (float)S * unit;     /* fp32: exact product, one rounding */
             }
             dpos += (uint64_t)(len - 1);
+        } else if (kind == 2 && mode == 3) {             /* RAW segment: len binary32 values */
+            if (dpos + 4 * (uint64_t)len > len_line) return ORC_ECORRUPT;
+            for (int j = 0; j < len; j++) xhat[pos + j] = f32_of_bits(rd32(p + dpos + 4 * (uint64_t)j));
+            dpos += 4 * (uint64_t)len;
         } else {
             return ORC_ECORRUPT;
         }

@@ -148,6 +148,15 @@ __device__ __forceinline__ SegInfo seg_info(const uint32_t *desc, const float *h
     return si;
 }
 
+// binary32 at any byte address of shared memory (RAW segments, FORMAT.md 2.7)
+__device__ __forceinline__ float lds_f32_any(uint32_t addr) {
+    const uint32_t al = addr & ~3u, sh = (addr & 3u) * 8u;
+    uint32_t w0, w1;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w0) : "r"(al));
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w1) : "r"(al + 4));
+    return __uint_as_float(__funnelshift_r(w0, w1, sh));
+}
+
 template <int OUT>
 __device__ __forceinline__ void emit8(uint8_t *row, uint32_t p0, uint32_t W, const float (&y)[8]) {
     if constexpr (OUT == SPP_OUT_F32) {
@@ -228,7 +237,8 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
         }
         return true;
     }
-    if (mode != kModeSeg) return false;
+    if (mode != kModeSeg && mode != kModeSegRaw) return false;
+    const uint32_t max_kind = mode == kModeSegRaw ? kRawSeg : kDiff;  // RAW segments: FORMAT.md 2.7
     const uint32_t nseg = hdr >> 16;
     if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;
     uint32_t *desc = reinterpret_cast<uint32_t *>(buf + 4);
@@ -249,14 +259,16 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
             kind = (d >> 16) & 0xFFu;
             eb = d >> 24;
         }
-        const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
+        const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : (kind == kRawSeg ? 4u * len : 0u);
         const uint32_t il = warp_incl_scan(len, lane), id = warp_incl_scan(dlen, lane);
         const uint32_t st = cl + il - len, db = cd + id - dlen;
         if (s < nseg) {
-            bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
-                   st + len > W || st % A != 0;
+            bad |= len == 0 || kind > max_kind ||
+                   (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) || st + len > W ||
+                   st % A != 0;
             if (st < W) atomicOr(&sbits[st >> 5], 1u << (st & 31));
-            const int a = (int)db - (int)st - 1;
+            // DIFF: the code of position p is byte a + p; RAW: its value is at bytes a + 4p
+            const int a = kind == kRawSeg ? (int)db - 4 * (int)st : (int)db - (int)st - 1;
             desc[s] = (uint32_t)(a + 16384) | (kind << 16) | (eb << 24);
         }
         cl += __shfl_sync(0xffffffffu, il, 31);
@@ -333,6 +345,12 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
             for (int j = 0; j < 8; j++) { hj[j] = si.h; scj[j] = si.sc; }
             started = (sb & 1u) ? 0xFFu : 0u;
             keep = si.kind == kRepeat ? 0xFFu : (sb & 1u);
+            if (act && si.kind == kRawSeg) {  // RAW segment: every position is its stored value
+#pragma unroll
+                for (int j = 0; j < 8; j++)
+                    if ((valid >> j) & 1u) hj[j] = lds_f32_any(dl_s + (uint32_t)(si.a + 4 * (int)(p0 + j)));
+                keep = 0xFFu;
+            }
             bigm = si.big ? 0xFFu : 0u;
         } else {
             // general path: segment heads inside the lane's 8 positions
@@ -342,6 +360,8 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
 #pragma unroll
             for (int j = 0; j < 8; j++) {
                 const uint32_t p = p0 + j;
+                float hraw = 0.f;
+                bool israw = false;
                 if ((sb >> j) & 1u) {
                     s++;
                     si = seg_info(desc, heads, s);
@@ -349,17 +369,22 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
                     run = 0.f;
                     started |= 0xFFu << j;
                     keep |= 1u << j;
+                    israw = si.kind == kRawSeg;
                 } else if ((valid >> j) & 1u) {
                     if (si.kind == kRepeat) {
                         keep |= 1u << j;
+                    } else if (si.kind == kRawSeg) {
+                        keep |= 1u << j;
+                        israw = true;
                     } else {
                         const float f = code_f_byte(dl[si.a + (int)p]);
                         run += f;
                         pl += f;
                     }
                 }
+                if (israw) hraw = lds_f32_any(dl_s + (uint32_t)(si.a + 4 * (int)p));
                 r[j] = run;
-                hj[j] = si.h;
+                hj[j] = israw ? hraw : si.h;
                 scj[j] = si.sc;
                 if (si.big) bigm |= 1u << j;
             }

@@ -27,8 +27,8 @@ constexpr int kEscBlock = 256;                   // voxels per eidx entry
 // DeepCAM header field offsets (FORMAT.md 2.1)
 namespace deepcam {
 constexpr int kC = 8, kH = 10, kW = 12, kAlign = 14, kL = 16, kDirOff = 24, kPayloadOff = 32, kTotal = 40;
-constexpr uint8_t kModeRaw = 0, kModeSeg = 1, kModeRaw16 = 2;  // RAW16: FORMAT.md 2.6
-constexpr uint8_t kRepeat = 0, kDiff = 1;
+constexpr uint8_t kModeRaw = 0, kModeSeg = 1, kModeRaw16 = 2, kModeSegRaw = 3;  // 2.6 RAW16, 2.7 SEG+RAW
+constexpr uint8_t kRepeat = 0, kDiff = 1, kRawSeg = 2;  // kRawSeg: FORMAT.md 2.7
 constexpr int kEminBias = 150;                   // emin = emin_b - 150
 constexpr int kEminBMin = 1, kEminBMax = 246;    // emin in [-149, 96]
 constexpr int kRepeatMin = 16;                   // encoder: identical run that opens a REPEAT

@@ -59,11 +59,12 @@ def deepcam_line(b, hdr, l):
     return dict(mode=1, size=len(p), nseg=nseg, segs=segs, delta=p[4 + 8 * nseg:])
 
 
-def build_seg_line(W, segs, deltas):
+def build_seg_line(W, segs, deltas, mode=1):
     """Assemble one SEG line payload by hand (FORMAT.md 2.1).  segs: list of
-    (len, kind, emin_b, head_f32); deltas: bytes for the DIFF segments."""
+    (len, kind, emin_b, head_f32); deltas: the delta-area bytes (DIFF codes;
+    with mode 3 also the binary32 values of RAW segments, FORMAT.md 2.7)."""
     n = len(segs)
-    out = bytearray(struct.pack("<BBH", 1, 0, n))
+    out = bytearray(struct.pack("<BBH", mode, 0, n))
     for ln, kind, eb, _ in segs:
         out += struct.pack("<HBB", ln, kind, eb)
     for _, _, _, h in segs:

@@ -454,6 +454,29 @@ def test_deepcam_handbuilt_lines(dev, orc, W):
     _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, "f32"))
 
 
+@pytest.mark.parametrize("W,A", [(64, 8), (37, 1), (1152, 36)])
+def test_deepcam_raw_segment_lines(dev, orc, W, A):
+    """FORMAT.md 2.7 lines (SEG with RAW segments, decoded on KD's general line
+    path) mixed with plain SEG and RAW lines: bit-exact, normalised and x-hat."""
+    from tests.test_oracle_pins import _raw_segment_line
+    rng = np.random.default_rng(100 + W)
+    C, H = 2, 12
+    lines = []
+    for l in range(C * H):
+        if l % 4 == 3:
+            lines.append(fmt.build_raw_line(rng.standard_normal(W).astype(np.float32)))
+        else:
+            lines.append(_raw_segment_line(rng, W, A)[l % 4 == 2])
+    b = fmt.build_deepcam_stream(C, H, W, lines, A=A)
+    shift, scale = np.float32([0.5, -3.0]), np.float32([2.0, 1e-3])
+    for out, sh, sc in (("f16", shift, scale), ("f32", shift, scale), ("f32", None, None)):
+        got, st = _decode("deepcam", [b, b], (C, H, W), out=out, shift=sh, scale=sc)
+        assert st == 0
+        want = _dc_ref(orc, b, (C, H, W), sh, sc, out)
+        _same_bits(got[0], want)
+        _same_bits(got[1], want)
+
+
 _EB_EDGES = [1, 2, 3, 4, 5, 6, 7, 60, 120, 147, 148, 149, 170, 200, 246]
 
 

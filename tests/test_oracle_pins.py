@@ -633,6 +633,60 @@ def test_deepcam_raw16_lines(orc, budget):
     assert n16 > 0 and b1.size < b0.size
 
 
+def _raw_segment_line(rng, W, A):
+    """(mode-3 line, the same line with each RAW segment replaced by a REPEAT
+    of 0, the RAW segments as (start, values)) -- FORMAT.md 2.7."""
+    segs3, segs1, d3, d1, raws, pos = [], [], bytearray(), bytearray(), [], 0
+    while pos < W:
+        ln = min(W - pos, A * int(rng.integers(1, 4)))
+        kind = int(rng.integers(0, 3))
+        h = np.float32(rng.standard_normal() * 10.0 ** rng.integers(-3, 4))
+        if kind == 2:
+            v = (rng.standard_normal(ln) * 10.0 ** rng.integers(-30, 30)).astype(np.float32)
+            v[rng.integers(0, ln)] = np.float32(2.0 ** -140)
+            segs3.append((ln, 2, 0, v[0]))
+            d3 += v.astype("<f4").tobytes()
+            segs1.append((ln, 0, 0, np.float32(0.0)))
+            raws.append((pos, v))
+        else:
+            eb = int(rng.integers(100, 160))
+            segs3.append((ln, kind, eb, h))
+            segs1.append((ln, kind, eb, h))
+            if kind == 1:
+                codes = bytes(int(c) for c in rng.integers(0, 256, size=ln - 1))
+                d3 += codes
+                d1 += codes
+        pos += ln
+    return fmt.build_seg_line(W, segs3, d3, mode=3), fmt.build_seg_line(W, segs1, d1), raws
+
+
+@pytest.mark.parametrize("W,A", [(64, 8), (37, 1), (1152, 36)])
+def test_deepcam_raw_segments_decode(orc, W, A):
+    """FORMAT.md 2.7 lines (SEG with RAW segments): a RAW segment's positions
+    are its stored binary32 values, and every other position decodes exactly
+    as in the same line with that segment made a REPEAT (segments decode
+    independently), which pins the 4-bytes-per-value delta-area layout."""
+    rng = np.random.default_rng(W)
+    for _ in range(8):
+        l3, l1, raws = _raw_segment_line(rng, W, A)
+        b3 = fmt.build_deepcam_stream(1, 1, W, [l3], A=A)
+        b1 = fmt.build_deepcam_stream(1, 1, W, [l1], A=A)
+        x3, x1 = orc.deepcam_decode_line(b3, 0, W), orc.deepcam_decode_line(b1, 0, W)
+        mask = np.ones(W, bool)
+        for st, v in raws:
+            assert np.array_equal(x3[st:st + len(v)].view(np.uint32), v.view(np.uint32))
+            mask[st:st + len(v)] = False
+        assert np.array_equal(x3[mask].view(np.uint32), x1[mask].view(np.uint32))
+    # RAW segments are not allowed in mode-1 lines
+    l3, _, raws = _raw_segment_line(np.random.default_rng(1), W, A)
+    while not raws:
+        l3, _, raws = _raw_segment_line(np.random.default_rng(len(l3)), W, A)
+    bad = bytearray(l3)
+    bad[0] = 1
+    with pytest.raises(Exception):
+        orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [bytes(bad)], A=A), 0, W)
+
+
 def test_deepcam_special_shapes(orc):
     for (C, H, W) in ((1, 1, 1), (1, 3, 2), (2, 2, 17), (1, 1, 16)):
         x = np.random.default_rng(C * 100 + W).standard_normal((C, H, W)).astype(np.float32)
