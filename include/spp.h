@@ -136,6 +136,9 @@ typedef struct {
     float rel_err;
     int err_budget;
     int raw16;
+    int raw_segments;  /* 1 = a line over the error budget may keep only its offending
+                          A-blocks raw, as RAW segments of a mode-3 line (FORMAT.md 2.7),
+                          when that is smaller and within the budget; 0 (default) = off */
 } spp_deepcam_params;
 
 /* spp_encode_deepcam with explicit policy knobs (params may be NULL = defaults);

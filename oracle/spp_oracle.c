@@ -557,22 +557,22 @@ static int ceil_log2(double q) {
  * byte size, or -1 if no aligned segmentation exists (the line is then RAW). */
 typedef struct { int len, kind, emin_b; float head; } seg_t;
 
-static int rep_len(const int *run, int i, int W, int A) {
-    int r = run[i];
-    return (i + r == W) ? r : (r / A) * A;
+/* identical run at i, cut at the range end E (E = W for a whole line) */
+static int rep_len(const int *run, int i, int E, int A) {
+    int r = run[i] < E - i ? run[i] : E - i;
+    return (i + r == E) ? r : (r / A) * A;
 }
 
-static int64_t encode_line(const float *x, int W, int A, int lookahead, int repeat_min, seg_t *segs,
-                           int *nseg_out, uint8_t *deltas, int64_t *ndelta_out, int *run) {
-    /* run lengths of bit-identical values */
-    run[W - 1] = 1;
-    for (int i = W - 2; i >= 0; i--)
-        run[i] = (bits_of_f32(x[i]) == bits_of_f32(x[i + 1])) ? run[i + 1] + 1 : 1;
-    int nseg = 0;
-    int64_t nd = 0;
-    int i = 0;
-    while (i < W) {
-        int rl = rep_len(run, i, W, A);
+/* The greedy policy of FORMAT.md 2.4 over positions [i0, E) of a line (E = W
+ * for the whole line; 2.7 encodes the ranges between RAW segments), appending
+ * to segs / deltas.  Returns -1 when no aligned segmentation exists. */
+static int encode_range(const float *x, int i0, int E, int A, int lookahead, int repeat_min, seg_t *segs,
+                        int *nseg_io, uint8_t *deltas, int64_t *nd_io, const int *run) {
+    int nseg = *nseg_io;
+    int64_t nd = *nd_io;
+    int i = i0;
+    while (i < E) {
+        int rl = rep_len(run, i, E, A);
         if (rl >= repeat_min) {
             segs[nseg].len = rl; segs[nseg].kind = 0; segs[nseg].emin_b = 0; segs[nseg].head = x[i];
             nseg++;
@@ -581,7 +581,7 @@ static int64_t encode_line(const float *x, int W, int A, int lookahead, int repe
         }
         float h = x[i];
         double m = 0.0;
-        for (int j = i + 1; j < W && j < i + lookahead; j++) {
+        for (int j = i + 1; j < E && j < i + lookahead; j++) {
             double d = fabs((double)x[j] - (double)x[j - 1]);
             if (d > m) m = d;
         }
@@ -599,8 +599,8 @@ static int64_t encode_line(const float *x, int W, int A, int lookahead, int repe
             float prev = h;
             int j = i + 1, overflow = 0;
             nd = nd0;
-            while (j < W) {
-                if (j % A == 0 && rep_len(run, j, W, A) >= repeat_min) break;
+            while (j < E) {
+                if (j % A == 0 && rep_len(run, j, E, A) >= repeat_min) break;
                 double t = ldexp((double)x[j] - (double)prev, -emin);
                 if (fabs(t) > 1984.5) { overflow = 1; break; }
                 int b = quantise(t);
@@ -622,6 +622,20 @@ static int64_t encode_line(const float *x, int W, int A, int lookahead, int repe
         nseg++;
         i = end;
     }
+    *nseg_io = nseg;
+    *nd_io = nd;
+    return 0;
+}
+
+static int64_t encode_line(const float *x, int W, int A, int lookahead, int repeat_min, seg_t *segs,
+                           int *nseg_out, uint8_t *deltas, int64_t *ndelta_out, int *run) {
+    /* run lengths of bit-identical values */
+    run[W - 1] = 1;
+    for (int i = W - 2; i >= 0; i--)
+        run[i] = (bits_of_f32(x[i]) == bits_of_f32(x[i + 1])) ? run[i + 1] + 1 : 1;
+    int nseg = 0;
+    int64_t nd = 0;
+    if (encode_range(x, 0, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) < 0) return -1;
     *nseg_out = nseg;
     *ndelta_out = nd;
     return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
@@ -657,6 +671,12 @@ int orc_deepcam_encode_p(const float *x, int C, int H, int W, int A, int lookahe
 }
 int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
                          int err_budget, int raw16, uint8_t *dst, size_t cap, size_t *size);
+int orc_deepcam_encode_s(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, int rawseg, uint8_t *dst, size_t cap, size_t *size);
+int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_deepcam_encode_s(x, C, H, W, A, lookahead, repeat_min, rel_err, err_budget, raw16, 0, dst, cap, size);
+}
 int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
                          int err_budget, uint8_t *dst, size_t cap, size_t *size) {
     return orc_deepcam_encode_r(x, C, H, W, A, lookahead, repeat_min, rel_err, err_budget, 0, dst, cap, size);
@@ -684,7 +704,9 @@ static int line_bad_count(const float *x, const seg_t *segs, int nseg, const uin
     int64_t d = 0;
     for (int s = 0; s < nseg; s++) {
         float h = segs[s].head;
-        if (segs[s].kind == 0) {
+        if (segs[s].kind == 2) {                           /* RAW segment: exact (FORMAT.md 2.7) */
+            d += 4 * (int64_t)segs[s].len;
+        } else if (segs[s].kind == 0) {
             for (int j = 0; j < segs[s].len; j++) if (fabs((double)h - (double)x[pos + j]) > rel * fabs((double)x[pos + j])) bad++;
         } else {
             float unit = ldexpf(1.0f, segs[s].emin_b - 150);
@@ -701,10 +723,64 @@ static int line_bad_count(const float *x, const seg_t *segs, int nseg, const uin
     return bad;
 }
 
-int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
-                         int err_budget, int raw16, uint8_t *dst, size_t cap, size_t *size) {
+/* FORMAT.md 2.7 encoder step: the blocks [bA, bA + A) holding a value above
+ * rel in the 2.4 encoding (segs0 / deltas0) become RAW segments (a run of
+ * them, one segment); the ranges between are re-encoded by the 2.4 policy.
+ * Returns the line's SEG size, or -1. */
+static int64_t encode_line_rawseg(const float *x, int W, int A, int lookahead, int repeat_min, double rel,
+                                  const seg_t *segs0, int nseg0, const uint8_t *deltas0, const int *run,
+                                  uint8_t *flag, seg_t *segs, int *nseg_out, uint8_t *deltas, int64_t *nd_out) {
+    /* x-hat of the 2.4 encoding, position by position (FORMAT.md 2.3) */
+    int pos = 0;
+    int64_t d = 0;
+    for (int s = 0; s < nseg0; s++) {
+        float h = segs0[s].head;
+        if (segs0[s].kind == 0) {
+            for (int j = 0; j < segs0[s].len; j++) flag[pos + j] = fabs((double)h - (double)x[pos + j]) > rel * fabs((double)x[pos + j]);
+        } else {
+            float unit = ldexpf(1.0f, segs0[s].emin_b - 150);
+            int64_t S = 0;
+            flag[pos] = fabs((double)h - (double)x[pos]) > rel * fabs((double)x[pos]);
+            for (int j = 1; j < segs0[s].len; j++) {
+                S += orc_deepcam_code(deltas0[d++]);
+                float xh = h + (float)S * unit;
+                flag[pos + j] = fabs((double)xh - (double)x[pos + j]) > rel * fabs((double)x[pos + j]);
+            }
+        }
+        pos += segs0[s].len;
+    }
+    int nb = (W + A - 1) / A, nseg = 0;
+    int64_t nd = 0;
+    int b = 0;
+    while (b < nb) {
+        int bad_b = 0;
+        for (int k = b * A; k < W && k < (b + 1) * A; k++) bad_b |= flag[k];
+        int b2 = b + 1;
+        for (; b2 < nb; b2++) {
+            int bb = 0;
+            for (int k = b2 * A; k < W && k < (b2 + 1) * A; k++) bb |= flag[k];
+            if (bb != bad_b) break;
+        }
+        int s0 = b * A, e0 = b2 * A < W ? b2 * A : W;
+        if (bad_b) {
+            segs[nseg].len = e0 - s0; segs[nseg].kind = 2; segs[nseg].emin_b = 0; segs[nseg].head = x[s0];
+            nseg++;
+            for (int k = s0; k < e0; k++) { wr32(deltas + nd, bits_of_f32(x[k])); nd += 4; }
+        } else if (encode_range(x, s0, e0, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) < 0) {
+            return -1;
+        }
+        b = b2;
+    }
+    *nseg_out = nseg;
+    *nd_out = nd;
+    return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
+}
+
+int orc_deepcam_encode_s(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, int rawseg, uint8_t *dst, size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     if (raw16 != 0 && raw16 != 1) return ORC_EINVAL;
+    if (rawseg != 0 && rawseg != 1) return ORC_EINVAL;
     uint64_t raw16_size = up16(16 + 2 * (uint64_t)W);
     if (lookahead < 2 || lookahead > 65535 || repeat_min < 2 || repeat_min > 65535) return ORC_EINVAL;
     if (err_budget < 0 || !(rel_err > 0.0f) || !(rel_err < 1e30f)) return ORC_EINVAL;
@@ -716,6 +792,10 @@ int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahe
     seg_t *segs = malloc(sizeof(seg_t) * (size_t)W);
     uint8_t *deltas = malloc((size_t)W);
     int *run = malloc(sizeof(int) * (size_t)W);
+    seg_t *segs2 = malloc(sizeof(seg_t) * (size_t)W);      /* FORMAT.md 2.7 candidate line */
+    uint8_t *deltas2 = malloc(5 * (size_t)W), *flag = malloc((size_t)W);
+    int nseg2 = 0;
+    int64_t nd2 = 0;
     /* pass 1: sizes */
     uint64_t pay = 0;
     for (uint64_t l = 0; l < L; l++) {
@@ -729,6 +809,12 @@ int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahe
             if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
                 seg_size = -1;                            /* over the error budget: RAW (FORMAT.md 2.5) */
                 if (raw16 && raw16_ok(xl, W, rel_err)) sz = raw16_size;   /* ... in binary16 (2.6) */
+                if (rawseg) {                             /* ... or with RAW segments (2.7) */
+                    int64_t rs = encode_line_rawseg(xl, W, A, lookahead, repeat_min, rel_err, segs, nseg, deltas, run,
+                                                    flag, segs2, &nseg2, deltas2, &nd2);
+                    if (rs >= 0 && (uint64_t)rs < sz && line_bad_count(xl, segs2, nseg2, deltas2, rel_err) < err_budget)
+                        sz = (uint64_t)rs;
+                }
             }
             if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
         }
@@ -736,8 +822,10 @@ int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahe
     }
     uint64_t total = payload_off + pay;
     *size = (size_t)total;
-    if (total > 0xFFFFFFFFull + payload_off) { free(segs); free(deltas); free(run); return ORC_EINVAL; }
-    if (!dst || cap < total) { free(segs); free(deltas); free(run); return ORC_ESMALL; }
+    if (total > 0xFFFFFFFFull + payload_off || !dst || cap < total) {
+        free(segs); free(deltas); free(run); free(segs2); free(deltas2); free(flag);
+        return total > 0xFFFFFFFFull + payload_off ? ORC_EINVAL : ORC_ESMALL;
+    }
     memset(dst, 0, (size_t)total);
     wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);
     wr16(dst + 8, (uint16_t)C); wr16(dst + 10, (uint16_t)H); wr16(dst + 12, (uint16_t)W);
@@ -753,12 +841,32 @@ int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahe
         for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
         int nseg = 0; int64_t nd = 0;
         int64_t seg_size = finite ? encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) : -1;
-        int use16 = 0;
+        int use16 = 0, use3 = 0;
         if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
             seg_size = -1;
             use16 = raw16 && raw16_ok(xl, W, rel_err);
+            if (rawseg) {
+                uint64_t alt = use16 ? raw16_size : raw_size;
+                int64_t rs = encode_line_rawseg(xl, W, A, lookahead, repeat_min, rel_err, segs, nseg, deltas, run,
+                                                flag, segs2, &nseg2, deltas2, &nd2);
+                if (rs >= 0 && (uint64_t)rs < alt && line_bad_count(xl, segs2, nseg2, deltas2, rel_err) < err_budget) {
+                    use3 = 1;
+                    use16 = 0;
+                    p[0] = 3; wr16(p + 2, (uint16_t)nseg2);
+                    for (int s = 0; s < nseg2; s++) {
+                        wr16(p + 4 + 4 * s, (uint16_t)segs2[s].len);
+                        p[4 + 4 * s + 2] = (uint8_t)segs2[s].kind;
+                        p[4 + 4 * s + 3] = (uint8_t)segs2[s].emin_b;
+                        wr32(p + 4 + 4 * (uint64_t)nseg2 + 4 * s, bits_of_f32(segs2[s].head));
+                    }
+                    memcpy(p + 4 + 8 * (uint64_t)nseg2, deltas2, (size_t)nd2);
+                    cur += (uint64_t)rs;
+                }
+            }
         }
-        if (use16) {
+        if (use3) {
+            /* written above */
+        } else if (use16) {
             p[0] = 2;
             for (int k = 0; k < W; k++) wr16(p + 16 + 2 * (uint64_t)k, orc_f32_to_f16(xl[k]));
             cur += raw16_size;
@@ -779,7 +887,7 @@ int orc_deepcam_encode_r(const float *x, int C, int H, int W, int A, int lookahe
         }
     }
     wr32(dst + dir_off + 4 * L, (uint32_t)cur);
-    free(segs); free(deltas); free(run);
+    free(segs); free(deltas); free(run); free(segs2); free(deltas2); free(flag);
     return ORC_OK;
 }
 

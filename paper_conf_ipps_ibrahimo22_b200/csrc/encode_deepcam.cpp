@@ -80,9 +80,10 @@ struct LineEncoder {
         deltas.reserve(w);
     }
 
-    int rep(int i) const {
-        const int r = run[i];
-        return i + r == W ? r : (r / A) * A;
+    // identical run at i, cut at the range end E (E = W for a whole line)
+    int rep(int i, int E) const {
+        const int r = run[i] < E - i ? run[i] : E - i;
+        return i + r == E ? r : (r / A) * A;
     }
 
     // SEG payload size, or -1 when no aligned segmentation exists (RAW)
@@ -91,9 +92,16 @@ struct LineEncoder {
         deltas.clear();
         run[W - 1] = 1;
         for (int i = W - 2; i >= 0; i--) run[i] = fbits(x[i]) == fbits(x[i + 1]) ? run[i + 1] + 1 : 1;
-        int i = 0;
-        while (i < W) {
-            const int rl = rep(i);
+        if (!encode_range(x, 0, W)) return -1;
+        return (int64_t)round_up16(4 + 8 * (uint64_t)segs.size() + deltas.size());
+    }
+
+    // the FORMAT.md 2.4 greedy policy over positions [i, E), appended to segs /
+    // deltas (2.7 re-encodes the ranges between RAW segments); false when no
+    // aligned segmentation exists
+    bool encode_range(const float *x, int i, const int E) {
+        while (i < E) {
+            const int rl = rep(i, E);
             if (rl >= repeat_min) {
                 segs.push_back(Seg{(uint16_t)rl, kRepeat, 0, x[i]});
                 i += rl;
@@ -101,7 +109,7 @@ struct LineEncoder {
             }
             const float h = x[i];
             double m = 0.0;
-            const int jend = (i + lookahead < W) ? i + lookahead : W;
+            const int jend = (i + lookahead < E) ? i + lookahead : E;
             for (int j = i + 1; j < jend; j++) {
                 double d = fabs((double)x[j] - (double)x[j - 1]);
                 if (d > m) m = d;
@@ -120,8 +128,8 @@ struct LineEncoder {
                 float prev = h;
                 int j = i + 1;
                 bool overflow = false;
-                for (; j < W; j++) {
-                    if (j % A == 0 && rep(j) >= repeat_min) break;
+                for (; j < E; j++) {
+                    if (j % A == 0 && rep(j, E) >= repeat_min) break;
                     double t = ldexp((double)x[j] - (double)prev, -emin);
                     if (fabs(t) > kMaxCode + 0.5) { overflow = true; break; }
                     int k;
@@ -134,13 +142,13 @@ struct LineEncoder {
                 if (!overflow) { end = j; break; }
                 end = (j / A) * A;
                 if (end > i) { deltas.resize(nd0 + (size_t)(end - i - 1)); break; }
-                if (emin >= 96) return -1;
+                if (emin >= 96) return false;
                 emin++;
             }
             segs.push_back(Seg{(uint16_t)(end - i), kDiff, (uint8_t)(emin + kEminBias), h});
             i = end;
         }
-        return (int64_t)round_up16(4 + 8 * (uint64_t)segs.size() + deltas.size());
+        return true;
     }
 };
 
@@ -153,7 +161,9 @@ int bad_values(const LineEncoder &e, const float *x, double rel) {
     size_t d = 0;
     auto over = [&](float xh, float xv) { return fabs((double)xh - (double)xv) > rel * fabs((double)xv); };
     for (const Seg &g : e.segs) {
-        if (g.kind == kRepeat) {
+        if (g.kind == kRawSeg) {  // exact (FORMAT.md 2.7)
+            d += 4 * (size_t)g.len;
+        } else if (g.kind == kRepeat) {
             for (int j = 0; j < g.len; j++) bad += over(g.head, x[pos + j]);
         } else {
             const float unit = ldexpf(1.0f, (int)g.emin_b - kEminBias);
@@ -169,6 +179,60 @@ int bad_values(const LineEncoder &e, const float *x, double rel) {
         pos += g.len;
     }
     return bad;
+}
+
+// FORMAT.md 2.7: from the 2.4 encoding in `e0`, the A-blocks holding a value
+// above rel become RAW segments (a run of them, one segment) and the ranges
+// between are re-encoded by the 2.4 policy, into `e`.  False if no aligned
+// segmentation exists.
+bool encode_rawseg(const LineEncoder &e0, LineEncoder &e, const float *x, double rel, std::vector<uint8_t> &flag) {
+    const int W = e0.W, A = e0.A;
+    flag.assign(W, 0);
+    int pos = 0;
+    size_t d = 0;
+    auto over = [&](float xh, float xv) { return fabs((double)xh - (double)xv) > rel * fabs((double)xv); };
+    for (const Seg &g : e0.segs) {
+        if (g.kind == kRepeat) {
+            for (int j = 0; j < g.len; j++) flag[pos + j] = over(g.head, x[pos + j]);
+        } else {
+            const float unit = ldexpf(1.0f, (int)g.emin_b - kEminBias);
+            int64_t S = 0;
+            flag[pos] = over(g.head, x[pos]);
+            for (int j = 1; j < g.len; j++) {
+                const uint8_t b = e0.deltas[d++];
+                const int mag = kCodes.mag[b & 127];
+                S += (b & 0x80) ? -mag : mag;
+                flag[pos + j] = over(g.head + (float)S * unit, x[pos + j]);
+            }
+        }
+        pos += g.len;
+    }
+    e.segs.clear();
+    e.deltas.clear();
+    e.run = e0.run;
+    const int nb = (W + A - 1) / A;
+    auto block_bad = [&](int b) {
+        for (int k = b * A; k < W && k < (b + 1) * A; k++)
+            if (flag[k]) return true;
+        return false;
+    };
+    int b = 0;
+    while (b < nb) {
+        const bool bad = block_bad(b);
+        int b2 = b + 1;
+        while (b2 < nb && block_bad(b2) == bad) b2++;
+        const int s0 = b * A, e1 = b2 * A < W ? b2 * A : W;
+        if (bad) {
+            e.segs.push_back(Seg{(uint16_t)(e1 - s0), kRawSeg, 0, x[s0]});
+            const size_t at = e.deltas.size();
+            e.deltas.resize(at + 4 * (size_t)(e1 - s0));
+            memcpy(e.deltas.data() + at, x + s0, 4 * (size_t)(e1 - s0));
+        } else if (!e.encode_range(x, s0, e1)) {
+            return false;
+        }
+        b = b2;
+    }
+    return true;
 }
 
 // binary32 -> binary16, round to nearest even (FORMAT.md 2.6 RAW16 lines)
@@ -221,7 +285,9 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     const float rel = params && params->rel_err != 0.0f ? params->rel_err : 0.1f;
     const int budget = params ? params->err_budget : 0;
     const int raw16 = params ? params->raw16 : 0;
+    const int rawseg = params ? params->raw_segments : 0;
     if (raw16 != 0 && raw16 != 1) return SPP_ERR_INVALID_ARG;
+    if (rawseg != 0 && rawseg != 1) return SPP_ERR_INVALID_ARG;
     const uint64_t raw16_size = round_up16(16 + 2 * (uint64_t)W);
     if (la < 2 || la > 65535 || rm < 2 || rm > 65535) return SPP_ERR_INVALID_ARG;
     if (budget < 0 || !(rel > 0.0f) || !(rel < 1e30f)) return SPP_ERR_INVALID_ARG;
@@ -250,8 +316,22 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     std::vector<uint8_t> is_seg(L);
     std::vector<uint32_t> dir(L + 1);
     std::vector<uint64_t> line_size(L);
+    // a line over the error budget: RAW16 (2.6) if allowed, or RAW segments (2.7)
+    // when that is smaller and within the budget; 3 = mode-3 line
+    auto over_budget = [&](LineEncoder &enc, LineEncoder &enc3, std::vector<uint8_t> &flag, const float *xl,
+                           uint64_t &sz) -> uint8_t {
+        uint8_t kind = 0;
+        sz = raw_size;
+        if (raw16 && raw16_ok(xl, W, rel)) { sz = raw16_size; kind = 2; }
+        if (rawseg && encode_rawseg(enc, enc3, xl, rel, flag)) {
+            const uint64_t s3 = round_up16(4 + 8 * (uint64_t)enc3.segs.size() + enc3.deltas.size());
+            if (s3 < sz && bad_values(enc3, xl, rel) < budget) { sz = s3; kind = 3; }
+        }
+        return kind;
+    };
     parallel_lines([&](uint64_t l0, uint64_t l1) {
-        LineEncoder enc(W, A, la, rm);
+        LineEncoder enc(W, A, la, rm), enc3(W, A, la, rm);
+        std::vector<uint8_t> flag;
         for (uint64_t l = l0; l < l1; l++) {
             const float *xl = x + l * (uint64_t)W;
             uint64_t sz = raw_size;
@@ -260,7 +340,7 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
                 int64_t seg = enc.encode(xl);
                 if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) {  // FORMAT.md 2.5
                     seg = -1;
-                    if (raw16 && raw16_ok(xl, W, rel)) { sz = raw16_size; is_seg[l] = 2; }  // 2.6
+                    is_seg[l] = over_budget(enc, enc3, flag, xl, sz);
                 }
                 if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
             }
@@ -295,7 +375,8 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     memcpy(out + dir_off, dir.data(), 4 * (L + 1));
     // pass 2: payloads
     parallel_lines([&](uint64_t l0, uint64_t l1) {
-    LineEncoder enc(W, A, la, rm);
+    LineEncoder enc(W, A, la, rm), enc3(W, A, la, rm);
+    std::vector<uint8_t> flag;
     for (uint64_t l = l0; l < l1; l++) {
         const float *xl = x + l * (uint64_t)W;
         uint8_t *p = out + payload_off + dir[l];
@@ -313,8 +394,16 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
             continue;
         }
         enc.encode(xl);
+        uint8_t mode = kModeSeg;
+        if (is_seg[l] == 3) {  // FORMAT.md 2.7: rebuild the RAW-segment line (deterministic)
+            uint64_t sz;
+            over_budget(enc, enc3, flag, xl, sz);
+            std::swap(enc.segs, enc3.segs);
+            std::swap(enc.deltas, enc3.deltas);
+            mode = kModeSegRaw;
+        }
         const uint16_t nseg = (uint16_t)enc.segs.size();
-        p[0] = kModeSeg;
+        p[0] = mode;
         memcpy(p + 2, &nseg, 2);
         for (int s = 0; s < nseg; s++) {
             const Seg &g = enc.segs[s];

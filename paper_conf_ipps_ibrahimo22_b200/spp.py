@@ -46,7 +46,7 @@ class spp_cosmo_params(C.Structure):
 
 class spp_deepcam_params(C.Structure):
     _fields_ = [("lookahead", C.c_int), ("repeat_min", C.c_int), ("rel_err", C.c_float), ("err_budget", C.c_int),
-                ("raw16", C.c_int)]
+                ("raw16", C.c_int), ("raw_segments", C.c_int)]
 
 
 class spp_decode_opts(C.Structure):
@@ -141,7 +141,7 @@ def spp_deepcam_max_encoded_size(Cc: int, H: int, W: int) -> int:
 
 
 def spp_encode_deepcam(x: np.ndarray, lookahead: int = 0, repeat_min: int = 0, rel_err: float = 0.0,
-                       err_budget: int = 0, raw16: bool = False) -> np.ndarray:
+                       err_budget: int = 0, raw16: bool = False, raw_segments: bool = False) -> np.ndarray:
     """fp32 [C, H, W] -> encoded uint8 stream (FORMAT.md 2); nonzero knobs go
     through spp_encode_deepcam_ex (0 = the FORMAT.md 2.4 default; err_budget
     > 0 = the FORMAT.md 2.5 error budget at relative error rel_err)."""
@@ -152,8 +152,9 @@ def spp_encode_deepcam(x: np.ndarray, lookahead: int = 0, repeat_min: int = 0, r
     cap = spp_deepcam_max_encoded_size(Cc, H, W)
     dst = np.empty(max(cap, 64), dtype=np.uint8)
     size = C.c_size_t(0)
-    if lookahead or repeat_min or rel_err or err_budget or raw16:
-        prm = spp_deepcam_params(int(lookahead), int(repeat_min), float(rel_err), int(err_budget), int(bool(raw16)))
+    if lookahead or repeat_min or rel_err or err_budget or raw16 or raw_segments:
+        prm = spp_deepcam_params(int(lookahead), int(repeat_min), float(rel_err), int(err_budget), int(bool(raw16)),
+                                 int(bool(raw_segments)))
         _check(load().spp_encode_deepcam_ex(a.ctypes.data, Cc, H, W, C.byref(prm), dst.ctypes.data, dst.size,
                                             C.byref(size)), "spp_encode_deepcam_ex")
     else:

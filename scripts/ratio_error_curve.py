@@ -47,12 +47,15 @@ def main():
     # FORMAT.md 2.5 error budget: a line with >= k values above 10% error stays RAW
     settings += [(0, 0, k) for k in (256, 64, 16, 4, 1)]
     settings += [(0, 0, -k) for k in (64, 16, 4, 1)]   # negative: the same budgets with RAW16 lines (2.6)
+    settings += [(0, 0, 10000 + k) for k in (64, 16, 4, 1)]   # +10000: budgets with RAW segments (2.7)
+    settings += [(0, 0, -(10000 + k)) for k in (16, 1)]       # both
     for la, rm, budget in settings:
         nbytes, bad, tot, bad_p, tot_p, med = 0, 0, 0, 0, 0, []
         nseg = 0
         nraw = 0
         for x in xs:
-            b = spp.spp_encode_deepcam(x, la, rm, err_budget=abs(budget), raw16=budget < 0)
+            b = spp.spp_encode_deepcam(x, la, rm, err_budget=abs(budget) % 10000, raw16=budget < 0,
+                                       raw_segments=abs(budget) > 10000)
             nbytes += b.size
             info = spp.spp_stream_info("deepcam", b)
             nraw += info[0]
@@ -68,7 +71,8 @@ def main():
             tot_p += r[precip].size
             med.append(float(np.median(r)))
         vals = args.samples * C * H * W
-        rows.append({"lookahead": la or 64, "repeat_min": rm or 16, "err_budget": abs(budget), "raw16": budget < 0,
+        rows.append({"lookahead": la or 64, "repeat_min": rm or 16, "err_budget": abs(budget) % 10000,
+                     "raw16": budget < 0, "raw_segments": abs(budget) > 10000,
                      "bytes_per_value": nbytes / vals,
                      "ratio_vs_fp32": 4.0 * vals / nbytes, "frac_rel_err_gt_10pct": bad / tot,
                      "frac_rel_err_gt_10pct_precip_channel": bad_p / max(1, tot_p),

@@ -56,7 +56,7 @@ def deepcam_line(b, hdr, l):
         ln, kind, eb = struct.unpack_from("<HBB", p, 4 + 4 * s)
         h = struct.unpack_from("<f", p, 4 + 4 * nseg + 4 * s)[0]
         segs.append(dict(len=ln, kind=kind, emin_b=eb, emin=eb - 150, head=np.float32(h)))
-    return dict(mode=1, size=len(p), nseg=nseg, segs=segs, delta=p[4 + 8 * nseg:])
+    return dict(mode=int(p[0]), size=len(p), nseg=nseg, segs=segs, delta=p[4 + 8 * nseg:])
 
 
 def build_seg_line(W, segs, deltas, mode=1):

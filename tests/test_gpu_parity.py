@@ -379,6 +379,25 @@ def test_deepcam_raw16_streams(dev, orc, budget):
         _same_bits(got[1], want)
 
 
+@pytest.mark.parametrize("budget,raw16", [(1, False), (4, True)])
+def test_deepcam_raw_segment_streams(dev, orc, budget, raw16):
+    """FORMAT.md 2.7 streams from the encoder (error budget + RAW segments) on
+    the full C3 shape: mode-3 lines among SEG (and RAW16) lines, bit-exact."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2013)
+    mean, rstd = deepcam_stats(x)
+    b = spp.spp_encode_deepcam(x, err_budget=budget, raw16=raw16, raw_segments=True)
+    h = fmt.deepcam_header(b)
+    assert 3 in {fmt.deepcam_line(b, h, l)["mode"] for l in range(0, h["L"], 3)}
+    for out, sh, sc in (("f16", mean, rstd), ("f32", None, None)):
+        got, st = _decode("deepcam", [b, b], x.shape, out=out, shift=sh, scale=sc)
+        assert st == 0
+        want = _dc_ref(orc, b, x.shape, sh, sc, out)
+        _same_bits(got[0], want)
+        _same_bits(got[1], want)
+
+
 @pytest.mark.parametrize("W", [37, 64])
 def test_deepcam_raw16_narrow_lines(dev, orc, W):
     """RAW16, RAW and SEG lines on the scalar (W = 37) and 8-wide (W = 64)

@@ -194,9 +194,10 @@ def test_deepcam_error_budget_matches_oracle(spp, orc, rel, budget):
     from synth import gen_deepcam
     x = gen_deepcam(2005, H=16)
     for raw16 in (False, True):
-        a = spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget, raw16=raw16)
-        b = orc.deepcam_encode(x, rel_err=rel, err_budget=budget, raw16=raw16)
-        assert a.size == b.size and np.array_equal(a, b)
+        for rawseg in (False, True):
+            a = spp.spp_encode_deepcam(x, rel_err=rel, err_budget=budget, raw16=raw16, raw_segments=rawseg)
+            b = orc.deepcam_encode(x, rel_err=rel, err_budget=budget, raw16=raw16, raw_segments=rawseg)
+            assert a.size == b.size and np.array_equal(a, b)
 
 
 def test_deepcam_encoder_knob_errors(spp):

@@ -687,6 +687,58 @@ def test_deepcam_raw_segments_decode(orc, W, A):
         orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [bytes(bad)], A=A), 0, W)
 
 
+@pytest.mark.parametrize("budget", [1, 8])
+def test_deepcam_raw_segment_policy(orc, budget):
+    """FORMAT.md 2.7 policy, checked with numpy on the oracle's own decodes: a
+    line over the budget becomes a mode-3 line whose RAW segments are exactly
+    the runs of A-blocks holding a value above 10% error in its default (2.4)
+    encoding, those values are exact, and the line is within the budget."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2012, H=16)
+    C, H, W = x.shape
+    A = 36
+    b0 = orc.deepcam_encode(x)
+    b3 = orc.deepcam_encode(x, err_budget=budget, raw_segments=True)
+    h0, h3 = fmt.deepcam_header(b0), fmt.deepcam_header(b3)
+    rel = np.float64(np.float32(0.1))
+    n3 = 0
+    for l in range(C * H):
+        c, y = divmod(l, H)
+        xs = x[c, y].astype(np.float64)
+        i0, i3 = fmt.deepcam_line(b0, h0, l), fmt.deepcam_line(b3, h3, l)
+        xh0 = orc.deepcam_decode_line(b0, l, W).astype(np.float64)
+        flags = np.abs(xh0 - xs) > rel * np.abs(xs)
+        if i0["mode"] != 1 or flags.sum() < budget:
+            assert i3 == i0
+            continue
+        if i3["mode"] != 3:                       # the RAW-segment line was not smaller / within budget
+            assert i3["mode"] == 0
+            continue
+        n3 += 1
+        blk = flags.reshape(-1, A).any(axis=1)
+        raw_runs, pos = [], 0
+        for sg in i3["segs"]:
+            if sg["kind"] == 2:
+                raw_runs.append((pos, pos + sg["len"]))
+            pos += sg["len"]
+        want, b = [], 0
+        while b < len(blk):
+            if blk[b]:
+                e = b
+                while e < len(blk) and blk[e]:
+                    e += 1
+                want.append((b * A, e * A))
+                b = e
+            else:
+                b += 1
+        assert raw_runs == want
+        xh3 = orc.deepcam_decode_line(b3, l, W)
+        for s0, e0 in raw_runs:
+            assert np.array_equal(xh3[s0:e0].view(np.uint32), x[c, y, s0:e0].view(np.uint32))
+        assert (np.abs(xh3.astype(np.float64) - xs) > rel * np.abs(xs)).sum() < budget
+    assert n3 > 0 and b3.size < orc.deepcam_encode(x, err_budget=budget).size
+
+
 def test_deepcam_special_shapes(orc):
     for (C, H, W) in ((1, 1, 1), (1, 3, 2), (2, 2, 17), (1, 1, 16)):
         x = np.random.default_rng(C * 100 + W).standard_normal((C, H, W)).astype(np.float32)
