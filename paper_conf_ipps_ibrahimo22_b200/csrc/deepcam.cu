@@ -31,8 +31,10 @@
 //                    (line record by st.async + bytes by TMA) into a 3-slot
 //                    ring; W = 1152 lines with 36-aligned segments decode in
 //                    one warp pass (decode_line_onepass) and leave as one TMA
-//                    bulk store of the staged row.  RAW and RAW16 lines
-//                    (FORMAT.md 2.6) take the general line path.
+//                    bulk store of the staged row; RAW segments of mode-3
+//                    lines (FORMAT.md 2.7) are read there by their lanes.
+//                    RAW and RAW16 lines (FORMAT.md 2.6) take the general
+//                    line path.
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -619,6 +621,9 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     constexpr int VPL = 36;
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
+    // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
+    // it never has more than 32 segments, so the fallback sees only mode 1
+    const uint32_t max_kind = (hdr & 0xFFu) == kModeSegRaw ? kRawSeg : kDiff;
     if (nseg > (uint32_t)kWarp) return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, lane);
     if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
     const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
@@ -632,19 +637,21 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
         eb = d >> 24;
         hs = reinterpret_cast<const float *>(buf + 4 + 4 * nseg)[lane];
     }
-    const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : 0;
+    const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : (kind == kRawSeg ? 4u * len : 0u);
     const uint32_t pk = len | (dlen << 16);
     const uint32_t inc = warp_incl_scan(pk, lane);
     const uint32_t ex = inc - pk;
     const uint32_t st = ex & 0xFFFFu, db = ex >> 16;
     const uint32_t blk = st / VPL;
-    bool bad = have && (len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
+    bool bad = have && (len == 0 || kind > max_kind || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
                         st + len > W || blk * VPL != st);
     const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
     bad = __any_sync(0xffffffffu, bad) || (tot & 0xFFFFu) != W || 4u + 8u * nseg + (tot >> 16) > bytes;
     if (bad) return false;
     const uint32_t word = __reduce_or_sync(0xffffffffu, have ? 1u << blk : 0u);  // head lanes
-    const uint32_t info = (uint32_t)((int)db - (int)st - 1 + 16384) | (kind << 16) | (eb << 24);
+    // DIFF: the code of position p is delta byte a + p; RAW: its value is at bytes a + 4p
+    const int a_s = kind == kRawSeg ? (int)db - 4 * (int)st : (int)db - (int)st - 1;
+    const uint32_t info = (uint32_t)(a_s + 16384) | (kind << 16) | (eb << 24);
 
     const uint32_t le_mask = 0xFFFFFFFFu >> (31 - lane);
     const uint32_t p0 = VPL * lane;
@@ -654,7 +661,8 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const float h = __shfl_sync(0xffffffffu, hs, s);
     const int a = (int)(d & 0xFFFFu) - 16384;
     const uint32_t skind = (d >> 16) & 0xFFu, seb = d >> 24;
-    const bool rep = skind == kRepeat;
+    const bool raw = skind == kRawSeg;
+    const bool rep = skind == kRepeat || raw;  // RAW lanes run the chain on zero codes, then take their values
     Bytes<VPL> bt;
     bt.load(dl_s + (uint32_t)(rep ? 0 : a + (int)p0));
     if (rep) {
@@ -707,6 +715,11 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
         const float2 y2 = fmul2_rn(fadd2_rn(ffma2_rn(S, sc2, h2), nsh2), scv2);
         y[i] = y2.x;
         y[HALF + i] = y2.y;
+    }
+    if (raw) {  // RAW segment lane: x̂ is the stored binary32 value, y = RN(RN(x̂ - shift) * scale)
+        const uint32_t va = dl_s + (uint32_t)(a + 4 * (int)p0);
+#pragma unroll
+        for (int i = 0; i < VPL; i++) y[i] = __fmul_rn(__fadd_rn(lds_f32_any(va + 4u * i), -shv), scv);
     }
     __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
     stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
@@ -844,7 +857,7 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
             }
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (VPL == 36 && buf[0] == kModeSegRaw))) {
                 if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
             }
@@ -1056,7 +1069,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (VPL == 36 && buf[0] == kModeSegRaw))) {
                 if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
             } else {

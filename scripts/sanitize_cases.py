@@ -52,3 +52,17 @@ print("deepcam ok", run("deepcam", [d, d], y.shape))
 print("deepcam bad nseg", run("deepcam", [d, dbad], y.shape))
 print("deepcam truncated", run("deepcam", [dtr, d], y.shape))
 print("deepcam bad dir", run("deepcam", [d, ddir], y.shape, out="f32"))
+# mode-3 lines (FORMAT.md 2.7): RAW segments on the one-pass path; a RAW
+# segment declared in a mode-1 line and a RAW segment longer than the line's
+# bytes must be reported, not read past
+r = spp.spp_encode_deepcam(y, err_budget=1, raw_segments=True)
+hr = fmt.deepcam_header(r)
+l3 = next(l for l in range(hr["L"]) if fmt.deepcam_line(r, hr, l)["mode"] == 3)
+o3 = hr["payload_off"] + int(hr["dir"][l3])
+rm1 = r.copy(); rm1[o3] = 1
+rlen = r.copy()
+seg = next(s for s, g in enumerate(fmt.deepcam_line(r, hr, l3)["segs"]) if g["kind"] == 2)
+rlen[o3 + 4 + 4 * seg: o3 + 6 + 4 * seg] = np.frombuffer(np.uint16(1152).tobytes(), np.uint8)
+print("deepcam raw segments ok", run("deepcam", [r, r], y.shape))
+print("deepcam raw segment in mode 1", run("deepcam", [r, rm1], y.shape))
+print("deepcam raw segment too long", run("deepcam", [rlen, r], y.shape, out="f32"))

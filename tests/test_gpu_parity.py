@@ -618,6 +618,27 @@ def test_deepcam_c4_launch_configuration(dev, orc):
     del out, o16
 
 
+def test_deepcam_raw_segment_onepass_corruption(dev):
+    """W = 1152, A = 36 (the one-pass path): a RAW segment (kind 2) in a mode-1
+    line, and a RAW segment whose 4 len bytes run past the line, are reported
+    as corrupt on the sample that holds them (FORMAT.md 2.7)."""
+    W, A = 1152, 36
+    v = np.arange(A, dtype=np.float32)
+    good = fmt.build_seg_line(W, [(A, 2, 0, v[0]), (W - A, 0, 0, 1.0)], v.astype("<f4").tobytes(), mode=3)
+    in_mode1 = fmt.build_seg_line(W, [(A, 2, 0, v[0]), (W - A, 0, 0, 1.0)], v.astype("<f4").tobytes(), mode=1)
+    too_long = fmt.build_seg_line(W, [(W - A, 2, 0, v[0]), (A, 0, 0, 1.0)], v.astype("<f4").tobytes(), mode=3)
+    ok = fmt.build_deepcam_stream(1, 2, W, [good, good], A=A)
+    for bad in (in_mode1, too_long):
+        b = fmt.build_deepcam_stream(1, 2, W, [good, bad], A=A)
+        _, st = _decode("deepcam", [ok, b], (1, 2, W), out="f16")
+        assert st == (3 | (1 << 8))
+    got, st = _decode("deepcam", [ok], (1, 2, W), out="f32")
+    assert st == 0
+    want = np.concatenate([v, np.ones(W - A, np.float32)])
+    _same_bits(got[0, 0, 0], want)
+    _same_bits(got[0, 0, 1], want)
+
+
 def test_deepcam_corruption_detected(dev):
     W = 64
     good = fmt.build_seg_line(W, [(W, 1, 140, 1.0)], [1] * (W - 1))
