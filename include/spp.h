@@ -176,6 +176,11 @@ typedef struct {
                                 stages them.  0 (default): the paper-format kernel, which reports
                                 such samples as SPP_ERR_UNSUPPORTED in `status` (odd shapes that
                                 take the scalar kernel decode them either way). */
+    int raw_segments;        /* DeepCAM: 1 = the batch may hold FORMAT.md 2.7 mode-3 lines
+                                (spp_encode_deepcam_ex raw_segments = 1): W = 1152 batches use the
+                                KD instance that decodes them in one warp pass.  0 (default): the
+                                mode-1 instance, on which mode-3 lines take the general line path
+                                (same bits, slower).  Other values -> SPP_ERR_INVALID_ARG. */
 } spp_decode_opts;
 
 /* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */

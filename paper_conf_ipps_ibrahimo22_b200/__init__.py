@@ -36,7 +36,7 @@ class Decoder:
     """
 
     def __init__(self, fmt: str, dims, out: str = "f16", transform: int | None = None, device=None,
-                 escape_keys: bool = False):
+                 escape_keys: bool = False, raw_segments: bool = False):
         import torch
         self.torch = torch
         spp.load()
@@ -46,6 +46,7 @@ class Decoder:
         self.out = out
         self.opts = spp_decode_opts_init(fmt, Cc, D, H, W, out=out, transform=transform)
         self.opts.escape_keys = int(bool(escape_keys))  # FORMAT.md 1.5 streams: the staging kernel
+        self.opts.raw_segments = int(bool(raw_segments))  # FORMAT.md 2.7 streams: the mode-3 KD instance
         self.device = torch.device(device or "cuda")
         self.status = torch.zeros(1, dtype=torch.int32, device=self.device)
         self._ws = None

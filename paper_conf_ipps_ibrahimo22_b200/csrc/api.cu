@@ -87,6 +87,7 @@ spp_status spp_decode_batch(spp_format fmt, const void *const *d_src, int n, voi
     if (o.out != SPP_OUT_F16 && o.out != SPP_OUT_F32 && o.out != SPP_OUT_I16) return SPP_ERR_INVALID_ARG;
     if (o.out == SPP_OUT_I16 && (fmt != SPP_FMT_COSMO || o.transform != 0)) return SPP_ERR_INVALID_ARG;
     if (fmt == SPP_FMT_COSMO && o.transform != 0 && o.transform != 1) return SPP_ERR_INVALID_ARG;
+    if (o.raw_segments != 0 && o.raw_segments != 1) return SPP_ERR_INVALID_ARG;
     if (n == 0) return SPP_OK;
     if (!d_src || !d_dst) return SPP_ERR_INVALID_ARG;
     if ((reinterpret_cast<uintptr_t>(d_dst) & 15) != 0) return SPP_ERR_INVALID_ARG;

@@ -615,7 +615,7 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
 // case): lane s holds segment s's table entry in registers; the head lanes form
 // one bitmap word (one warp OR-reduction) and every lane fetches its segment's
 // parameters by shuffle.  Falls back to the shared-memory tables otherwise.
-template <int OUT>
+template <int OUT, bool RAWSEG>  // RAWSEG: a mode-3 line (FORMAT.md 2.7); mode-1 lines run without its code
 __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
                                                     uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
     constexpr int VPL = 36;
@@ -623,7 +623,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const uint32_t nseg = hdr >> 16;
     // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
     // it never has more than 32 segments, so the fallback sees only mode 1
-    const uint32_t max_kind = (hdr & 0xFFu) == kModeSegRaw ? kRawSeg : kDiff;
+    constexpr uint32_t max_kind = RAWSEG ? kRawSeg : kDiff;
     if (nseg > (uint32_t)kWarp) return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, lane);
     if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
     const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
@@ -661,7 +661,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const float h = __shfl_sync(0xffffffffu, hs, s);
     const int a = (int)(d & 0xFFFFu) - 16384;
     const uint32_t skind = (d >> 16) & 0xFFu, seb = d >> 24;
-    const bool raw = skind == kRawSeg;
+    const bool raw = RAWSEG && skind == kRawSeg;
     const bool rep = skind == kRepeat || raw;  // RAW lanes run the chain on zero codes, then take their values
     Bytes<VPL> bt;
     bt.load(dl_s + (uint32_t)(rep ? 0 : a + (int)p0));
@@ -729,6 +729,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     return true;
 }
 
+// mode-3 lines out of line: the mode-1 loop keeps its code footprint
 template <int OUT, bool VEC, int VPL>
 __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decode(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
@@ -857,8 +858,8 @@ __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decod
             }
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (VPL == 36 && buf[0] == kModeSegRaw))) {
-                if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
+                if constexpr (VPL == 36) ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
             }
             else
@@ -909,7 +910,7 @@ constexpr uint32_t kWsNs = SPP_KD_WS_NS;
 static_assert(kWsNs >= 2 && kWsNs <= 8, "slot ring");
 constexpr uint32_t kWsCtl = 32 * kWsNs;  // per consumer: full[NS], empty[NS] mbarriers + info[NS] (16 B each)
 
-template <int OUT, bool VEC, int VPL>
+template <int OUT, bool VEC, int VPL, bool RAWSEG>  // RAWSEG: opts.raw_segments (mode-3 lines in one pass)
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
@@ -1069,8 +1070,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (VPL == 36 && buf[0] == kModeSegRaw))) {
-                if constexpr (VPL == 36) ok = decode_line_onepass<OUT>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (RAWSEG && buf[0] == kModeSegRaw))) {
+                if constexpr (VPL == 36) {
+                    if (!RAWSEG || buf[0] == kModeSeg)
+                        ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                    else
+                        ok = decode_line_onepass<OUT, true>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                }
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
             } else {
                 ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
@@ -1093,7 +1099,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     }
 }
 
-template <int OUT, bool VEC, int VPL>
+template <int OUT, bool VEC, int VPL, bool RAWSEG>
 spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
                         const DeviceProps &dp) {
     const uint32_t W = (uint32_t)o.W;
@@ -1110,7 +1116,7 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
     while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
     if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
     const int smem = wpc * (int)warp_bytes;
-    auto kern = kd_decode_ws<OUT, VEC, VPL>;
+    auto kern = kd_decode_ws<OUT, VEC, VPL, RAWSEG>;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return SPP_ERR_CUDA;
     int occ = 0;
@@ -1172,20 +1178,26 @@ spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const sp
     const bool vec = o.W % 8 == 0 && (reinterpret_cast<uintptr_t>(d_dst) % align) == 0;
     const bool v36 = vec && o.W == 1152;  // the DeepCAM line: 32 lanes x 36 positions, one pass
     spp_status r = SPP_ERR_INVALID_ARG;
+    // opts.raw_segments: the W = 1152 instance that also takes mode-3 lines
+    // (FORMAT.md 2.7) in one pass; without it they take the general line path
+    const bool rs = v36 && o.raw_segments;
 #if SPP_KD_WS
-#define SPP_LAUNCH_KD launch_kd_ws
+#define SPP_LAUNCH_KD(OUT, VEC, VPL) launch_kd_ws<OUT, VEC, VPL, false>(meta, n, d_dst, o, stream, dp)
+#define SPP_LAUNCH_KD_RS(OUT) launch_kd_ws<OUT, true, 36, true>(meta, n, d_dst, o, stream, dp)
 #else
-#define SPP_LAUNCH_KD launch_kd
+#define SPP_LAUNCH_KD(OUT, VEC, VPL) launch_kd<OUT, VEC, VPL>(meta, n, d_dst, o, stream, dp)
+#define SPP_LAUNCH_KD_RS(OUT) launch_kd<OUT, true, 36>(meta, n, d_dst, o, stream, dp)
 #endif
     if (o.out == SPP_OUT_F32)
-        r = v36 ? SPP_LAUNCH_KD<SPP_OUT_F32, true, 36>(meta, n, d_dst, o, stream, dp)
-                : vec ? SPP_LAUNCH_KD<SPP_OUT_F32, true, 8>(meta, n, d_dst, o, stream, dp)
-                      : SPP_LAUNCH_KD<SPP_OUT_F32, false, 8>(meta, n, d_dst, o, stream, dp);
+        r = rs ? SPP_LAUNCH_KD_RS(SPP_OUT_F32)
+               : v36 ? SPP_LAUNCH_KD(SPP_OUT_F32, true, 36)
+                     : vec ? SPP_LAUNCH_KD(SPP_OUT_F32, true, 8) : SPP_LAUNCH_KD(SPP_OUT_F32, false, 8);
     else if (o.out == SPP_OUT_F16)
-        r = v36 ? SPP_LAUNCH_KD<SPP_OUT_F16, true, 36>(meta, n, d_dst, o, stream, dp)
-                : vec ? SPP_LAUNCH_KD<SPP_OUT_F16, true, 8>(meta, n, d_dst, o, stream, dp)
-                      : SPP_LAUNCH_KD<SPP_OUT_F16, false, 8>(meta, n, d_dst, o, stream, dp);
+        r = rs ? SPP_LAUNCH_KD_RS(SPP_OUT_F16)
+               : v36 ? SPP_LAUNCH_KD(SPP_OUT_F16, true, 36)
+                     : vec ? SPP_LAUNCH_KD(SPP_OUT_F16, true, 8) : SPP_LAUNCH_KD(SPP_OUT_F16, false, 8);
 #undef SPP_LAUNCH_KD
+#undef SPP_LAUNCH_KD_RS
     if (r == SPP_OK && ev && cudaEventRecord(ev[2], stream) != cudaSuccess) return SPP_ERR_CUDA;
     return r;
 }

@@ -53,7 +53,7 @@ class spp_decode_opts(C.Structure):
     _fields_ = [("out", C.c_int), ("transform", C.c_int), ("shift", C.c_void_p), ("scale", C.c_void_p),
                 ("status", C.c_void_p), ("src_bytes", C.c_void_p), ("workspace", C.c_void_p),
                 ("workspace_size", C.c_size_t), ("C", C.c_int), ("D", C.c_int), ("H", C.c_int), ("W", C.c_int),
-                ("timing_events", C.c_void_p), ("escape_keys", C.c_int)]
+                ("timing_events", C.c_void_p), ("escape_keys", C.c_int), ("raw_segments", C.c_int)]
 
 
 _lib = None

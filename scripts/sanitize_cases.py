@@ -63,6 +63,7 @@ rm1 = r.copy(); rm1[o3] = 1
 rlen = r.copy()
 seg = next(s for s, g in enumerate(fmt.deepcam_line(r, hr, l3)["segs"]) if g["kind"] == 2)
 rlen[o3 + 4 + 4 * seg: o3 + 6 + 4 * seg] = np.frombuffer(np.uint16(1152).tobytes(), np.uint8)
-print("deepcam raw segments ok", run("deepcam", [r, r], y.shape))
-print("deepcam raw segment in mode 1", run("deepcam", [r, rm1], y.shape))
-print("deepcam raw segment too long", run("deepcam", [rlen, r], y.shape, out="f32"))
+for rs in (False, True):  # general line path / one-pass instance (opts.raw_segments)
+    print("deepcam raw segments ok", rs, run("deepcam", [r, r], y.shape, raw_segments=rs))
+    print("deepcam raw segment in mode 1", rs, run("deepcam", [r, rm1], y.shape, raw_segments=rs))
+    print("deepcam raw segment too long", rs, run("deepcam", [rlen, r], y.shape, out="f32", raw_segments=rs))

@@ -44,9 +44,10 @@ def _same_bits(got: np.ndarray, want: np.ndarray):
         assert np.array_equal(got, want)
 
 
-def _decode(fmt_name, bufs, dims, out="f16", transform=None, shift=None, scale=None, escape_keys=False):
+def _decode(fmt_name, bufs, dims, out="f16", transform=None, shift=None, scale=None, escape_keys=False,
+            raw_segments=False):
     from paper_conf_ipps_ibrahimo22_b200 import Decoder
-    dec = Decoder(fmt_name, dims, out=out, transform=transform, escape_keys=escape_keys)
+    dec = Decoder(fmt_name, dims, out=out, transform=transform, escape_keys=escape_keys, raw_segments=raw_segments)
     if shift is not None or scale is not None:
         dec.set_normalisation(shift, scale)
     srcs = [_to_dev(b) for b in bufs]
@@ -379,8 +380,9 @@ def test_deepcam_raw16_streams(dev, orc, budget):
         _same_bits(got[1], want)
 
 
+@pytest.mark.parametrize("rs", [False, True])
 @pytest.mark.parametrize("budget,raw16", [(1, False), (4, True)])
-def test_deepcam_raw_segment_streams(dev, orc, budget, raw16):
+def test_deepcam_raw_segment_streams(dev, orc, budget, raw16, rs):
     """FORMAT.md 2.7 streams from the encoder (error budget + RAW segments) on
     the full C3 shape: mode-3 lines among SEG (and RAW16) lines, bit-exact."""
     from synth import deepcam_stats, gen_deepcam
@@ -391,7 +393,7 @@ def test_deepcam_raw_segment_streams(dev, orc, budget, raw16):
     h = fmt.deepcam_header(b)
     assert 3 in {fmt.deepcam_line(b, h, l)["mode"] for l in range(0, h["L"], 3)}
     for out, sh, sc in (("f16", mean, rstd), ("f32", None, None)):
-        got, st = _decode("deepcam", [b, b], x.shape, out=out, shift=sh, scale=sc)
+        got, st = _decode("deepcam", [b, b], x.shape, out=out, shift=sh, scale=sc, raw_segments=rs)
         assert st == 0
         want = _dc_ref(orc, b, x.shape, sh, sc, out)
         _same_bits(got[0], want)
@@ -473,10 +475,11 @@ def test_deepcam_handbuilt_lines(dev, orc, W):
     _same_bits(got[0], _dc_ref(orc, b, (C, H, W), None, None, "f32"))
 
 
-@pytest.mark.parametrize("W,A", [(64, 8), (37, 1), (1152, 36)])
-def test_deepcam_raw_segment_lines(dev, orc, W, A):
-    """FORMAT.md 2.7 lines (SEG with RAW segments, decoded on KD's general line
-    path) mixed with plain SEG and RAW lines: bit-exact, normalised and x-hat."""
+@pytest.mark.parametrize("W,A,rs", [(64, 8, False), (37, 1, True), (1152, 36, False), (1152, 36, True)])
+def test_deepcam_raw_segment_lines(dev, orc, W, A, rs):
+    """FORMAT.md 2.7 lines (SEG with RAW segments: KD's general line path, or
+    the one-pass path with opts.raw_segments at W = 1152) mixed with plain SEG
+    and RAW lines: bit-exact, normalised and x-hat."""
     from tests.test_oracle_pins import _raw_segment_line
     rng = np.random.default_rng(100 + W)
     C, H = 2, 12
@@ -489,7 +492,7 @@ def test_deepcam_raw_segment_lines(dev, orc, W, A):
     b = fmt.build_deepcam_stream(C, H, W, lines, A=A)
     shift, scale = np.float32([0.5, -3.0]), np.float32([2.0, 1e-3])
     for out, sh, sc in (("f16", shift, scale), ("f32", shift, scale), ("f32", None, None)):
-        got, st = _decode("deepcam", [b, b], (C, H, W), out=out, shift=sh, scale=sc)
+        got, st = _decode("deepcam", [b, b], (C, H, W), out=out, shift=sh, scale=sc, raw_segments=rs)
         assert st == 0
         want = _dc_ref(orc, b, (C, H, W), sh, sc, out)
         _same_bits(got[0], want)
@@ -618,8 +621,9 @@ def test_deepcam_c4_launch_configuration(dev, orc):
     del out, o16
 
 
-def test_deepcam_raw_segment_onepass_corruption(dev):
-    """W = 1152, A = 36 (the one-pass path): a RAW segment (kind 2) in a mode-1
+@pytest.mark.parametrize("rs", [False, True])
+def test_deepcam_raw_segment_onepass_corruption(dev, rs):
+    """W = 1152, A = 36 (one-pass path with rs): a RAW segment (kind 2) in a mode-1
     line, and a RAW segment whose 4 len bytes run past the line, are reported
     as corrupt on the sample that holds them (FORMAT.md 2.7)."""
     W, A = 1152, 36
@@ -630,9 +634,9 @@ def test_deepcam_raw_segment_onepass_corruption(dev):
     ok = fmt.build_deepcam_stream(1, 2, W, [good, good], A=A)
     for bad in (in_mode1, too_long):
         b = fmt.build_deepcam_stream(1, 2, W, [good, bad], A=A)
-        _, st = _decode("deepcam", [ok, b], (1, 2, W), out="f16")
+        _, st = _decode("deepcam", [ok, b], (1, 2, W), out="f16", raw_segments=rs)
         assert st == (3 | (1 << 8))
-    got, st = _decode("deepcam", [ok], (1, 2, W), out="f32")
+    got, st = _decode("deepcam", [ok], (1, 2, W), out="f32", raw_segments=rs)
     assert st == 0
     want = np.concatenate([v, np.ones(W - A, np.float32)])
     _same_bits(got[0, 0, 0], want)
