@@ -149,6 +149,12 @@ def test_decode_argument_validation_without_gpu(spp):
     bad = spp.spp_decode_opts_init("cosmo", 3, 8, 8, 8)
     assert lib.spp_decode_batch(1, 16, 1, 256, ctypes.byref(bad), None) == spp.SPP_ERR_INVALID_ARG
     o = spp.spp_decode_opts_init("deepcam", 16, 1, 768, 1152)
+    assert o.raw_segments == 0                                                         # default instance
+    o.raw_segments = 2                                                                 # only 0 / 1
+    assert lib.spp_decode_batch(2, 16, 1, 256, ctypes.byref(o), None) == spp.SPP_ERR_INVALID_ARG
+    o.raw_segments = 1
+    assert lib.spp_decode_batch(2, 16, 1, 256, ctypes.byref(o), None) == spp.SPP_ERR_BUFFER_TOO_SMALL  # no ws
+    o.raw_segments = 0
     assert lib.spp_decode_batch(2, 16, 1, 256, ctypes.byref(o), None) == spp.SPP_ERR_BUFFER_TOO_SMALL  # no ws
     assert spp.spp_decode_workspace_size("deepcam", 4, o) > 0
     assert spp.spp_decoded_sample_bytes("deepcam", o) == 16 * 768 * 1152 * 2
