@@ -178,9 +178,9 @@ typedef struct {
                                 take the scalar kernel decode them either way). */
     int raw_segments;        /* DeepCAM: 1 = the batch may hold FORMAT.md 2.7 mode-3 lines
                                 (spp_encode_deepcam_ex raw_segments = 1): W = 1152 batches use the
-                                KD instance that decodes them in one warp pass.  0 (default): the
-                                mode-1 instance, on which mode-3 lines take the general line path
-                                (same bits, slower).  Other values -> SPP_ERR_INVALID_ARG. */
+                                KD instance that decodes them (and FORMAT.md 2.6 RAW16 lines) in one
+                                warp pass.  0 (default): the mode-1 instance, on which those lines
+                                take the general line path (same bits, slower).  Other values -> SPP_ERR_INVALID_ARG. */
 } spp_decode_opts;
 
 /* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */

@@ -730,6 +730,37 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
 }
 
 // mode-3 lines out of line: the mode-1 loop keeps its code footprint
+// One-pass RAW16 line (FORMAT.md 2.6) of W = 32*36 values, on the instance
+// opts.raw_segments selects: lane l widens its 36 binary16 values (72 B at
+// 16 + 72 l, 8-B aligned) exactly, y = RN(RN(x - shift) * scale), and the row
+// leaves like a one-pass SEG row (staged in the slot, one TMA bulk store).
+template <int OUT>
+__device__ __forceinline__ bool decode_line_raw16_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, float shv,
+                                                          float scv, uint8_t *row, int lane) {
+    constexpr int VPL = 36;
+    if (16u + 2u * W > bytes) return false;
+    const uint32_t src = smem_u32(buf + 16) + 2u * VPL * (uint32_t)lane;
+    uint32_t w[VPL / 2];
+#pragma unroll
+    for (int k = 0; k < VPL / 4; k++) {
+        const uint2 v = lds_u2(src + 8u * k);
+        w[2 * k] = v.x;
+        w[2 * k + 1] = v.y;
+    }
+    float y[VPL];
+#pragma unroll
+    for (int j = 0; j < VPL; j++) {
+        const float xv = __half2float(__ushort_as_half((unsigned short)((w[j >> 1] >> (16 * (j & 1))) & 0xFFFFu)));
+        y[j] = __fmul_rn(__fsub_rn(xv, shv), scv);
+    }
+    __syncwarp();  // every lane has read its values: reuse the slot for the row
+    stage_vpl<OUT, VPL>(smem_u32(buf) + VPL * (uint32_t)lane * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+    return true;
+}
+
 template <int OUT, bool VEC, int VPL>
 __global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decode(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
@@ -1070,7 +1101,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
             uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (RAWSEG && buf[0] == kModeSegRaw))) {
+            if (RAWSEG && buf[0] == kModeRaw16) {
+                if constexpr (RAWSEG && VPL == 36) ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, lane);
+            } else if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (RAWSEG && buf[0] == kModeSegRaw))) {
                 if constexpr (VPL == 36) {
                     if (!RAWSEG || buf[0] == kModeSeg)
                         ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);

@@ -28,13 +28,15 @@ def main():
     B = 256
     rows = []
     for name, kw in (("default", {}), ("budget1", dict(err_budget=1)), ("budget1_raw16", dict(err_budget=1, raw16=True)),
+                     ("budget1_raw16_onepass", dict(err_budget=1, raw16=True, _onepass=True)),
                      ("budget1_rawseg", dict(err_budget=1, raw_segments=True)),
                      ("budget16_rawseg", dict(err_budget=16, raw_segments=True)),
                      ("budget1_rawseg_general", dict(err_budget=1, raw_segments=True, _general=True))):
         kw = dict(kw)
         general = kw.pop("_general", False)  # mode-3 lines on the general line path (opts.raw_segments = 0)
+        onepass = kw.pop("_onepass", False)  # RAW16 lines on the opts.raw_segments instance
         bufs = [spp.spp_encode_deepcam(x, **kw) for x in xs]
-        dec = Decoder("deepcam", xs[0].shape, raw_segments=bool(kw.get("raw_segments")) and not general)
+        dec = Decoder("deepcam", xs[0].shape, raw_segments=(bool(kw.get("raw_segments")) and not general) or onepass)
         dec.set_normalisation(mean, rstd)
         out = dec.alloc_out(B)
         src = [torch.from_numpy(bufs[i % 2]).cuda() for i in range(B)]

@@ -622,6 +622,37 @@ def test_deepcam_c4_launch_configuration(dev, orc):
 
 
 @pytest.mark.parametrize("rs", [False, True])
+def test_deepcam_raw16_lines_w1152(dev, orc, rs):
+    """FORMAT.md 2.6 RAW16 lines at W = 1152 among SEG lines (one-pass instance
+    with rs, else the general line path): bit-exact, normalised and x-hat; a
+    RAW16 line shorter than 16 + 2 W bytes is reported."""
+    W, C, H = 1152, 2, 6
+    rng = np.random.default_rng(7)
+    h16 = rng.integers(0, 1 << 16, size=(C * H, W), dtype=np.uint16)
+    h16[:, ::5] = 0x7C00 | (h16[:, ::5] & 0x8000)          # infinities
+    h16[:, 1::7] &= 0x83FF                                  # subnormals and zeros
+    h16[(h16 & 0x7C00) == 0x7C00] &= 0xFC00                 # no NaN patterns (the encoder never writes them)
+    lines = []
+    for l in range(C * H):
+        if l % 3 == 1:
+            lines.append(fmt.build_seg_line(W, [(W, 1, 140, 1.0)], [1] * (W - 1)))
+        else:
+            lines.append(bytes([2]) + b"\0" * 15 + h16[l].astype("<u2").tobytes())
+    b = fmt.build_deepcam_stream(C, H, W, lines, A=36)
+    shift, scale = np.float32([0.5, -3.0]), np.float32([2.0, 1e-3])
+    for out, sh, sc in (("f16", shift, scale), ("f32", shift, scale), ("f32", None, None)):
+        got, st = _decode("deepcam", [b, b], (C, H, W), out=out, shift=sh, scale=sc, raw_segments=rs)
+        assert st == 0
+        want = _dc_ref(orc, b, (C, H, W), sh, sc, out)
+        _same_bits(got[0], want)
+        _same_bits(got[1], want)
+    short = bytes([2]) + b"\0" * 15 + b"\0" * (2 * W - 16)
+    bad = fmt.build_deepcam_stream(C, H, W, lines[:-1] + [short], A=36)
+    _, st = _decode("deepcam", [b, bad], (C, H, W), out="f16", raw_segments=rs)
+    assert st == (3 | (1 << 8))
+
+
+@pytest.mark.parametrize("rs", [False, True])
 def test_deepcam_raw_segment_onepass_corruption(dev, rs):
     """W = 1152, A = 36 (one-pass path with rs): a RAW segment (kind 2) in a mode-1
     line, and a RAW segment whose 4 len bytes run past the line, are reported
