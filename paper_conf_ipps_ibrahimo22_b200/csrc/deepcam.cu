@@ -31,10 +31,11 @@
 //                    (line record by st.async + bytes by TMA) into a 3-slot
 //                    ring; W = 1152 lines with 36-aligned segments decode in
 //                    one warp pass (decode_line_onepass) and leave as one TMA
-//                    bulk store of the staged row; RAW segments of mode-3
-//                    lines (FORMAT.md 2.7) are read there by their lanes.
-//                    RAW and RAW16 lines (FORMAT.md 2.6) take the general
-//                    line path.
+//                    bulk store of the staged row.  The instance selected
+//                    by opts.raw_segments also takes mode-3 lines (FORMAT.md
+//                    2.7: RAW-segment lanes read their stored values) and
+//                    RAW16 lines (2.6) in one pass; otherwise those, and RAW
+//                    lines, take the general line path.
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
