@@ -224,6 +224,9 @@ spp_status spp_pipeline_create(spp_pipeline **out, spp_format fmt, const spp_dec
 void spp_pipeline_destroy(spp_pipeline *p);
 
 /* Decode n host-resident samples into d_dst (layout as spp_decode_batch).
+ * Calls on one pipeline are ordered: each call's first decode waits (on the
+ * device) for the previous call's last decode, whatever streams they used, since
+ * they share the pipeline's workspace and staging ring.
  *   h_src     : HOST array of n HOST pointers (pinned for async copies)
  *   src_bytes : HOST array of n sizes (multiples of 16)
  *   opts      : as spp_decode_batch; opts->workspace/src_bytes are ignored
@@ -238,13 +241,6 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
 
 /* Number of decode launches and copies the last spp_decode_host call enqueued. */
 int spp_pipeline_last_launches(const spp_pipeline *p);
-
-/* Optional performance hint (device-wide, opt-in): reserve `bytes` of L2 as the
- * persisting set-aside (cudaLimitPersistingL2CacheSize) so that the CosmoFlow
- * LUT rows, which the decoder reads with an L2 evict-last policy, survive the
- * output stream.  0 releases the set-aside.  Affects the whole current device;
- * the granted size is returned in *granted (may be clamped by the driver). */
-spp_status spp_set_l2_persisting(size_t bytes, size_t *granted);
 
 const char *spp_status_string(spp_status s);
 

@@ -53,17 +53,22 @@ class Decoder:
         self._ws_n = 0
         self.shift = None
         self.scale = None
+        # bumped whenever a device buffer a captured decode refers to is replaced
+        # (workspace, shift/scale): CUDA graphs captured earlier must be dropped
+        self.version = 0
 
     def set_normalisation(self, shift, scale):
         """DeepCAM per-channel (shift, scale) as device fp32 tensors [C] (or None)."""
         t = self.torch
         self.shift = None if shift is None else t.as_tensor(shift, dtype=t.float32, device=self.device).contiguous()
         self.scale = None if scale is None else t.as_tensor(scale, dtype=t.float32, device=self.device).contiguous()
+        self.version += 1
 
     def workspace(self, n: int):
         need = spp.spp_decode_workspace_size(self.fmt, n, self.opts)
         if self._ws is None or self._ws.numel() < need:
             self._ws = self.torch.empty(max(need, 256), dtype=self.torch.uint8, device=self.device)
+            self.version += 1
         return self._ws, need
 
     def alloc_out(self, n: int):

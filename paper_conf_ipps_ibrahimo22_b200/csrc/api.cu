@@ -14,13 +14,17 @@ namespace spp {
 
 spp_status current_device_props(DeviceProps *out) {
     static std::mutex mu;
-    static DeviceProps cache[64];
-    static bool have[64] = {false};
+    static DeviceProps cache[kMaxDevices];
+    static bool have[kMaxDevices] = {false};
     int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return SPP_ERR_CUDA;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return SPP_ERR_CUDA;
     std::lock_guard<std::mutex> lock(mu);
     if (!have[dev]) {
         DeviceProps p;
+        p.dev = dev;
+        if (cudaDeviceGetAttribute(&p.smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev) != cudaSuccess ||
+            cudaDeviceGetAttribute(&p.smem_reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev) != cudaSuccess)
+            return SPP_ERR_CUDA;
         if (cudaDeviceGetAttribute(&p.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return SPP_ERR_CUDA;
         if (cudaDeviceGetAttribute(&p.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess)
             return SPP_ERR_CUDA;
@@ -110,7 +114,7 @@ spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, in
         if (r32(0) != kCosmoMagic || r16(4) != kVersion) return SPP_ERR_CORRUPT;
         const uint32_t nU = r32(cosmo::kNU), T = r32(cosmo::kNSlab);
         const uint64_t slab_off = r64(cosmo::kSlabOff);
-        if (T < 1 || slab_off + 32ull * T > src_bytes) return SPP_ERR_CORRUPT;
+        if (T < 1 || slab_off > src_bytes || 32ull * T > src_bytes - slab_off) return SPP_ERR_CORRUPT;
         info[0] = nU;
         info[1] = T;
         info[2] = r32(slab_off + 8);
@@ -121,11 +125,11 @@ spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, in
         if (r32(0) != kDeepcamMagic || r16(4) != kVersion) return SPP_ERR_CORRUPT;
         const uint32_t L = r32(deepcam::kL);
         const uint64_t dir_off = r64(deepcam::kDirOff), pay = r64(deepcam::kPayloadOff);
-        if (dir_off + 4ull * (L + 1) > src_bytes) return SPP_ERR_CORRUPT;
+        if (dir_off > src_bytes || 4ull * (L + 1) > src_bytes - dir_off || pay > src_bytes) return SPP_ERR_CORRUPT;
         int64_t raw = 0, seg = 0, segs = 0, dbytes = 0;
         for (uint32_t l = 0; l < L; l++) {
             const uint64_t a = r32(dir_off + 4ull * l), e = r32(dir_off + 4ull * l + 4);
-            if (pay + e > src_bytes || e < a + 16) return SPP_ERR_CORRUPT;
+            if (e > src_bytes - pay || e < a + 16) return SPP_ERR_CORRUPT;
             const uint8_t *p = b + pay + a;
             if (p[0] == deepcam::kModeRaw || p[0] == deepcam::kModeRaw16) { raw++; continue; }
             seg++;
@@ -146,18 +150,6 @@ spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, in
         return SPP_OK;
     }
     return SPP_ERR_INVALID_ARG;
-}
-
-spp_status spp_set_l2_persisting(size_t bytes, size_t *granted) {
-    int dev = 0, maxp = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess) return SPP_ERR_CUDA;
-    if (cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess) return SPP_ERR_CUDA;
-    const size_t want = bytes < (size_t)maxp ? bytes : (size_t)maxp;
-    if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) != cudaSuccess) return SPP_ERR_CUDA;
-    size_t got = 0;
-    if (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) != cudaSuccess) return SPP_ERR_CUDA;
-    if (granted) *granted = got;
-    return SPP_OK;
 }
 
 const char *spp_status_string(spp_status s) {

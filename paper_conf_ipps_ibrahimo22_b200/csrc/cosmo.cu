@@ -138,8 +138,11 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
             T = ld_le32(b + kNSlab);
             U_off = ld_le64(b + kUOff);
             const uint64_t slab_off = ld_le64(b + kSlabOff), total = ld_le64(b + kTotal);
+            // every range checked as off <= total && len <= total - off: stream-supplied
+            // 64-bit offsets never wrap an addition
+            auto in_range = [&](uint64_t off, uint64_t len) { return off <= total && len <= total - off; };
             ok = total <= limit && nU >= 1 && nU <= (uint32_t)kMaxU && T >= 1 && T <= (uint32_t)D &&
-                 U_off + 2ull * nU <= total && slab_off + (uint64_t)kSlabBytes * T <= total &&
+                 in_range(U_off, 2ull * nU) && in_range(slab_off, (uint64_t)kSlabBytes * T) &&
                  (slab_off & 15) == 0 && (U_off & 1) == 0;
             const uint64_t plane = (uint64_t)H * W;
             uint32_t zexp = 0;
@@ -159,14 +162,15 @@ __global__ void __launch_bounds__(kPrologueThreads) kc0_prologue(const void *con
                 }
                 else if (kw == kRawSlab) ok = ok && G == 0;
                 else ok = 0;
-                if (kw != kRawSlab) ok = ok && (lut_off & 15) == 0 && lut_off + 8ull * G <= total;
+                if (kw != kRawSlab) ok = ok && (lut_off & 15) == 0 && in_range(lut_off, 8ull * G);
                 if (kw == kEscaped) {  // FORMAT.md 1.5: eidx[0] = 0, the escape list inside the stream
                     const uint64_t nb = (Nt + kEscBlock - 1) / kEscBlock;
-                    const uint64_t esc_off = keys_off + ((4 * (nb + 1) + 15) & ~15ull) + ((Nt + 15) & ~15ull);
-                    ok = ok && (keys_off & 15) == 0 && esc_off <= total && ld_le32(b + keys_off) == 0 &&
-                         esc_off + 2ull * ld_le32(b + keys_off + 4 * nb) <= total;
+                    const uint64_t head = ((4 * (nb + 1) + 15) & ~15ull) + ((Nt + 15) & ~15ull);
+                    ok = ok && (keys_off & 15) == 0 && in_range(keys_off, head);
+                    const uint64_t esc_off = ok ? keys_off + head : 0;
+                    ok = ok && ld_le32(b + keys_off) == 0 && in_range(esc_off, 2ull * ld_le32(b + keys_off + 4 * nb));
                 } else if (kw != 0) {
-                    ok = ok && (keys_off & 15) == 0 && keys_off + (uint64_t)(kw == kRawSlab ? 8 : kw) * Nt <= total;
+                    ok = ok && (keys_off & 15) == 0 && in_range(keys_off, (uint64_t)(kw == kRawSlab ? 8 : kw) * Nt);
                 }
                 zexp = z1;
             }
@@ -971,13 +975,7 @@ spp_status launch_expand(const void *const *d_src, int n, const float *fU, const
     auto kern = kc_expand<OUT, VEC, ESC>;
     const int entry_bytes = OUT == SPP_OUT_F32 ? 16 : 8;
     const int smem = kSmemBytes;
-    static int attr_done[16] = {0};  // per template instance (device-agnostic attribute)
-    const int key = ((OUT - 1) * 2 + (VEC ? 1 : 0)) * 2 + (ESC ? 1 : 0);
-    if (!attr_done[key]) {
-        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
-            return SPP_ERR_CUDA;
-        attr_done[key] = 1;
-    }
+    if (set_smem_attr<kc_expand<OUT, VEC, ESC>>(smem, dp) != SPP_OK) return SPP_ERR_CUDA;  // per device
     int occ = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, smem) != cudaSuccess || occ < 1)
         return SPP_ERR_CUDA;

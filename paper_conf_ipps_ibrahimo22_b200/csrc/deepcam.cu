@@ -8,34 +8,29 @@
 // loop-carried dependency is handled with hierarchical parallelism — here one
 // warp per line, lanes cooperating on the inner loop.
 //
-//   KD0  kd0_parse   one thread per sample: validate header, publish the line
-//                    directory / payload pointers.
-//   KD   kd_decode   persistent warps, each over a contiguous range of lines.
-//                    Lane 0 prefetches the directory two lines ahead and
-//                    issues a 1-D TMA bulk copy (cp.async.bulk + mbarrier) of
-//                    the next line into the warp's second smem buffer while
-//                    the warp decodes the current one (double buffering).
-//                    Decode of a SEG line:
-//                      1. warp scans of segment lengths / delta-byte counts ->
-//                         start bitmap + per-segment byte base (in place);
-//                      2. per 256-position chunk, lane l owns positions
-//                         [8l, 8l+8): 8 delta bytes -> 8 exact codes (as fp32
-//                         multiples of 2^-130: every partial sum is exact),
-//                         lane-serial prefix, warp segmented scan (reset at
-//                         segment heads) -> S_j, x̂ = fma(S_j, 2^emin, h)
-//                         (one rounding; FORMAT.md 2.3 reading S13);
-//                      3. y = (x̂ - shift) * scale (two roundings), RNE to fp16,
-//                         one 16-B streaming store per lane (512 B per warp).
-//   KD   kd_decode_ws  (the default) the same decode, warp-specialised: one
-//                    producer warp per CTA streams each consumer warp's lines
-//                    (line record by st.async + bytes by TMA) into a 3-slot
-//                    ring; W = 1152 lines with 36-aligned segments decode in
-//                    one warp pass (decode_line_onepass) and leave as one TMA
-//                    bulk store of the staged row.  The instance selected
-//                    by opts.raw_segments also takes mode-3 lines (FORMAT.md
-//                    2.7: RAW-segment lanes read their stored values) and
-//                    RAW16 lines (2.6) in one pass; otherwise those, and RAW
-//                    lines, take the general line path.
+//   KD0  kd0_parse     one thread per sample: validate header, publish the line
+//                      directory / payload pointers.
+//   KD   kd_decode_ws  persistent, warp-specialised: one producer warp per CTA
+//                      streams each consumer warp's lines (line record by
+//                      st.async + bytes by 1-D TMA) into a 3-slot ring in shared
+//                      memory; each consumer warp decodes one line at a time.
+//                      Line paths (all bit-identical, FORMAT.md 2.3):
+//                      * one pass (W = 1152, A = 36, <= 32 segments): lane l owns
+//                        positions [36l, 36l+36), codes -> exact fp16 pairs, two
+//                        exact fp32 prefix chains, one warp scan; the row is
+//                        staged in a per-warp row buffer and leaves by one TMA
+//                        bulk store (decode_line_onepass);
+//                      * aligned (A = positions per lane): block bitmap + scans
+//                        (decode_line_aligned);
+//                      * general (any A, RAW / RAW16 / mode-3 lines): start bitmap,
+//                        prefix counts, segmented warp scan (decode_line);
+//                      * global (a line longer than the ring, or W too large for
+//                        the shared tables): decoded straight from HBM, segment
+//                        by segment, with an exact int32 prefix scan
+//                        (decode_line_global).  Every FORMAT-legal line decodes.
+//                      The instance selected by opts.raw_segments also takes
+//                      mode-3 lines (FORMAT.md 2.7) and RAW16 lines (2.6) in one
+//                      pass.
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -59,11 +54,9 @@ struct DcMeta {  // written by KD0, read by KD (32 B)
     uint32_t align;  // declared segment alignment A (FORMAT.md 2.1)
 };
 
-constexpr int kMaxWarpsPerCta = 8;
-#ifndef SPP_KD_MINB
-#define SPP_KD_MINB 3  // CTAs per SM the register allocation targets (3 x 8 warps: 80 registers, no spills)
-#endif
-constexpr int kMaxW = 16383;  // GPU path: per-segment byte base packed in 16 bits
+// Lines of W > kSmemMaxW take the global path (the shared start-bitmap / prefix
+// tables of the general path are sized by W); FORMAT.md allows W <= 65535.
+constexpr uint32_t kSmemMaxW = 8192;
 
 __global__ void kd0_parse(const void *const *__restrict__ src, const uint64_t *__restrict__ src_bytes, int n, int C,
                           int H, int W, DcMeta *__restrict__ meta, uint32_t *__restrict__ status) {
@@ -79,8 +72,10 @@ __global__ void kd0_parse(const void *const *__restrict__ src, const uint64_t *_
              ld_le16(b + kH) == H && ld_le16(b + kW) == W && ld_le32(b + kL) == L;
         const uint64_t dir_off = ld_le64(b + kDirOff), pay = ld_le64(b + kPayloadOff), total = ld_le64(b + kTotal);
         const uint32_t A = ld_le16(b + kAlign);
-        ok = ok && total <= limit && (dir_off & 3) == 0 && dir_off + 4 * (L + 1) <= total && (pay & 15) == 0 &&
-             pay <= total && A >= 1 && (uint32_t)W % A == 0;
+        // every range as off <= total && len <= total - off: stream-supplied 64-bit
+        // offsets never wrap an addition
+        ok = ok && total <= limit && (dir_off & 3) == 0 && dir_off <= total && 4 * (L + 1) <= total - dir_off &&
+             (pay & 15) == 0 && pay <= total && A >= 1 && (uint32_t)W % A == 0;
         if (ok) m = DcMeta{b + dir_off, b + pay, total - pay, 1u, A};
     }
     if (!ok) report(status, SPP_ERR_CORRUPT, s);
@@ -130,8 +125,13 @@ __device__ __forceinline__ float code_f_byte(uint32_t b) {
 }
 
 // per-segment packed info written in place of the descriptor:
-//   bits 0..15  byte base a + 16384 (delta byte of position p is dl[a + p])
-//   bits 16..23 kind, bits 24..31 emin_b
+//   bits 0..21  byte base a + 2^21 (DIFF: the delta byte of position p is dl[a + p];
+//               RAW segment: its value is the binary32 at dl + a + 4p), any W <= 65535
+//   bits 22..23 kind (validated <= 2 before packing), bits 24..31 emin_b
+constexpr int kBaseBias = 1 << 21;
+__device__ __forceinline__ uint32_t pack_seg(int a, uint32_t kind, uint32_t eb) {
+    return ((uint32_t)(a + kBaseBias) & 0x3FFFFFu) | ((kind & 3u) << 22) | (eb << 24);
+}
 struct SegInfo {
     float h;
     float sc;      // 2^(emin+130) (emin <= -3) or 2^(emin+30) (big)
@@ -143,8 +143,8 @@ __device__ __forceinline__ SegInfo seg_info(const uint32_t *desc, const float *h
     const uint32_t d = desc[s];
     SegInfo si;
     si.h = heads[s];
-    si.a = (int)(d & 0xFFFFu) - 16384;
-    si.kind = (d >> 16) & 0xFFu;
+    si.a = (int)(d & 0x3FFFFFu) - kBaseBias;
+    si.kind = (d >> 22) & 3u;
     const uint32_t eb = d >> 24;
     si.big = eb >= 148u;
     si.sc = __uint_as_float((si.big ? (eb + 7u) : (eb + 107u)) << 23);
@@ -272,7 +272,7 @@ __device__ __forceinline__ bool decode_line(uint8_t *buf, uint32_t bytes, uint32
             if (st < W) atomicOr(&sbits[st >> 5], 1u << (st & 31));
             // DIFF: the code of position p is byte a + p; RAW: its value is at bytes a + 4p
             const int a = kind == kRawSeg ? (int)db - 4 * (int)st : (int)db - (int)st - 1;
-            desc[s] = (uint32_t)(a + 16384) | (kind << 16) | (eb << 24);
+            desc[s] = pack_seg(a, kind, eb);
         }
         cl += __shfl_sync(0xffffffffu, il, 31);
         cd += __shfl_sync(0xffffffffu, id, 31);
@@ -471,10 +471,27 @@ __device__ __forceinline__ void stage_vpl(uint32_t sdst, const float (&y)[VPL]) 
     }
 }
 
+// The one-pass instances stage each output row in a per-warp row buffer (not
+// in the line's input slot, which the producer refills by TMA): acquire waits
+// until the previous row's bulk store has finished reading the buffer, release
+// hands the staged row to the TMA engine.  The input slot is only ever read by
+// the consumer's generic loads, so its release/refill needs no proxy fence.
+__device__ __forceinline__ void row_buffer_acquire(int lane) {
+    if (lane == 0) bulk_wait_read_all();
+    __syncwarp();
+}
+template <int OUT>
+__device__ __forceinline__ void row_buffer_release(uint8_t *row, uint8_t *rowbuf, uint32_t W, int lane) {
+    fence_proxy_async_smem();  // this lane's row writes -> visible to the async proxy
+    __syncwarp();
+    if (lane == 0) bulk_s2g(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+}
+
 template <int OUT, int VPL>
 __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
-                                                    uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
-    constexpr bool STAGED = VPL == 36;  // one pass per line (W = 32 * VPL), TMA bulk store of the row
+                                                    uint32_t nbw, float shv, float scv, uint8_t *row, uint8_t *rowbuf,
+                                                    int lane) {
+    constexpr bool STAGED = VPL == 36;  // one pass per line (W = 32 * VPL): row staged in rowbuf, one TMA bulk store
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
     if (nseg < 1 || nseg > W || 4u + 8u * nseg > bytes) return false;
@@ -507,7 +524,7 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             bad |= len == 0 || kind > kDiff || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
                    st + len > W || blk * VPL != st;
             if (st < W) atomicOr(&bbits[blk >> 5], 1u << (blk & 31));
-            desc[s] = (uint32_t)((int)db - (int)st - 1 + 16384) | (kind << 16) | (eb << 24);
+            desc[s] = pack_seg((int)db - (int)st - 1, kind, eb);
         }
         cacc += __shfl_sync(0xffffffffu, inc, 31);
     }
@@ -598,17 +615,13 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             }
         }
         if constexpr (STAGED) {
-            __syncwarp();  // every lane has read its delta bytes and segment: reuse the slot for the row
-            stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+            row_buffer_acquire(lane);
+            stage_vpl<OUT, VPL>(smem_u32(rowbuf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
         } else {
             emit_vpl<OUT, VPL>(row, p0, y);
         }
     }
-    if constexpr (STAGED) {
-        fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
-        __syncwarp();
-        if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
-    }
+    if constexpr (STAGED) row_buffer_release<OUT>(row, rowbuf, W, lane);
     return true;
 }
 
@@ -618,14 +631,16 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
 // parameters by shuffle.  Falls back to the shared-memory tables otherwise.
 template <int OUT, bool RAWSEG>  // RAWSEG: a mode-3 line (FORMAT.md 2.7); mode-1 lines run without its code
 __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
-                                                    uint32_t nbw, float shv, float scv, uint8_t *row, int lane) {
+                                                    uint32_t nbw, float shv, float scv, uint8_t *row, uint8_t *rowbuf,
+                                                    int lane) {
     constexpr int VPL = 36;
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
     // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
     // it never has more than 32 segments, so the fallback sees only mode 1
     constexpr uint32_t max_kind = RAWSEG ? kRawSeg : kDiff;
-    if (nseg > (uint32_t)kWarp) return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, lane);
+    if (nseg > (uint32_t)kWarp)
+        return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, rowbuf, lane);
     if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
     const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
     const bool have = (uint32_t)lane < nseg;
@@ -652,7 +667,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const uint32_t word = __reduce_or_sync(0xffffffffu, have ? 1u << blk : 0u);  // head lanes
     // DIFF: the code of position p is delta byte a + p; RAW: its value is at bytes a + 4p
     const int a_s = kind == kRawSeg ? (int)db - 4 * (int)st : (int)db - (int)st - 1;
-    const uint32_t info = (uint32_t)(a_s + 16384) | (kind << 16) | (eb << 24);
+    const uint32_t info = pack_seg(a_s, kind, eb);
 
     const uint32_t le_mask = 0xFFFFFFFFu >> (31 - lane);
     const uint32_t p0 = VPL * lane;
@@ -660,8 +675,8 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const int s = __popc(word & le_mask) - 1;  // segment of this lane (position 0 is always a head)
     const uint32_t d = __shfl_sync(0xffffffffu, info, s);
     const float h = __shfl_sync(0xffffffffu, hs, s);
-    const int a = (int)(d & 0xFFFFu) - 16384;
-    const uint32_t skind = (d >> 16) & 0xFFu, seb = d >> 24;
+    const int a = (int)(d & 0x3FFFFFu) - kBaseBias;
+    const uint32_t skind = (d >> 22) & 3u, seb = d >> 24;
     const bool raw = RAWSEG && skind == kRawSeg;
     const bool rep = skind == kRepeat || raw;  // RAW lanes run the chain on zero codes, then take their values
     Bytes<VPL> bt;
@@ -722,11 +737,9 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
 #pragma unroll
         for (int i = 0; i < VPL; i++) y[i] = __fmul_rn(__fadd_rn(lds_f32_any(va + 4u * i), -shv), scv);
     }
-    __syncwarp();  // every lane has read its delta bytes: reuse the slot for the row
-    stage_vpl<OUT, VPL>(smem_u32(buf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
-    fence_proxy_async_smem();  // make this lane's row writes visible to the TMA engine
-    __syncwarp();
-    if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+    row_buffer_acquire(lane);
+    stage_vpl<OUT, VPL>(smem_u32(rowbuf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+    row_buffer_release<OUT>(row, rowbuf, W, lane);
     return true;
 }
 
@@ -737,7 +750,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
 // leaves like a one-pass SEG row (staged in the slot, one TMA bulk store).
 template <int OUT>
 __device__ __forceinline__ bool decode_line_raw16_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, float shv,
-                                                          float scv, uint8_t *row, int lane) {
+                                                          float scv, uint8_t *row, uint8_t *rowbuf, int lane) {
     constexpr int VPL = 36;
     if (16u + 2u * W > bytes) return false;
     const uint32_t src = smem_u32(buf + 16) + 2u * VPL * (uint32_t)lane;
@@ -754,174 +767,133 @@ __device__ __forceinline__ bool decode_line_raw16_onepass(uint8_t *buf, uint32_t
         const float xv = __half2float(__ushort_as_half((unsigned short)((w[j >> 1] >> (16 * (j & 1))) & 0xFFFFu)));
         y[j] = __fmul_rn(__fsub_rn(xv, shv), scv);
     }
-    __syncwarp();  // every lane has read its values: reuse the slot for the row
-    stage_vpl<OUT, VPL>(smem_u32(buf) + VPL * (uint32_t)lane * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
-    fence_proxy_async_smem();
-    __syncwarp();
-    if (lane == 0) bulk_s2g(row, buf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+    row_buffer_acquire(lane);
+    stage_vpl<OUT, VPL>(smem_u32(rowbuf) + VPL * (uint32_t)lane * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+    row_buffer_release<OUT>(row, rowbuf, W, lane);
     return true;
 }
 
-template <int OUT, bool VEC, int VPL>
-__global__ void __launch_bounds__(kMaxWarpsPerCta * kWarp, SPP_KD_MINB) kd_decode(
-    const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
-    const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
-    uint32_t *__restrict__ status) {
-    extern __shared__ __align__(16) uint8_t smem_raw[];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int wpc = blockDim.x >> 5;
-    uint8_t *base = smem_raw + (size_t)warp * warp_bytes;
-    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + 2 * cap);  // also the aligned path's block bitmap
-    uint32_t *wpre = sbits + nwords;
-    uint64_t *mbar = reinterpret_cast<uint64_t *>(base + 2 * cap + 8 * nwords);
-    const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
-    const uint32_t cap_data = cap - 16;       // one slot; the last 16 B are read slack
-    const uint32_t big_cap = 2 * cap - 16;    // both slots (any legal SEG line fits, FORMAT.md 2.1)
-    const uint32_t nbw = (W / VPL + 31) / 32;
-
-    const uint64_t T = (uint64_t)n * L;
-    const uint64_t NW = (uint64_t)gridDim.x * wpc;
-    const uint64_t gw = (uint64_t)blockIdx.x * wpc + warp;
-    const uint64_t g_begin = gw * T / NW, g_end = (gw + 1) * T / NW;
-    if (g_begin >= g_end) return;
-
-    if (lane == 0) {
-        mbar_init(&mbar[0], 1);
-        mbar_init(&mbar[1], 1);
-        fence_mbar_init();
+// ---------------------------------------------------------------------------
+// Global-memory line path: any FORMAT-legal line the shared-memory ring cannot
+// hold (a SEG line longer than the ring, e.g. W = 1152 at A = 1 with ~1,150
+// segments, or a mode-3 line with many short RAW segments) and every line of a
+// sample whose W exceeds kSmemMaxW.  The warp walks the segments in order
+// (32 descriptors per step: scans of len / delta-byte counts, validated before
+// any byte of those segments is read) and decodes each segment with all lanes:
+// REPEAT broadcasts the head, a RAW segment copies its binary32 values, a DIFF
+// segment takes an exact int32 inclusive scan of its codes (S_j, |S_j| < 2^24 in
+// a valid stream, FORMAT.md 2.3) and x̂ = RN(h + S_j * 2^emin) as one fma of exact
+// operands (reading S13).  Rows are written with per-lane scalar stores (rare
+// path: correctness, not bandwidth).  Out of line so the hot loop keeps its
+// registers.
+__device__ __forceinline__ int code_int(uint32_t b) {  // FORMAT.md 2.2
+    const int E = (b >> 4) & 7, M = b & 15;
+    const int mag = E == 0 ? M : (16 + M) << (E - 1);
+    return (b & 0x80u) ? -mag : mag;
+}
+__device__ __forceinline__ float pow2_emin(uint32_t eb) {  // 2^(eb - 150), eb in [1, 246]: exact
+    const int e = (int)eb - 150;
+    return e >= -126 ? __uint_as_float((uint32_t)(e + 127) << 23) : __uint_as_float(1u << (e + 149));
+}
+__device__ __forceinline__ uint32_t ldg_u8(const uint8_t *p) {
+    uint32_t v;
+    asm volatile("ld.global.nc.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+template <int OUT>
+__device__ __forceinline__ void emit1(uint8_t *row, uint32_t p, float xh, float shv, float scv) {
+    const float y = __fmul_rn(__fsub_rn(xh, shv), scv);
+    if constexpr (OUT == SPP_OUT_F32) reinterpret_cast<float *>(row)[p] = y;
+    else reinterpret_cast<__half *>(row)[p] = __float2half_rn(y);
+}
+template <int OUT>
+__device__ __noinline__ bool decode_line_global(const uint8_t *__restrict__ p, uint32_t bytes, uint32_t W, uint32_t A,
+                                                float shv, float scv, uint8_t *__restrict__ row, int lane) {
+    const uint32_t mode = ldg_u8(p);
+    if (mode == kModeRaw) {  // 16-B aligned line: aligned binary32 loads
+        if (16ull + 4ull * W > bytes) return false;
+        const float *x = reinterpret_cast<const float *>(p + 16);
+        for (uint32_t q = lane; q < W; q += kWarp) emit1<OUT>(row, q, __ldg(x + q), shv, scv);
+        return true;
     }
-    __syncwarp();
-
-
-    // Directory window: lane k holds the validated directory entry of line
-    // wbase + k (source pointer, bytes, flags), loaded and checked by all lanes
-    // at once every 32 lines; per line the pipeline only shuffles one entry.
-    uint64_t wbase = 0;
-    uint64_t w_src = 0;
-    uint32_t w_bytes = 0, w_flags = 0;  // flags: bit 0 big, bits 16.. alignment
-    float w_shv = 0.f, w_scv = 1.f;     // the line's channel constants (c = (g mod L) / H)
-    auto load_window = [&](uint64_t wb) {
-        wbase = wb;
-        const uint64_t g = wb + lane;
-        w_bytes = 0;
-        w_flags = 0;
-        w_src = 0;
-        if (g < g_end) {
-            const uint64_t sk = g / L;
-            const uint32_t lk = (uint32_t)(g - sk * L);
-            const uint32_t ck = lk / H;
-            w_shv = shift ? __ldg(shift + ck) : 0.f;
-            w_scv = scale ? __ldg(scale + ck) : 1.f;
-            const DcMeta m = meta[sk];
-            if (m.valid) {
-                const uint32_t *dir = reinterpret_cast<const uint32_t *>(m.dir);
-                const uint32_t da = __ldg(dir + lk), db = __ldg(dir + lk + 1);
-                const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= m.limit && db - da >= 16;
-                if (!ok) {
-                    report(status, SPP_ERR_CORRUPT, (int64_t)sk);
-                } else if (db - da > big_cap) {
-                    report(status, SPP_ERR_UNSUPPORTED, (int64_t)sk);
-                } else {
-                    w_bytes = db - da;
-                    w_src = reinterpret_cast<uint64_t>(m.payload + da);
-                    w_flags = (w_bytes > cap_data ? 1u : 0u) | (m.align << 16);
+    if (mode == kModeRaw16) {
+        if (16ull + 2ull * W > bytes) return false;
+        const __half *x = reinterpret_cast<const __half *>(p + 16);
+        for (uint32_t q = lane; q < W; q += kWarp) emit1<OUT>(row, q, __half2float(__ldg(x + q)), shv, scv);
+        return true;
+    }
+    if (mode != kModeSeg && mode != kModeSegRaw) return false;
+    const uint32_t max_kind = mode == kModeSegRaw ? kRawSeg : kDiff;
+    const uint32_t nseg = ldg_u8(p + 2) | (ldg_u8(p + 3) << 8);
+    if (nseg < 1 || nseg > W || 4ull + 8ull * nseg > bytes) return false;
+    const uint32_t *desc = reinterpret_cast<const uint32_t *>(p + 4);
+    const float *heads = reinterpret_cast<const float *>(p + 4 + 4 * nseg);
+    const uint8_t *dl = p + 4 + 8 * nseg;
+    const uint64_t dl_cap = bytes - (4ull + 8ull * nseg);  // delta area bytes available
+    uint32_t cl = 0;
+    uint64_t cd = 0;
+    for (uint32_t b0 = 0; b0 < nseg; b0 += kWarp) {
+        const uint32_t s = b0 + lane;
+        uint32_t len = 0, kind = 0, eb = 0;
+        float h = 0.f;
+        if (s < nseg) {
+            const uint32_t d = __ldg(desc + s);
+            len = d & 0xFFFFu;
+            kind = (d >> 16) & 0xFFu;
+            eb = d >> 24;
+            h = __ldg(heads + s);
+        }
+        const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : (kind == kRawSeg ? 4u * len : 0u);
+        const uint32_t il = warp_incl_scan(len, lane), id = warp_incl_scan(dlen, lane);  // < 2^18 each
+        const uint32_t st = cl + il - len;
+        const uint64_t db = cd + id - dlen;
+        const bool bad = s < nseg && (len == 0 || kind > max_kind ||
+                                      (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
+                                      (uint64_t)st + len > W || st % A != 0);
+        cl += __shfl_sync(0xffffffffu, il, 31);
+        cd += __shfl_sync(0xffffffffu, id, 31);
+        if (__any_sync(0xffffffffu, bad) || cd > dl_cap) return false;  // this step's bytes lie inside the line
+        const uint32_t cnt = min((uint32_t)kWarp, nseg - b0);
+        for (uint32_t k = 0; k < cnt; k++) {
+            const uint32_t kst = __shfl_sync(0xffffffffu, st, k), klen = __shfl_sync(0xffffffffu, len, k);
+            const uint32_t kkind = __shfl_sync(0xffffffffu, kind, k), keb = __shfl_sync(0xffffffffu, eb, k);
+            const uint64_t kdb = __shfl_sync(0xffffffffu, db, k);
+            const float kh = __shfl_sync(0xffffffffu, h, k);
+            if (kkind == kRepeat) {
+                for (uint32_t j = lane; j < klen; j += kWarp) emit1<OUT>(row, kst + j, kh, shv, scv);
+            } else if (kkind == kRawSeg) {  // FORMAT.md 2.7: the values are binary32 at the byte base
+                for (uint32_t j = lane; j < klen; j += kWarp) {
+                    const uint8_t *v = dl + kdb + 4ull * j;
+                    const uint32_t bits = ldg_u8(v) | (ldg_u8(v + 1) << 8) | (ldg_u8(v + 2) << 16) | (ldg_u8(v + 3) << 24);
+                    emit1<OUT>(row, kst + j, __uint_as_float(bits), shv, scv);
+                }
+            } else {  // DIFF: S_j = code(d_0) + ... + code(d_{j-1}) for the position j of the segment
+                const float unit = pow2_emin(keb);
+                int carry = 0;
+                for (uint32_t j0 = 0; j0 < klen; j0 += kWarp) {
+                    const uint32_t j = j0 + lane;
+                    const int c = (j >= 1 && j < klen) ? code_int(ldg_u8(dl + kdb + (j - 1))) : 0;
+                    const int S = warp_incl_scan(c, lane) + carry;
+                    carry = __shfl_sync(0xffffffffu, S, 31);
+                    if (j < klen) emit1<OUT>(row, kst + j, j == 0 ? kh : __fmaf_rn((float)S, unit, kh), shv, scv);
                 }
             }
         }
-    };
-    // entry of line g (g in the current window), broadcast to all lanes
-    auto entry = [&](uint64_t g, const uint8_t *&src, uint32_t &bytes, uint32_t &flags) {
-        const int k = (int)(g - wbase);
-        src = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_src, k));
-        bytes = __shfl_sync(0xffffffffu, w_bytes, k);
-        flags = __shfl_sync(0xffffffffu, w_flags, k);
-    };
-    auto consts = [&](uint64_t g, float &sh, float &sc) {  // g in the current window
-        const int k = (int)(g - wbase);
-        sh = __shfl_sync(0xffffffffu, w_shv, k);
-        sc = __shfl_sync(0xffffffffu, w_scv, k);
-    };
-    auto issue = [&](int slot, const uint8_t *src, uint32_t bytes) {  // lane 0
-        if constexpr (VPL == 36) bulk_wait_read_all();  // a staged row may still be leaving this slot
-        mbar_arrive_expect_tx(&mbar[slot], bytes);
-        bulk_g2s(base + slot * cap, src, bytes, &mbar[slot]);
-    };
-
-    uint32_t phases = 0;  // bit k: parity of slot k's mbarrier
-    int slot = 0;
-    load_window(g_begin);
-    const uint8_t *cur_src;
-    uint32_t cur_bytes, cur_flags;
-    entry(g_begin, cur_src, cur_bytes, cur_flags);
-    if (lane == 0 && cur_bytes && !(cur_flags & 1u)) issue(0, cur_src, cur_bytes);
-    for (uint64_t g = g_begin; g < g_end; g++) {
-        float shv, scv;
-        consts(g, shv, scv);  // before the window may move on to g + 1
-        const uint8_t *nxt_src = nullptr;
-        uint32_t nxt_bytes = 0, nxt_flags = 0, nxt_issued = 0;
-        if (g + 1 < g_end) {
-            if (g + 1 >= wbase + kWarp) load_window(g + 1);
-            entry(g + 1, nxt_src, nxt_bytes, nxt_flags);
-            // an oversize current line occupies both slots: issue the next one later
-            if (nxt_bytes && !(nxt_flags & 1u) && !(cur_flags & 1u)) {
-                if (lane == 0) issue(slot ^ 1, nxt_src, nxt_bytes);
-                nxt_issued = 1;
-            }
-        }
-        const uint32_t bytes = cur_bytes;
-        const uint32_t big = cur_flags & 1u;
-        const uint32_t al = cur_flags >> 16;
-        if (bytes) {
-            uint8_t *buf = base + slot * cap;
-            if (big) {
-                if constexpr (VPL == 36) {
-                    if (lane == 0) bulk_wait_read_all();  // both slots are about to be overwritten
-                    __syncwarp();
-                }
-                // stage across both slots with plain 16-B loads (rare: SEG line larger than RAW)
-                const uint4 *src4 = reinterpret_cast<const uint4 *>(cur_src);
-                for (uint32_t k = lane; k < bytes / 16; k += kWarp) reinterpret_cast<uint4 *>(base)[k] = src4[k];
-                fence_proxy_async_smem();  // generic writes before later TMA writes to these slots
-                __syncwarp();
-                buf = base;
-            } else {
-                mbar_wait(&mbar[slot], (phases >> slot) & 1u);
-                phases ^= 1u << slot;
-            }
-            uint8_t *row = dst + g * (uint64_t)W * ob;
-            bool ok;
-            if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg)) {
-                if constexpr (VPL == 36) ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
-                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
-            }
-            else
-                ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
-            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
-        }
-        __syncwarp();
-        if (lane == 0 && nxt_bytes && !(nxt_flags & 1u) && !nxt_issued) issue(slot ^ 1, nxt_src, nxt_bytes);
-        slot ^= 1;
-        cur_bytes = nxt_bytes;
-        cur_flags = nxt_flags;
-        cur_src = nxt_src;
     }
-    if constexpr (VPL == 36) {
-        if (lane == 0) bulk_wait_all();  // shared memory must outlive the last row stores
-    }
+    return cl == W;
 }
 
 // ---------------------------------------------------------------------------
-// Warp-specialised KD (default): the last warp of each CTA is a producer whose
-// lane k streams the lines of consumer warp k into that warp's two shared
-// slots (directory read + validation, channel constants, 1-D TMA bulk copy,
+// Warp-specialised KD: the last warp of each CTA is a producer whose lane k
+// streams the lines of consumer warp k into that warp's ring of input slots
+// (directory read + validation, channel constants, 1-D TMA bulk copy,
 // full/empty mbarriers per slot), so the decoding warps spend their issue
 // slots on decoding only.  A consumer waits for its slot, decodes the line
-// exactly as kd_decode does (same device functions), and releases the slot
-// once its staged row has left shared memory.  An oversize line (> one slot)
-// is copied across both slots after both are released.
-#ifndef SPP_KD_WS
-#define SPP_KD_WS 1
-#endif
+// and releases the slot as soon as it has read it (one-pass rows are staged in
+// the warp's own row buffer, never in the input slot).  A line longer than one
+// slot takes the whole ring; a line longer than the ring (or any line when W
+// exceeds the shared tables) is handed over as a record only and decoded from
+// HBM by decode_line_global.
 #ifndef SPP_KD_WS_WPC
 #define SPP_KD_WS_WPC 11  // consumer warps per CTA (+1 producer warp)
 #endif
@@ -936,32 +908,33 @@ constexpr int kWsWarps = SPP_KD_WS_WPC + 1;
 #define SPP_KD_WS_NS 3  // input slots per consumer warp (a ring)
 #endif
 #ifndef SPP_KD_WS_SLOT
-#define SPP_KD_WS_SLOT 2560  // target slot bytes (>= the staged row); longer lines take the whole ring
+#define SPP_KD_WS_SLOT 2048  // target slot bytes; longer lines take the whole ring, longer still the global path
 #endif
 constexpr uint32_t kWsNs = SPP_KD_WS_NS;
 static_assert(kWsNs >= 2 && kWsNs <= 8, "slot ring");
 constexpr uint32_t kWsCtl = 32 * kWsNs;  // per consumer: full[NS], empty[NS] mbarriers + info[NS] (16 B each)
+constexpr uint32_t kFlagBig = 1u, kFlagGlobal = 2u;  // line record flags (bits 16.. = alignment A)
 
 template <int OUT, bool VEC, int VPL, bool RAWSEG>  // RAWSEG: opts.raw_segments (mode-3 lines in one pass)
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
-    const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t nwords, uint32_t warp_bytes,
-    uint32_t *__restrict__ status) {
+    const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t rowb, uint32_t nwords,
+    uint32_t warp_bytes, uint32_t *__restrict__ status) {
     extern __shared__ __align__(16) uint8_t smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int wpc = (int)(blockDim.x >> 5) - 1;  // consumer warps; warp wpc produces
     const size_t ob = OUT == SPP_OUT_F32 ? 4 : 2;
-    const uint32_t cap_data = cap - 16;     // one slot; the last 16 B are read slack
+    const uint32_t cap_data = cap - 16;         // one slot; the last 16 B are read slack
     const uint32_t big_cap = kWsNs * cap - 16;  // the whole ring
     const uint64_t T = (uint64_t)n * L;
     const uint64_t NW = (uint64_t)gridDim.x * wpc;
-    const uint32_t ctl_off = (kWsNs * cap + 8 * nwords + 15u) & ~15u;  // 16-B aligned: info[] is read as uint4
+    const uint32_t ctl_off = (kWsNs * cap + rowb + 4 * nwords + 15u) & ~15u;  // 16-B aligned: info[] is read as uint4
     auto ctl = [&](int w) { return reinterpret_cast<uint64_t *>(smem_raw + (size_t)w * warp_bytes + ctl_off); };
 
     if (warp == wpc && lane < wpc) {
         uint64_t *c = ctl(lane);
         for (uint32_t i = 0; i < kWsNs; i++) {
-            mbar_init(&c[i], 1);            // full[i]: the producer lane's arrival + the TMA bytes
+            mbar_init(&c[i], 1);              // full[i]: the producer lane's arrival + the TMA bytes
             mbar_init(&c[kWsNs + i], kWarp);  // empty[i]: every consumer lane (each has read the slot)
         }
         fence_mbar_init();
@@ -1011,12 +984,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
                 const bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= m.limit && db - da >= 16;
                 if (!ok) {
                     report(status, SPP_ERR_CORRUPT, (int64_t)sk);
-                } else if (db - da > big_cap) {
-                    report(status, SPP_ERR_UNSUPPORTED, (int64_t)sk);
                 } else {
                     e_bytes = db - da;
                     e_src = m.payload + da;
-                    e_flags = (e_bytes > cap_data ? 1u : 0u) | (m.align << 16);
+                    // too long for the ring, or W beyond the shared tables: decoded from HBM
+                    e_flags = (nwords == 0 || e_bytes > big_cap ? kFlagGlobal : (e_bytes > cap_data ? kFlagBig : 0u)) |
+                              (m.align << 16);
                 }
             }
         };
@@ -1032,7 +1005,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
         while (__any_sync(0xffffffffu, active)) {
             bool did = false;
             if (active) {
-                const bool big = e_flags & 1u;
+                const bool big = e_flags & kFlagBig;
+                const bool glob = e_flags & kFlagGlobal;
                 bool ready;
                 if (!big) {
                     ready = !((used >> s) & 1u) || mbar_test(&empty[s], (par >> s) & 1u);
@@ -1042,12 +1016,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
                         ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
                 }
                 if (ready) {
-                    // the line record (16 B, st.async) and its bytes (TMA) both count
-                    // on full[s]; a zero-byte line delivers only the record
-                    mbar_arrive_expect_tx(&full[s], e_bytes + 16u);
+                    // the line record (16 B, st.async) and its bytes (TMA) both count on
+                    // full[s]; a zero-byte line delivers only the record, a global line
+                    // its record with the source address in place of the channel constants
+                    const uint32_t tx = glob ? 0u : e_bytes;
+                    mbar_arrive_expect_tx(&full[s], tx + 16u);
+                    const uint64_t sa = reinterpret_cast<uint64_t>(e_src);
                     st_async_u4(smem_u32(&info[s]),
-                                make_uint4(e_bytes, e_flags, __float_as_uint(shv), __float_as_uint(scv)), &full[s]);
-                    if (e_bytes) bulk_g2s(big ? rb : rb + s * cap, e_src, e_bytes, &full[s]);
+                                glob ? make_uint4(e_bytes, e_flags, (uint32_t)sa, (uint32_t)(sa >> 32))
+                                     : make_uint4(e_bytes, e_flags, __float_as_uint(shv), __float_as_uint(scv)),
+                                &full[s]);
+                    if (tx) bulk_g2s(big ? rb : rb + s * cap, e_src, tx, &full[s]);
                     const uint32_t took = big ? (1u << kWsNs) - 1u : 1u << s;
                     par ^= took & used;
                     used |= took;
@@ -1085,11 +1064,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     const uint64_t gw = (uint64_t)blockIdx.x * wpc + warp;
     const uint64_t g_begin = gw * T / NW, g_end = (gw + 1) * T / NW;
     uint8_t *base = smem_raw + (size_t)warp * warp_bytes;
-    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + kWsNs * cap);
-    uint32_t *wpre = sbits + nwords;
+    uint8_t *rowbuf = base + kWsNs * cap;  // one-pass instances: the staged output row
+    uint32_t *sbits = reinterpret_cast<uint32_t *>(base + kWsNs * cap + rowb);
+    uint32_t *wpre = sbits + nwords / 2;
     uint64_t *full = ctl(warp), *empty = full + kWsNs;
     const uint32_t info_s = smem_u32(full + 2 * kWsNs);
     const uint32_t nbw = (W / VPL + 31) / 32;
+    const uint32_t nsb = nwords / 2;  // words of the start bitmap (and of its prefix counts)
     uint32_t fph = 0;  // bit s: parity of slot s's next full phase
     uint32_t s = 0;
     for (uint64_t g = g_begin; g < g_end; g++, s = s + 1 == kWsNs ? 0u : s + 1) {
@@ -1097,32 +1078,40 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
         fph ^= 1u << s;
         const uint4 inf = lds_u4(info_s + 16u * s);
         const uint32_t bytes = inf.x, flags = inf.y, al = flags >> 16;
+        uint8_t *row = dst + g * (uint64_t)W * ob;
+        if (flags & kFlagGlobal) {
+            // record only: release the slot at once, decode the line from HBM
+            mbar_arrive(&empty[s]);
+            const uint8_t *src = reinterpret_cast<const uint8_t *>((uint64_t)inf.w << 32 | inf.z);
+            const uint32_t c = (uint32_t)(g % L) / H;
+            const float shv = shift ? __ldg(shift + c) : 0.f, scv = scale ? __ldg(scale + c) : 1.f;
+            const bool ok = decode_line_global<OUT>(src, bytes, W, al, shv, scv, row, lane);
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
+            continue;
+        }
         if (bytes) {
-            uint8_t *buf = (flags & 1u) ? base : base + s * cap;
+            uint8_t *buf = (flags & kFlagBig) ? base : base + s * cap;
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
-            uint8_t *row = dst + g * (uint64_t)W * ob;
             bool ok;
             if (RAWSEG && buf[0] == kModeRaw16) {
-                if constexpr (RAWSEG && VPL == 36) ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, lane);
+                if constexpr (RAWSEG && VPL == 36)
+                    ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, rowbuf, lane);
             } else if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (RAWSEG && buf[0] == kModeSegRaw))) {
                 if constexpr (VPL == 36) {
                     if (!RAWSEG || buf[0] == kModeSeg)
-                        ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                        ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
                     else
-                        ok = decode_line_onepass<OUT, true>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                        ok = decode_line_onepass<OUT, true>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
                 }
-                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, lane);
+                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
             } else {
-                ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nwords, shv, scv, row, lane);
+                ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nsb, shv, scv, row, lane);
             }
             if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
         }
-        if constexpr (VPL == 36) {
-            if (lane == 0) bulk_wait_read_all();  // the staged row has left the slot
-        }
         __syncwarp();
         // every lane releases: its own reads of the slot and of info[s] precede its arrival
-        if (flags & 1u) {
+        if (flags & kFlagBig) {
             for (uint32_t i = 0; i < kWsNs; i++) mbar_arrive(&empty[i]);  // the line took the whole ring
         } else {
             mbar_arrive(&empty[s]);
@@ -1137,22 +1126,35 @@ template <int OUT, bool VEC, int VPL, bool RAWSEG>
 spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
                         const DeviceProps &dp) {
     const uint32_t W = (uint32_t)o.W;
-    // slot: a typical SEG line (~1 B/value) and the staged output row; a RAW
-    // line (or any longer line) takes the whole ring, which always holds RAW
+    const bool smem_tables = W <= kSmemMaxW;  // else every line takes the global path
+    // slot: a typical SEG line (~1 B/value); a RAW line (or any longer line)
+    // takes the whole ring; a line longer than the ring is decoded from HBM
     const uint32_t raw = (uint32_t)round_up16(16 + 4ull * W);
-    const uint32_t row = VPL == 36 ? W * (OUT == SPP_OUT_F32 ? 4u : 2u) : 0u;
-    uint32_t cap_in = std::min<uint32_t>(raw, SPP_KD_WS_SLOT);
-    cap_in = std::max<uint32_t>(cap_in, (uint32_t)round_up16((raw + kWsNs - 1) / kWsNs));
-    const uint32_t cap = (uint32_t)round_up16(std::max(cap_in, row)) + 16;
-    const uint32_t nwords = (W + 31) / 32 + 1;
-    const uint32_t warp_bytes = (uint32_t)round_up16(kWsNs * cap + 8 * nwords) + kWsCtl;
+    uint32_t cap_in = 16;
+    if (smem_tables) {
+        cap_in = std::min<uint32_t>(raw, SPP_KD_WS_SLOT);
+        cap_in = std::max<uint32_t>(cap_in, std::min<uint32_t>((uint32_t)round_up16((raw + kWsNs - 1) / kWsNs),
+                                                               2 * SPP_KD_WS_SLOT));
+    }
+    const uint32_t cap = (uint32_t)round_up16(cap_in) + 16;
+    const uint32_t rowb = VPL == 36 ? W * (OUT == SPP_OUT_F32 ? 4u : 2u) : 0u;  // one-pass row buffer
+    const uint32_t nwords = smem_tables ? 2 * ((W + 31) / 32 + 1) : 0u;        // start bitmap + prefix counts
+    const uint32_t warp_bytes = (uint32_t)round_up16(kWsNs * cap + rowb + 4 * nwords) + kWsCtl;
+    // consumer warps per CTA: as many as fit two CTAs per SM (else one)
     int wpc = SPP_KD_WS_WPC;
-    while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
-    if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
+    auto fits = [&](int w, int ctas) {
+        return (size_t)w * warp_bytes <= (size_t)dp.smem_optin &&
+               (size_t)ctas * ((size_t)w * warp_bytes + dp.smem_reserved) <= (size_t)dp.smem_per_sm;
+    };
+    while (wpc > 1 && !fits(wpc, 2)) wpc--;
+    if (!fits(wpc, 2)) {
+        wpc = SPP_KD_WS_WPC;
+        while (wpc > 1 && !fits(wpc, 1)) wpc--;
+    }
+    if (!fits(wpc, 1)) return SPP_ERR_UNSUPPORTED;
     const int smem = wpc * (int)warp_bytes;
     auto kern = kd_decode_ws<OUT, VEC, VPL, RAWSEG>;
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
-        return SPP_ERR_CUDA;
+    if (set_smem_attr<kd_decode_ws<OUT, VEC, VPL, RAWSEG>>(smem, dp) != SPP_OK) return SPP_ERR_CUDA;
     int occ = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, (wpc + 1) * kWarp, smem) != cudaSuccess || occ < 1)
         return SPP_ERR_CUDA;
@@ -1162,33 +1164,8 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
     int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
     grid += grid & 1;
     kern<<<grid, (wpc + 1) * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift,
-                                                     o.scale, static_cast<uint8_t *>(d_dst), cap, nwords, warp_bytes,
-                                                     o.status);
-    return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
-}
-
-template <int OUT, bool VEC, int VPL>
-spp_status launch_kd(const DcMeta *meta, int n, void *d_dst, const spp_decode_opts &o, cudaStream_t stream,
-                     const DeviceProps &dp) {
-    const uint32_t W = (uint32_t)o.W;
-    const uint32_t cap = (uint32_t)round_up16(16 + 4ull * W) + 16;
-    const uint32_t nwords = (W + 31) / 32 + 1;  // start bitmap (+1 spare word), and its prefix counts
-    const uint32_t warp_bytes = (uint32_t)round_up16(2 * cap + 8 * nwords + 16);  // keeps every warp region 16-B aligned
-    int wpc = kMaxWarpsPerCta;
-    while (wpc > 1 && (size_t)wpc * warp_bytes > (size_t)dp.smem_optin) wpc--;
-    if ((size_t)warp_bytes > (size_t)dp.smem_optin) return SPP_ERR_UNSUPPORTED;
-    const int smem = wpc * (int)warp_bytes;
-    auto kern = kd_decode<OUT, VEC, VPL>;
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
-        return SPP_ERR_CUDA;
-    int occ = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, wpc * kWarp, smem) != cudaSuccess || occ < 1)
-        return SPP_ERR_CUDA;
-    const uint64_t lines = (uint64_t)n * o.C * o.H;
-    const uint64_t max_ctas = (uint64_t)dp.sms * occ;
-    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
-    kern<<<grid, wpc * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift, o.scale,
-                                               static_cast<uint8_t *>(d_dst), cap, nwords, warp_bytes, o.status);
+                                                     o.scale, static_cast<uint8_t *>(d_dst), cap, rowb, nwords,
+                                                     warp_bytes, o.status);
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }
 
@@ -1198,7 +1175,6 @@ size_t deepcam_workspace_bytes(int n) { return n <= 0 ? 0 : round_up16((size_t)n
 
 spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const spp_decode_opts &o,
                           cudaStream_t stream) {
-    if (o.W > kMaxW) return SPP_ERR_UNSUPPORTED;
     DeviceProps dp;
     spp_status st = current_device_props(&dp);
     if (st != SPP_OK) return st;
@@ -1215,13 +1191,8 @@ spp_status deepcam_decode(const void *const *d_src, int n, void *d_dst, const sp
     // opts.raw_segments: the W = 1152 instance that also takes mode-3 lines
     // (FORMAT.md 2.7) in one pass; without it they take the general line path
     const bool rs = v36 && o.raw_segments;
-#if SPP_KD_WS
 #define SPP_LAUNCH_KD(OUT, VEC, VPL) launch_kd_ws<OUT, VEC, VPL, false>(meta, n, d_dst, o, stream, dp)
 #define SPP_LAUNCH_KD_RS(OUT) launch_kd_ws<OUT, true, 36, true>(meta, n, d_dst, o, stream, dp)
-#else
-#define SPP_LAUNCH_KD(OUT, VEC, VPL) launch_kd<OUT, VEC, VPL>(meta, n, d_dst, o, stream, dp)
-#define SPP_LAUNCH_KD_RS(OUT) launch_kd<OUT, true, 36>(meta, n, d_dst, o, stream, dp)
-#endif
     if (o.out == SPP_OUT_F32)
         r = rs ? SPP_LAUNCH_KD_RS(SPP_OUT_F32)
                : v36 ? SPP_LAUNCH_KD(SPP_OUT_F32, true, 36)

@@ -31,6 +31,8 @@ struct spp_pipeline {
     cudaStream_t copy = nullptr;
     std::vector<cudaEvent_t> copied, freed;
     std::vector<int> freed_pending;
+    cudaEvent_t done = nullptr;  // recorded after a call's last decode; the next call's stream waits on it
+    bool done_pending = false;
     int last_launches = 0;
 };
 
@@ -44,6 +46,7 @@ static void destroy_impl(spp_pipeline *p) {
         if (p->freed[i]) { cudaEventSynchronize(p->freed[i]); cudaEventDestroy(p->freed[i]); }
         if (p->copied[i]) cudaEventDestroy(p->copied[i]);
     }
+    if (p->done) { cudaEventSynchronize(p->done); cudaEventDestroy(p->done); }
     if (p->copy) cudaStreamDestroy(p->copy);
     cudaFree(p->d_stage);
     cudaFree(p->d_ptrs);
@@ -85,6 +88,7 @@ spp_status spp_pipeline_create(spp_pipeline **out, spp_format fmt, const spp_dec
     for (int i = 0; ok && i < nslots; i++)
         ok = cudaEventCreateWithFlags(&p->copied[i], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&p->freed[i], cudaEventDisableTiming) == cudaSuccess;
+    ok = ok && cudaEventCreateWithFlags(&p->done, cudaEventDisableTiming) == cudaSuccess;
     if (!ok) {
         cudaGetLastError();
         destroy_impl(p);
@@ -114,6 +118,9 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
     spp_decode_opts o = *opts;
     o.workspace = p->d_ws;
     o.workspace_size = p->ws_bytes;
+    // the previous call may still be decoding on another stream: the shared
+    // workspace (per-chunk meta / f(U)) must not be rewritten before it is done
+    if (p->done_pending && cudaStreamWaitEvent(st, p->done, 0) != cudaSuccess) return SPP_ERR_CUDA;
     int i = 0, chunk = 0;
     while (i < n) {
         const int slot = chunk % p->nslots;
@@ -168,6 +175,8 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
         i += k;
         chunk++;
     }
+    if (cudaEventRecord(p->done, st) != cudaSuccess) return SPP_ERR_CUDA;
+    p->done_pending = true;
     return SPP_OK;
 }
 

@@ -161,6 +161,7 @@ class DecodeLoader:
             self.copied_pending = [False] * depth
             decoder.workspace(self.B)           # allocate before any capture
             self.graphs = [None] * depth
+            self.graph_version = decoder.version  # graphs hold the decoder's buffer addresses
         else:
             self.pipe = HostPipeline(decoder, slot_bytes=shard.max_sample_bytes() * chunk + 4096, nslots=3,
                                      max_chunk=chunk)
@@ -176,6 +177,12 @@ class DecodeLoader:
         self.copied[s].record(self.stream)
         self.copied_pending[s] = True
         if self.use_graph and n == self.B:
+            if self.graph_version != self.dec.version:
+                # the decoder replaced its workspace or normalisation tensors since
+                # capture: replaying would read freed memory / stale constants
+                self.stream.synchronize()
+                self.graphs = [None] * self.depth
+                self.graph_version = self.dec.version
             if self.graphs[s] is None:
                 self.dec.decode(self.ptr_dev[s], out=self.out[s], n=n)   # warm-up outside capture
                 g = t.cuda.CUDAGraph()

@@ -30,7 +30,7 @@ EXPORTS = (
     "spp_encode_deepcam_ex", "spp_encode_cosmo_ex",
     "spp_stream_info", "spp_decode_opts_init", "spp_decode_workspace_size", "spp_decoded_sample_bytes",
     "spp_decode_batch", "spp_decode_launches", "spp_pipeline_create", "spp_pipeline_destroy", "spp_decode_host",
-    "spp_pipeline_last_launches", "spp_set_l2_persisting", "spp_status_string", "spp_version",
+    "spp_pipeline_last_launches", "spp_status_string", "spp_version",
 )
 
 
@@ -86,7 +86,6 @@ def load() -> C.CDLL:
         "spp_pipeline_destroy": ([P], None),
         "spp_decode_host": ([P, P, P, I, P, C.POINTER(spp_decode_opts), P], I),
         "spp_pipeline_last_launches": ([P], I),
-        "spp_set_l2_persisting": ([SZ, C.POINTER(SZ)], I),
         "spp_status_string": ([I], C.c_char_p),
         "spp_version": ([], C.c_char_p),
     }
@@ -215,13 +214,6 @@ def spp_decode_host(handle: int, h_ptrs: Sequence[int], sizes: Sequence[int], d_
     ptrs = (C.c_void_p * n)(*h_ptrs)
     sz = (C.c_size_t * n)(*sizes)
     _check(load().spp_decode_host(handle, ptrs, sz, n, d_dst, C.byref(opts), stream), "spp_decode_host")
-
-
-def spp_set_l2_persisting(nbytes: int) -> int:
-    """Reserve an L2 persisting set-aside (device-wide, opt-in); returns the granted bytes."""
-    got = C.c_size_t(0)
-    _check(load().spp_set_l2_persisting(int(nbytes), C.byref(got)), "spp_set_l2_persisting")
-    return int(got.value)
 
 
 def spp_pipeline_last_launches(handle: int) -> int:

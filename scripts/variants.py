@@ -13,6 +13,9 @@ VARIANTS = {
     "kc_alllanes": [],
     "kc_lane0": ["SPP_KC_ALL_LANES_RELEASE=0"],
 }
+# VARIANTS_JSON='{"name": ["DEFINE=1", ...], ...}' overrides the table (build and run)
+if os.environ.get("VARIANTS_JSON"):
+    VARIANTS = json.loads(os.environ["VARIANTS_JSON"])
 OUT = ROOT / "paper_conf_ipps_ibrahimo22_b200" / "variants"
 
 

@@ -53,23 +53,34 @@ def test_gpu_arm_contract():
 
 
 @pytest.mark.gpu
-def test_gpu_arm_two_ranks():
+@pytest.mark.parametrize("scaling", ["weak", "strong"])
+def test_gpu_arm_two_ranks(scaling):
     """The multi-rank path of bench.py (torchrun, one process per rank, barrier +
-    MAX over ranks, whole-job throughput) with two ranks sharing this GPU over
-    gloo (the driver's scaling run uses NCCL, one GPU per rank)."""
+    MAX over ranks, whole-job throughput) for BOTH workloads (C2 headline + C4
+    secondary), with two ranks sharing this GPU over gloo (the driver's scaling
+    run uses NCCL, one GPU per rank)."""
     import os
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("needs a CUDA device")
     env = dict(os.environ, SPP_DIST_BACKEND="gloo")
+    port = 29731 + (scaling == "strong")
     out = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
-                          "--master-addr=127.0.0.1", "--master-port=29731", str(ROOT / "bench.py"), "--gpus", "2",
-                          "--batch", "32", "--pool", "2", "--steps", "3", "--warmup", "3", "--e2e-steps", "1"],
-                         capture_output=True, text=True, timeout=900, cwd=str(ROOT), env=env)
+                          "--master-addr=127.0.0.1", f"--master-port={port}", str(ROOT / "bench.py"), "--gpus", "2",
+                          "--batch", "32", "--secondary-batch", "4", "--pool", "2", "--steps", "3", "--warmup", "3",
+                          "--e2e-steps", "1", "--scaling", scaling],
+                         capture_output=True, text=True, timeout=1200, cwd=str(ROOT), env=env)
     assert out.returncode == 0, out.stderr[-2000:]
     lines = [l for l in out.stdout.splitlines() if l.strip().startswith("{")]
     assert len(lines) == 1, out.stdout
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["value"] > 0 and d["cpu_baseline"] is None
-    assert d["value"] == pytest.approx(2 * 32 * 3 / (d["ms_per_step"] * 3 / 1e3), rel=1e-6)
+    total = 64 if scaling == "weak" else 32
+    assert d["n_gpus"] == 2 and d["scaling"] == scaling and d["value"] > 0 and d["cpu_baseline"] is None
+    assert d["config"]["samples_per_step_all_ranks"] == total
+    assert d["value"] == pytest.approx(total * 3 / (d["ms_per_step"] * 3 / 1e3), rel=1e-6)
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] == 2 * 3
+    assert len(d["per_rank"]) == 2 and all(r["h2d_gbs"] > 0 and r["overlap"] > 0 for r in d["per_rank"])
+    assert len(d["config"]["placement"]) == 2
+    s = d["secondary"]                          # DeepCAM C4 at N = 2 as well
+    assert s["cfg"] == "C4" and s["value"] > 0 and s["units_per_step"] == (8 if scaling == "weak" else 4)
+    assert s["roofline"]["frac"] > 0 and len(s["per_rank"]) == 2 and s["cpu_baseline"] is None
