@@ -139,6 +139,17 @@ typedef struct {
     int raw_segments;  /* 1 = a line over the error budget may keep only its offending
                           A-blocks raw, as RAW segments of a mode-3 line (FORMAT.md 2.7),
                           when that is smaller and within the budget; 0 (default) = off */
+    const float *repeat_tol;  /* host fp32[C] or NULL (= all 0): per-channel REPEAT tolerance
+                                 (FORMAT.md 2.8; "all neighbouring values are similar",
+                                 DESIGN.md S15).  tau_c > 0: a run of values within tau_c of
+                                 its first value, |x_j - x_i| <= tau_c, may become a REPEAT
+                                 of x_i (decoded error <= tau_c); 0: bit-identical runs only.
+                                 Each finite and >= 0, else SPP_ERR_INVALID_ARG. */
+    const float *max_abs_err; /* host fp32[C] or NULL (= all 0): per-channel absolute error
+                                 bound (FORMAT.md 2.8).  eps_c > 0: every decoded value of
+                                 channel c satisfies |x̂ - x| <= eps_c; a SEG line that would
+                                 exceed it is kept uncompressed (RAW, or RAW16 / RAW segments
+                                 when allowed and within the bound).  0: no bound. */
 } spp_deepcam_params;
 
 /* spp_encode_deepcam with explicit policy knobs (params may be NULL = defaults);

@@ -73,6 +73,8 @@ def lib():
         L.orc_deepcam_encode_r.restype = I
         L.orc_deepcam_encode_s.argtypes = [P, I, I, I, I, I, I, C.c_float, I, I, I, P, SZ, C.POINTER(SZ)]
         L.orc_deepcam_encode_s.restype = I
+        L.orc_deepcam_encode_t.argtypes = [P, I, I, I, I, I, I, C.c_float, I, I, I, P, P, P, SZ, C.POINTER(SZ)]
+        L.orc_deepcam_encode_t.restype = I
         L.orc_f16_to_f32.argtypes = [C.c_uint16]; L.orc_f16_to_f32.restype = C.c_float
         L.orc_deepcam_align.argtypes = [I]; L.orc_deepcam_align.restype = I
         _lib = L
@@ -145,11 +147,13 @@ def f16_to_f32(h: int) -> float:
 
 def deepcam_encode(x: np.ndarray, align: int | None = None, lookahead: int = 64, repeat_min: int = 16,
                    rel_err: float = 0.1, err_budget: int = 0, raw16: bool = False,
-                   raw_segments: bool = False) -> np.ndarray:
+                   raw_segments: bool = False, repeat_tol=None, max_abs_err=None) -> np.ndarray:
     """FORMAT.md 2.4 encoder; `align` overrides the default alignment rule,
     `lookahead` / `repeat_min` the policy knobs (defaults 64 / 16);
     `err_budget` > 0 applies the FORMAT.md 2.5 error budget (a SEG line with
-    that many values above `rel_err` relative error is written RAW)."""
+    that many values above `rel_err` relative error is written RAW);
+    `repeat_tol` / `max_abs_err` (fp32[C] or None) the FORMAT.md 2.8 per-channel
+    REPEAT tolerance and absolute error bound."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     assert a.ndim == 3
     Cc, H, W = a.shape
@@ -157,8 +161,13 @@ def deepcam_encode(x: np.ndarray, align: int | None = None, lookahead: int = 64,
     dst = np.zeros(cap, dtype=np.uint8)
     size = C.c_size_t(0)
     A = lib().orc_deepcam_align(W) if align is None else int(align)
-    _check(lib().orc_deepcam_encode_s(_p(a), Cc, H, W, A, int(lookahead), int(repeat_min), float(rel_err),
-                                      int(err_budget), int(bool(raw16)), int(bool(raw_segments)), _p(dst), cap,
+    rt = None if repeat_tol is None else np.ascontiguousarray(repeat_tol, dtype=np.float32)
+    me = None if max_abs_err is None else np.ascontiguousarray(max_abs_err, dtype=np.float32)
+    assert rt is None or rt.shape == (Cc,)
+    assert me is None or me.shape == (Cc,)
+    _check(lib().orc_deepcam_encode_t(_p(a), Cc, H, W, A, int(lookahead), int(repeat_min), float(rel_err),
+                                      int(err_budget), int(bool(raw16)), int(bool(raw_segments)),
+                                      None if rt is None else _p(rt), None if me is None else _p(me), _p(dst), cap,
                                       C.byref(size)), "deepcam_encode")
     return dst[: size.value].copy()
 

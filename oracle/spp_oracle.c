@@ -557,9 +557,19 @@ static int ceil_log2(double q) {
  * byte size, or -1 if no aligned segmentation exists (the line is then RAW). */
 typedef struct { int len, kind, emin_b; float head; } seg_t;
 
-/* identical run at i, cut at the range end E (E = W for a whole line) */
-static int rep_len(const int *run, int i, int E, int A) {
-    int r = run[i] < E - i ? run[i] : E - i;
+/* The run that may become a REPEAT segment at i, cut at the range end E
+ * (E = W for a whole line).  tau = 0: the run of bit-identical values
+ * (FORMAT.md 2.4, run[] precomputed).  tau > 0 (FORMAT.md 2.8, "all
+ * neighbouring values are similar", reading S15): the longest run of values
+ * within tau of x[i], |x[j] - x[i]| <= tau in binary64. */
+static int run_at(const float *x, const int *run, int i, int E, double tau) {
+    if (tau == 0.0) return run[i] < E - i ? run[i] : E - i;
+    int k = 1;
+    while (i + k < E && fabs((double)x[i + k] - (double)x[i]) <= tau) k++;
+    return k;
+}
+static int rep_len(const float *x, const int *run, int i, int E, int A, double tau) {
+    int r = run_at(x, run, i, E, tau);
     return (i + r == E) ? r : (r / A) * A;
 }
 
@@ -567,12 +577,12 @@ static int rep_len(const int *run, int i, int E, int A) {
  * for the whole line; 2.7 encodes the ranges between RAW segments), appending
  * to segs / deltas.  Returns -1 when no aligned segmentation exists. */
 static int encode_range(const float *x, int i0, int E, int A, int lookahead, int repeat_min, seg_t *segs,
-                        int *nseg_io, uint8_t *deltas, int64_t *nd_io, const int *run) {
+                        int *nseg_io, uint8_t *deltas, int64_t *nd_io, const int *run, double tau) {
     int nseg = *nseg_io;
     int64_t nd = *nd_io;
     int i = i0;
     while (i < E) {
-        int rl = rep_len(run, i, E, A);
+        int rl = rep_len(x, run, i, E, A, tau);
         if (rl >= repeat_min) {
             segs[nseg].len = rl; segs[nseg].kind = 0; segs[nseg].emin_b = 0; segs[nseg].head = x[i];
             nseg++;
@@ -600,7 +610,7 @@ static int encode_range(const float *x, int i0, int E, int A, int lookahead, int
             int j = i + 1, overflow = 0;
             nd = nd0;
             while (j < E) {
-                if (j % A == 0 && rep_len(run, j, E, A) >= repeat_min) break;
+                if (j % A == 0 && rep_len(x, run, j, E, A, tau) >= repeat_min) break;
                 double t = ldexp((double)x[j] - (double)prev, -emin);
                 if (fabs(t) > 1984.5) { overflow = 1; break; }
                 int b = quantise(t);
@@ -628,14 +638,14 @@ static int encode_range(const float *x, int i0, int E, int A, int lookahead, int
 }
 
 static int64_t encode_line(const float *x, int W, int A, int lookahead, int repeat_min, seg_t *segs,
-                           int *nseg_out, uint8_t *deltas, int64_t *ndelta_out, int *run) {
+                           int *nseg_out, uint8_t *deltas, int64_t *ndelta_out, int *run, double tau) {
     /* run lengths of bit-identical values */
     run[W - 1] = 1;
     for (int i = W - 2; i >= 0; i--)
         run[i] = (bits_of_f32(x[i]) == bits_of_f32(x[i + 1])) ? run[i + 1] + 1 : 1;
     int nseg = 0;
     int64_t nd = 0;
-    if (encode_range(x, 0, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) < 0) return -1;
+    if (encode_range(x, 0, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run, tau) < 0) return -1;
     *nseg_out = nseg;
     *ndelta_out = nd;
     return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
@@ -682,73 +692,57 @@ int orc_deepcam_encode_q(const float *x, int C, int H, int W, int A, int lookahe
     return orc_deepcam_encode_r(x, C, H, W, A, lookahead, repeat_min, rel_err, err_budget, 0, dst, cap, size);
 }
 
-/* FORMAT.md 2.6: a line the error budget keeps uncompressed may be stored as
- * binary16 when every value is finite and its RNE binary16 rounding is within
- * rel of it (same metric as line_bad_count) */
-static int raw16_ok(const float *x, int W, double rel) {
-    for (int k = 0; k < W; k++) {
-        if (!isfinite(x[k])) return 0;
-        float h = orc_f16_to_f32(orc_f32_to_f16(x[k]));
-        if (!isfinite(h) || fabs((double)h - (double)x[k]) > rel * fabs((double)x[k])) return 0;
-    }
-    return 1;
-}
-
-/* FORMAT.md 2.5 ("areas with abrupt changes are kept uncompressed";
- * P:86 "roughly 3% of the values with larger than 10% error"): the number of
- * values of an encoded SEG line whose relative error exceeds rel (DESIGN.md
- * S19: |x̂ - x| > rel |x|, so x = 0 counts iff x̂ != 0), x̂ rebuilt from the
- * segments and codes exactly as the decoder of FORMAT.md 2.3 does. */
-static int line_bad_count(const float *x, const seg_t *segs, int nseg, const uint8_t *deltas, double rel) {
-    int bad = 0, pos = 0;
+/* x̂ of an encoded SEG line, position by position, exactly as the decoder of
+ * FORMAT.md 2.3 rebuilds it (RAW segments of 2.7: their stored values). */
+static void line_xhat(const float *x, const seg_t *segs, int nseg, const uint8_t *deltas, float *xh) {
+    int pos = 0;
     int64_t d = 0;
     for (int s = 0; s < nseg; s++) {
         float h = segs[s].head;
         if (segs[s].kind == 2) {                           /* RAW segment: exact (FORMAT.md 2.7) */
+            for (int j = 0; j < segs[s].len; j++) xh[pos + j] = x[pos + j];
             d += 4 * (int64_t)segs[s].len;
-        } else if (segs[s].kind == 0) {
-            for (int j = 0; j < segs[s].len; j++) if (fabs((double)h - (double)x[pos + j]) > rel * fabs((double)x[pos + j])) bad++;
-        } else {
+        } else if (segs[s].kind == 0) {                    /* REPEAT: the head */
+            for (int j = 0; j < segs[s].len; j++) xh[pos + j] = h;
+        } else {                                           /* DIFF: h, then RN(h + S * 2^emin) */
             float unit = ldexpf(1.0f, segs[s].emin_b - 150);
             int64_t S = 0;
-            if (fabs((double)h - (double)x[pos]) > rel * fabs((double)x[pos])) bad++;
+            xh[pos] = h;
             for (int j = 1; j < segs[s].len; j++) {
                 S += orc_deepcam_code(deltas[d++]);
-                float xh = h + (float)S * unit;
-                if (fabs((double)xh - (double)x[pos + j]) > rel * fabs((double)x[pos + j])) bad++;
+                xh[pos + j] = h + (float)S * unit;
             }
         }
         pos += segs[s].len;
     }
-    return bad;
 }
 
-/* FORMAT.md 2.7 encoder step: the blocks [bA, bA + A) holding a value above
- * rel in the 2.4 encoding (segs0 / deltas0) become RAW segments (a run of
- * them, one segment); the ranges between are re-encoded by the 2.4 policy.
- * Returns the line's SEG size, or -1. */
-static int64_t encode_line_rawseg(const float *x, int W, int A, int lookahead, int repeat_min, double rel,
-                                  const seg_t *segs0, int nseg0, const uint8_t *deltas0, const int *run,
-                                  uint8_t *flag, seg_t *segs, int *nseg_out, uint8_t *deltas, int64_t *nd_out) {
-    /* x-hat of the 2.4 encoding, position by position (FORMAT.md 2.3) */
-    int pos = 0;
-    int64_t d = 0;
-    for (int s = 0; s < nseg0; s++) {
-        float h = segs0[s].head;
-        if (segs0[s].kind == 0) {
-            for (int j = 0; j < segs0[s].len; j++) flag[pos + j] = fabs((double)h - (double)x[pos + j]) > rel * fabs((double)x[pos + j]);
-        } else {
-            float unit = ldexpf(1.0f, segs0[s].emin_b - 150);
-            int64_t S = 0;
-            flag[pos] = fabs((double)h - (double)x[pos]) > rel * fabs((double)x[pos]);
-            for (int j = 1; j < segs0[s].len; j++) {
-                S += orc_deepcam_code(deltas0[d++]);
-                float xh = h + (float)S * unit;
-                flag[pos + j] = fabs((double)xh - (double)x[pos + j]) > rel * fabs((double)x[pos + j]);
-            }
-        }
-        pos += segs0[s].len;
+/* The two error bounds a value is checked against (binary64 on binary32
+ * operands).  Relative (FORMAT.md 2.5; "areas with abrupt changes are kept
+ * uncompressed", "roughly 3% of the values with larger than 10% error";
+ * DESIGN.md S19): |x̂ - x| > rel |x|, so x = 0 counts iff x̂ != 0.  Absolute
+ * (FORMAT.md 2.8, per channel): |x̂ - x| > eps, eps > 0. */
+static int over_rel(float xh, float x, double rel) { return fabs((double)xh - (double)x) > rel * fabs((double)x); }
+static int over_abs(float xh, float x, double eps) { return eps > 0.0 && fabs((double)xh - (double)x) > eps; }
+
+/* FORMAT.md 2.6: every value finite and its RNE binary16 rounding within rel
+ * of it (and within eps when eps > 0, FORMAT.md 2.8) */
+static int raw16_ok(const float *x, int W, double rel, double eps) {
+    for (int k = 0; k < W; k++) {
+        if (!isfinite(x[k])) return 0;
+        float h = orc_f16_to_f32(orc_f32_to_f16(x[k]));
+        if (!isfinite(h) || over_rel(h, x[k], rel) || over_abs(h, x[k], eps)) return 0;
     }
+    return 1;
+}
+
+/* FORMAT.md 2.7 encoder step: the blocks [bA, bA + A) holding a flagged value
+ * of the 2.4 encoding (flag[] filled by the caller) become RAW segments (a run
+ * of them, one segment); the ranges between are re-encoded by the 2.4 policy.
+ * Returns the line's SEG size, or -1. */
+static int64_t encode_line_rawseg(const float *x, int W, int A, int lookahead, int repeat_min, const uint8_t *flag,
+                                  const int *run, double tau, seg_t *segs, int *nseg_out, uint8_t *deltas,
+                                  int64_t *nd_out) {
     int nb = (W + A - 1) / A, nseg = 0;
     int64_t nd = 0;
     int b = 0;
@@ -766,7 +760,7 @@ static int64_t encode_line_rawseg(const float *x, int W, int A, int lookahead, i
             segs[nseg].len = e0 - s0; segs[nseg].kind = 2; segs[nseg].emin_b = 0; segs[nseg].head = x[s0];
             nseg++;
             for (int k = s0; k < e0; k++) { wr32(deltas + nd, bits_of_f32(x[k])); nd += 4; }
-        } else if (encode_range(x, s0, e0, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) < 0) {
+        } else if (encode_range(x, s0, e0, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run, tau) < 0) {
             return -1;
         }
         b = b2;
@@ -776,119 +770,145 @@ static int64_t encode_line_rawseg(const float *x, int W, int A, int lookahead, i
     return (int64_t)up16(4 + 8 * (uint64_t)nseg + (uint64_t)nd);
 }
 
+typedef struct {
+    int A, lookahead, repeat_min, err_budget, raw16, rawseg;
+    double rel;
+    seg_t *segs, *segs2;
+    uint8_t *deltas, *deltas2, *flag;
+    int *run;
+    float *xh;
+    int nseg, nseg2;
+    int64_t nd, nd2;
+} enc_ctx;
+
+/* The line's encoding (FORMAT.md 2.4-2.8): 0 RAW, 1 SEG (segs/deltas), 2 RAW16,
+ * 3 SEG with RAW segments (segs2/deltas2); *size = its payload bytes.
+ * tau / eps: the line's channel's REPEAT tolerance and absolute bound (2.8). */
+static int decide_line(const float *x, int W, enc_ctx *c, double tau, double eps, uint64_t *size) {
+    uint64_t raw_size = up16(16 + 4 * (uint64_t)W), raw16_size = up16(16 + 2 * (uint64_t)W);
+    for (int k = 0; k < W; k++)
+        if (!isfinite(x[k])) { *size = raw_size; return 0; }     /* non-finite: RAW (2.4 step 1) */
+    int64_t seg_size = encode_line(x, W, c->A, c->lookahead, c->repeat_min, c->segs, &c->nseg, c->deltas, &c->nd,
+                                   c->run, tau);
+    if (seg_size >= 0 && (c->err_budget > 0 || eps > 0.0)) {
+        line_xhat(x, c->segs, c->nseg, c->deltas, c->xh);
+        int nrel = 0, nabs = 0;
+        for (int k = 0; k < W; k++) { nrel += over_rel(c->xh[k], x[k], c->rel); nabs += over_abs(c->xh[k], x[k], eps); }
+        if ((c->err_budget > 0 && nrel >= c->err_budget) || nabs > 0) {
+            /* kept uncompressed (2.5 / 2.8): RAW, RAW16 (2.6) or RAW segments (2.7) */
+            int mode = 0;
+            uint64_t sz = raw_size;
+            if (c->raw16 && raw16_ok(x, W, c->rel, eps)) { mode = 2; sz = raw16_size; }
+            if (c->rawseg) {
+                for (int k = 0; k < W; k++)
+                    c->flag[k] = (c->err_budget > 0 && over_rel(c->xh[k], x[k], c->rel)) || over_abs(c->xh[k], x[k], eps);
+                int64_t rs = encode_line_rawseg(x, W, c->A, c->lookahead, c->repeat_min, c->flag, c->run, tau, c->segs2,
+                                                &c->nseg2, c->deltas2, &c->nd2);
+                if (rs >= 0 && (uint64_t)rs < sz) {
+                    line_xhat(x, c->segs2, c->nseg2, c->deltas2, c->xh);
+                    int r2 = 0, a2 = 0;
+                    for (int k = 0; k < W; k++) { r2 += over_rel(c->xh[k], x[k], c->rel); a2 += over_abs(c->xh[k], x[k], eps); }
+                    if ((c->err_budget == 0 || r2 < c->err_budget) && a2 == 0) { mode = 3; sz = (uint64_t)rs; }
+                }
+            }
+            *size = sz;
+            return mode;
+        }
+    }
+    if (seg_size >= 0 && (uint64_t)seg_size < raw_size) { *size = (uint64_t)seg_size; return 1; }
+    *size = raw_size;                                    /* RAW on a tie (2.4 step 3) */
+    return 0;
+}
+
+int orc_deepcam_encode_t(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, int rawseg, const float *repeat_tol, const float *max_abs_err,
+                         uint8_t *dst, size_t cap, size_t *size);
 int orc_deepcam_encode_s(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
                          int err_budget, int raw16, int rawseg, uint8_t *dst, size_t cap, size_t *size) {
+    return orc_deepcam_encode_t(x, C, H, W, A, lookahead, repeat_min, rel_err, err_budget, raw16, rawseg, NULL, NULL,
+                                dst, cap, size);
+}
+
+/* The DeepCAM encoder (FORMAT.md 2.4-2.8) with every knob.  repeat_tol /
+ * max_abs_err: NULL or fp32[C], each finite and >= 0 (0 = off). */
+int orc_deepcam_encode_t(const float *x, int C, int H, int W, int A, int lookahead, int repeat_min, float rel_err,
+                         int err_budget, int raw16, int rawseg, const float *repeat_tol, const float *max_abs_err,
+                         uint8_t *dst, size_t cap, size_t *size) {
     if (!x || !size || C < 1 || H < 1 || W < 1 || C > 65535 || H > 65535 || W > 65535) return ORC_EINVAL;
     if (raw16 != 0 && raw16 != 1) return ORC_EINVAL;
     if (rawseg != 0 && rawseg != 1) return ORC_EINVAL;
-    uint64_t raw16_size = up16(16 + 2 * (uint64_t)W);
     if (lookahead < 2 || lookahead > 65535 || repeat_min < 2 || repeat_min > 65535) return ORC_EINVAL;
     if (err_budget < 0 || !(rel_err > 0.0f) || !(rel_err < 1e30f)) return ORC_EINVAL;
     if ((uint64_t)C * H > 0xFFFFFFFFull || A < 1 || W % A != 0) return ORC_EINVAL;
+    for (int c = 0; c < C; c++) {
+        if (repeat_tol && !(repeat_tol[c] >= 0.0f && repeat_tol[c] < INFINITY)) return ORC_EINVAL;
+        if (max_abs_err && !(max_abs_err[c] >= 0.0f && max_abs_err[c] < INFINITY)) return ORC_EINVAL;
+    }
     init_mags();
     uint64_t L = (uint64_t)C * H;
     uint64_t dir_off = 64, payload_off = up16(dir_off + 4 * (L + 1));
-    uint64_t raw_size = up16(16 + 4 * (uint64_t)W);
-    seg_t *segs = malloc(sizeof(seg_t) * (size_t)W);
-    uint8_t *deltas = malloc((size_t)W);
-    int *run = malloc(sizeof(int) * (size_t)W);
-    seg_t *segs2 = malloc(sizeof(seg_t) * (size_t)W);      /* FORMAT.md 2.7 candidate line */
-    uint8_t *deltas2 = malloc(5 * (size_t)W), *flag = malloc((size_t)W);
-    int nseg2 = 0;
-    int64_t nd2 = 0;
+    enc_ctx c = {A, lookahead, repeat_min, err_budget, raw16, rawseg, (double)rel_err, NULL, NULL, NULL, NULL, NULL,
+                 NULL, NULL, 0, 0, 0, 0};
+    c.segs = malloc(sizeof(seg_t) * (size_t)W);
+    c.segs2 = malloc(sizeof(seg_t) * (size_t)W);
+    c.deltas = malloc((size_t)W);
+    c.deltas2 = malloc(5 * (size_t)W);
+    c.flag = malloc((size_t)W);
+    c.run = malloc(sizeof(int) * (size_t)W);
+    c.xh = malloc(sizeof(float) * (size_t)W);
     /* pass 1: sizes */
     uint64_t pay = 0;
     for (uint64_t l = 0; l < L; l++) {
-        const float *xl = x + l * (uint64_t)W;
-        int finite = 1;
-        for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
-        uint64_t sz = raw_size;
-        if (finite) {
-            int nseg; int64_t nd;
-            int64_t seg_size = encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run);
-            if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
-                seg_size = -1;                            /* over the error budget: RAW (FORMAT.md 2.5) */
-                if (raw16 && raw16_ok(xl, W, rel_err)) sz = raw16_size;   /* ... in binary16 (2.6) */
-                if (rawseg) {                             /* ... or with RAW segments (2.7) */
-                    int64_t rs = encode_line_rawseg(xl, W, A, lookahead, repeat_min, rel_err, segs, nseg, deltas, run,
-                                                    flag, segs2, &nseg2, deltas2, &nd2);
-                    if (rs >= 0 && (uint64_t)rs < sz && line_bad_count(xl, segs2, nseg2, deltas2, rel_err) < err_budget)
-                        sz = (uint64_t)rs;
-                }
-            }
-            if (seg_size >= 0 && (uint64_t)seg_size < raw_size) sz = (uint64_t)seg_size;
-        }
+        int ch = (int)(l / (uint64_t)H);
+        uint64_t sz;
+        decide_line(x + l * (uint64_t)W, W, &c, repeat_tol ? repeat_tol[ch] : 0.0, max_abs_err ? max_abs_err[ch] : 0.0,
+                    &sz);
         pay += sz;
     }
     uint64_t total = payload_off + pay;
     *size = (size_t)total;
-    if (total > 0xFFFFFFFFull + payload_off || !dst || cap < total) {
-        free(segs); free(deltas); free(run); free(segs2); free(deltas2); free(flag);
-        return total > 0xFFFFFFFFull + payload_off ? ORC_EINVAL : ORC_ESMALL;
-    }
-    memset(dst, 0, (size_t)total);
-    wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);
-    wr16(dst + 8, (uint16_t)C); wr16(dst + 10, (uint16_t)H); wr16(dst + 12, (uint16_t)W);
-    wr16(dst + 14, (uint16_t)A);
-    wr32(dst + 16, (uint32_t)L);
-    wr64(dst + 24, dir_off); wr64(dst + 32, payload_off); wr64(dst + 40, total);
-    uint64_t cur = 0;
-    for (uint64_t l = 0; l < L; l++) {
-        wr32(dst + dir_off + 4 * l, (uint32_t)cur);
-        const float *xl = x + l * (uint64_t)W;
-        uint8_t *p = dst + payload_off + cur;
-        int finite = 1;
-        for (int k = 0; k < W; k++) if (!isfinite(xl[k])) { finite = 0; break; }
-        int nseg = 0; int64_t nd = 0;
-        int64_t seg_size = finite ? encode_line(xl, W, A, lookahead, repeat_min, segs, &nseg, deltas, &nd, run) : -1;
-        int use16 = 0, use3 = 0;
-        if (seg_size >= 0 && err_budget > 0 && line_bad_count(xl, segs, nseg, deltas, rel_err) >= err_budget) {
-            seg_size = -1;
-            use16 = raw16 && raw16_ok(xl, W, rel_err);
-            if (rawseg) {
-                uint64_t alt = use16 ? raw16_size : raw_size;
-                int64_t rs = encode_line_rawseg(xl, W, A, lookahead, repeat_min, rel_err, segs, nseg, deltas, run,
-                                                flag, segs2, &nseg2, deltas2, &nd2);
-                if (rs >= 0 && (uint64_t)rs < alt && line_bad_count(xl, segs2, nseg2, deltas2, rel_err) < err_budget) {
-                    use3 = 1;
-                    use16 = 0;
-                    p[0] = 3; wr16(p + 2, (uint16_t)nseg2);
-                    for (int s = 0; s < nseg2; s++) {
-                        wr16(p + 4 + 4 * s, (uint16_t)segs2[s].len);
-                        p[4 + 4 * s + 2] = (uint8_t)segs2[s].kind;
-                        p[4 + 4 * s + 3] = (uint8_t)segs2[s].emin_b;
-                        wr32(p + 4 + 4 * (uint64_t)nseg2 + 4 * s, bits_of_f32(segs2[s].head));
-                    }
-                    memcpy(p + 4 + 8 * (uint64_t)nseg2, deltas2, (size_t)nd2);
-                    cur += (uint64_t)rs;
+    int rc = ORC_OK;
+    if (total > 0xFFFFFFFFull + payload_off) rc = ORC_EINVAL;
+    else if (!dst || cap < total) rc = ORC_ESMALL;
+    if (rc == ORC_OK) {
+        memset(dst, 0, (size_t)total);
+        wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);
+        wr16(dst + 8, (uint16_t)C); wr16(dst + 10, (uint16_t)H); wr16(dst + 12, (uint16_t)W);
+        wr16(dst + 14, (uint16_t)A);
+        wr32(dst + 16, (uint32_t)L);
+        wr64(dst + 24, dir_off); wr64(dst + 32, payload_off); wr64(dst + 40, total);
+        uint64_t cur = 0;
+        for (uint64_t l = 0; l < L; l++) {
+            wr32(dst + dir_off + 4 * l, (uint32_t)cur);
+            const float *xl = x + l * (uint64_t)W;
+            uint8_t *p = dst + payload_off + cur;
+            int ch = (int)(l / (uint64_t)H);
+            uint64_t sz;
+            int mode = decide_line(xl, W, &c, repeat_tol ? repeat_tol[ch] : 0.0, max_abs_err ? max_abs_err[ch] : 0.0,
+                                   &sz);
+            p[0] = (uint8_t)mode;
+            if (mode == 0) {
+                for (int k = 0; k < W; k++) wr32(p + 16 + 4 * (uint64_t)k, bits_of_f32(xl[k]));
+            } else if (mode == 2) {
+                for (int k = 0; k < W; k++) wr16(p + 16 + 2 * (uint64_t)k, orc_f32_to_f16(xl[k]));
+            } else {
+                const seg_t *sg = mode == 1 ? c.segs : c.segs2;
+                int ns = mode == 1 ? c.nseg : c.nseg2;
+                wr16(p + 2, (uint16_t)ns);
+                for (int s = 0; s < ns; s++) {
+                    wr16(p + 4 + 4 * s, (uint16_t)sg[s].len);
+                    p[4 + 4 * s + 2] = (uint8_t)sg[s].kind;
+                    p[4 + 4 * s + 3] = (uint8_t)sg[s].emin_b;
+                    wr32(p + 4 + 4 * (uint64_t)ns + 4 * s, bits_of_f32(sg[s].head));
                 }
+                memcpy(p + 4 + 8 * (uint64_t)ns, mode == 1 ? c.deltas : c.deltas2, (size_t)(mode == 1 ? c.nd : c.nd2));
             }
+            cur += sz;
         }
-        if (use3) {
-            /* written above */
-        } else if (use16) {
-            p[0] = 2;
-            for (int k = 0; k < W; k++) wr16(p + 16 + 2 * (uint64_t)k, orc_f32_to_f16(xl[k]));
-            cur += raw16_size;
-        } else if (seg_size >= 0 && (uint64_t)seg_size < raw_size) {
-            p[0] = 1; wr16(p + 2, (uint16_t)nseg);
-            for (int s = 0; s < nseg; s++) {
-                wr16(p + 4 + 4 * s, (uint16_t)segs[s].len);
-                p[4 + 4 * s + 2] = (uint8_t)segs[s].kind;
-                p[4 + 4 * s + 3] = (uint8_t)segs[s].emin_b;
-                wr32(p + 4 + 4 * (uint64_t)nseg + 4 * s, bits_of_f32(segs[s].head));
-            }
-            memcpy(p + 4 + 8 * (uint64_t)nseg, deltas, (size_t)nd);
-            cur += (uint64_t)seg_size;
-        } else {
-            p[0] = 0;
-            for (int k = 0; k < W; k++) wr32(p + 16 + 4 * (uint64_t)k, bits_of_f32(xl[k]));
-            cur += raw_size;
-        }
+        wr32(dst + dir_off + 4 * L, (uint32_t)cur);
     }
-    wr32(dst + dir_off + 4 * L, (uint32_t)cur);
-    free(segs); free(deltas); free(run); free(segs2); free(deltas2); free(flag);
-    return ORC_OK;
+    free(c.segs); free(c.segs2); free(c.deltas); free(c.deltas2); free(c.flag); free(c.run); free(c.xh);
+    return rc;
 }
 
 /* ---------------- array helpers for the Python tests ---------------------- */

@@ -904,6 +904,9 @@ constexpr int kWsWarps = SPP_KD_WS_WPC + 1;
 #ifndef SPP_KD_PROD_SLEEP_NS
 #define SPP_KD_PROD_SLEEP_NS 100  // producer back-off when no slot was free this round
 #endif
+#ifndef SPP_KD_PROD_REACQUIRE
+#define SPP_KD_PROD_REACQUIRE 1
+#endif
 #ifndef SPP_KD_WS_NS
 #define SPP_KD_WS_NS 3  // input slots per consumer warp (a ring)
 #endif
@@ -1014,6 +1017,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
                     ready = true;
                     for (uint32_t i = 0; i < kWsNs; i++)
                         ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
+                }
+                if (ready && SPP_KD_PROD_REACQUIRE) {
+                    // the phases just found complete by test_wait are taken again with
+                    // try_wait (returns at once): same acquire semantics, but the form
+                    // compute-sanitizer's racecheck models, so it sees the consumer's
+                    // reads of the slot ordered before this refill
+                    for (uint32_t i = 0; i < kWsNs; i++)
+                        if ((((big ? (1u << kWsNs) - 1u : 1u << s) & used) >> i) & 1u)
+                            mbar_wait(&empty[i], (par >> i) & 1u);
                 }
                 if (ready) {
                     // the line record (16 B, st.async) and its bytes (TMA) both count on

@@ -14,6 +14,8 @@
 #include <string.h>
 
 #include <algorithm>
+#include <cmath>
+#include <utility>
 #include <cstdlib>
 #include <thread>
 #include <vector>
@@ -71,6 +73,8 @@ inline int alignment_for(int W) { return W == 1152 ? 36 : (W % 8 == 0 ? 8 : 1); 
 struct LineEncoder {
     int W, A;
     int lookahead, repeat_min;  // FORMAT.md 2.4 policy knobs (defaults 64, 16)
+    double tau = 0.0;           // FORMAT.md 2.8 REPEAT tolerance of the line's channel (0: bit-identical runs)
+    const float *xl = nullptr;  // the line being encoded (tolerant runs scan it)
     std::vector<int> run;
     std::vector<Seg> segs;
     std::vector<uint8_t> deltas;
@@ -80,9 +84,18 @@ struct LineEncoder {
         deltas.reserve(w);
     }
 
-    // identical run at i, cut at the range end E (E = W for a whole line)
+    // REPEAT candidate at i, cut at the range end E (E = W for a whole line):
+    // bit-identical values (tau = 0, FORMAT.md 2.4) or values within tau of x[i]
+    // ("all neighbouring values are similar"; FORMAT.md 2.8)
     int rep(int i, int E) const {
-        const int r = run[i] < E - i ? run[i] : E - i;
+        int r;
+        if (tau == 0.0) {
+            r = run[i] < E - i ? run[i] : E - i;
+        } else {
+            const double h = xl[i];
+            r = 1;
+            while (i + r < E && fabs((double)xl[i + r] - h) <= tau) r++;
+        }
         return i + r == E ? r : (r / A) * A;
     }
 
@@ -90,6 +103,7 @@ struct LineEncoder {
     int64_t encode(const float *x) {
         segs.clear();
         deltas.clear();
+        xl = x;
         run[W - 1] = 1;
         for (int i = W - 2; i >= 0; i--) run[i] = fbits(x[i]) == fbits(x[i + 1]) ? run[i + 1] + 1 : 1;
         if (!encode_range(x, 0, W)) return -1;
@@ -152,68 +166,67 @@ struct LineEncoder {
     }
 };
 
-// FORMAT.md 2.5 error budget (P:82 abrupt areas kept uncompressed, P:86 the
-// "> 10% error" statistic): values of the line just encoded whose relative
-// error exceeds rel (S19: |x̂ - x| > rel |x|), x̂ rebuilt from the
-// segments and codes by the decoder's arithmetic (FORMAT.md 2.3).
-int bad_values(const LineEncoder &e, const float *x, double rel) {
-    int bad = 0, pos = 0;
+// x̂ of the line just encoded, by the decoder's arithmetic (FORMAT.md 2.3; RAW
+// segments of 2.7 decode to their stored values)
+void rebuild(const LineEncoder &e, const float *x, std::vector<float> &xh) {
+    xh.resize(e.W);
+    int pos = 0;
     size_t d = 0;
-    auto over = [&](float xh, float xv) { return fabs((double)xh - (double)xv) > rel * fabs((double)xv); };
     for (const Seg &g : e.segs) {
-        if (g.kind == kRawSeg) {  // exact (FORMAT.md 2.7)
+        if (g.kind == kRawSeg) {
+            std::copy(x + pos, x + pos + g.len, xh.begin() + pos);
             d += 4 * (size_t)g.len;
         } else if (g.kind == kRepeat) {
-            for (int j = 0; j < g.len; j++) bad += over(g.head, x[pos + j]);
+            std::fill(xh.begin() + pos, xh.begin() + pos + g.len, g.head);
         } else {
             const float unit = ldexpf(1.0f, (int)g.emin_b - kEminBias);
             int64_t S = 0;
-            bad += over(g.head, x[pos]);
+            xh[pos] = g.head;
             for (int j = 1; j < g.len; j++) {
                 const uint8_t b = e.deltas[d++];
                 const int mag = kCodes.mag[b & 127];
                 S += (b & 0x80) ? -mag : mag;
-                bad += over(g.head + (float)S * unit, x[pos + j]);
+                xh[pos + j] = g.head + (float)S * unit;
             }
         }
         pos += g.len;
     }
-    return bad;
 }
 
-// FORMAT.md 2.7: from the 2.4 encoding in `e0`, the A-blocks holding a value
-// above rel become RAW segments (a run of them, one segment) and the ranges
-// between are re-encoded by the 2.4 policy, into `e`.  False if no aligned
-// segmentation exists.
-bool encode_rawseg(const LineEncoder &e0, LineEncoder &e, const float *x, double rel, std::vector<uint8_t> &flag) {
-    const int W = e0.W, A = e0.A;
-    flag.assign(W, 0);
-    int pos = 0;
-    size_t d = 0;
-    auto over = [&](float xh, float xv) { return fabs((double)xh - (double)xv) > rel * fabs((double)xv); };
-    for (const Seg &g : e0.segs) {
-        if (g.kind == kRepeat) {
-            for (int j = 0; j < g.len; j++) flag[pos + j] = over(g.head, x[pos + j]);
-        } else {
-            const float unit = ldexpf(1.0f, (int)g.emin_b - kEminBias);
-            int64_t S = 0;
-            flag[pos] = over(g.head, x[pos]);
-            for (int j = 1; j < g.len; j++) {
-                const uint8_t b = e0.deltas[d++];
-                const int mag = kCodes.mag[b & 127];
-                S += (b & 0x80) ? -mag : mag;
-                flag[pos + j] = over(g.head + (float)S * unit, x[pos + j]);
-            }
+// Error bounds of a decoded value (binary64 on the binary32 operands):
+// relative (FORMAT.md 2.5, "> 10% error", S19: |x̂ - x| > rel |x|)
+// and the per-channel absolute bound eps of FORMAT.md 2.8 (|x̂ - x| > eps, eps > 0)
+struct Bounds {
+    double rel, eps;
+    bool use_rel;  // the error budget is on
+    bool rel_over(float xh, float x) const { return fabs((double)xh - (double)x) > rel * fabs((double)x); }
+    bool abs_over(float xh, float x) const { return eps > 0.0 && fabs((double)xh - (double)x) > eps; }
+    // (values over rel, values over eps) of a rebuilt line
+    std::pair<int, int> count(const std::vector<float> &xh, const float *x, int W) const {
+        int r = 0, a = 0;
+        for (int k = 0; k < W; k++) {
+            r += rel_over(xh[k], x[k]);
+            a += abs_over(xh[k], x[k]);
         }
-        pos += g.len;
+        return {r, a};
     }
+};
+
+// FORMAT.md 2.7: the A-blocks of `e0`'s encoding holding a value over the bounds
+// become RAW segments (a run of them, one segment); the ranges between are
+// re-encoded by the 2.4 policy, into `e`.  False if no aligned segmentation exists.
+bool encode_rawseg(const LineEncoder &e0, const std::vector<float> &xh0, LineEncoder &e, const float *x,
+                   const Bounds &bd) {
+    const int W = e0.W, A = e0.A;
     e.segs.clear();
     e.deltas.clear();
     e.run = e0.run;
+    e.tau = e0.tau;
+    e.xl = x;
     const int nb = (W + A - 1) / A;
     auto block_bad = [&](int b) {
         for (int k = b * A; k < W && k < (b + 1) * A; k++)
-            if (flag[k]) return true;
+            if ((bd.use_rel && bd.rel_over(xh0[k], x[k])) || bd.abs_over(xh0[k], x[k])) return true;
         return false;
     };
     int b = 0;
@@ -247,12 +260,12 @@ inline float f16_to_f32(uint16_t u) {
     memcpy(&h, &u, 2);
     return (float)h;
 }
-// FORMAT.md 2.6: every value finite and its binary16 rounding within rel of it
-bool raw16_ok(const float *x, int W, double rel) {
+// FORMAT.md 2.6 / 2.8: every value finite and its binary16 rounding within the bounds
+bool raw16_ok(const float *x, int W, const Bounds &bd) {
     for (int k = 0; k < W; k++) {
         if (!isfinite(x[k])) return false;
         const float h = f16_to_f32(f32_to_f16(x[k]));
-        if (!isfinite(h) || fabs((double)h - (double)x[k]) > rel * fabs((double)x[k])) return false;
+        if (!isfinite(h) || bd.rel_over(h, x[k]) || bd.abs_over(h, x[k])) return false;
     }
     return true;
 }
@@ -286,11 +299,16 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     const int budget = params ? params->err_budget : 0;
     const int raw16 = params ? params->raw16 : 0;
     const int rawseg = params ? params->raw_segments : 0;
+    const float *tol = params ? params->repeat_tol : nullptr;      // FORMAT.md 2.8, fp32[C] or NULL
+    const float *abs_err = params ? params->max_abs_err : nullptr;  // FORMAT.md 2.8, fp32[C] or NULL
     if (raw16 != 0 && raw16 != 1) return SPP_ERR_INVALID_ARG;
     if (rawseg != 0 && rawseg != 1) return SPP_ERR_INVALID_ARG;
     const uint64_t raw16_size = round_up16(16 + 2 * (uint64_t)W);
     if (la < 2 || la > 65535 || rm < 2 || rm > 65535) return SPP_ERR_INVALID_ARG;
     if (budget < 0 || !(rel > 0.0f) || !(rel < 1e30f)) return SPP_ERR_INVALID_ARG;
+    for (int c = 0; c < C; c++)
+        if ((tol && !(tol[c] >= 0.0f && std::isfinite(tol[c]))) || (abs_err && !(abs_err[c] >= 0.0f && std::isfinite(abs_err[c]))))
+            return SPP_ERR_INVALID_ARG;
     const uint64_t L = (uint64_t)C * H;
     const uint64_t dir_off = spp::kHeaderBytes;
     const uint64_t payload_off = round_up16(dir_off + 4 * (L + 1));
@@ -312,40 +330,50 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
             th.emplace_back([&, i]() { body(L * i / nthr, L * (i + 1) / nthr); });
         for (auto &t : th) t.join();
     };
-    // pass 1: per-line size (SEG vs RAW)
-    std::vector<uint8_t> is_seg(L);
+    // Per-line choice (FORMAT.md 2.4-2.8): the line mode (0 RAW, 1 SEG in `enc`,
+    // 2 RAW16, 3 SEG with RAW segments in `enc3`) and its payload bytes.  A SEG
+    // line over the error budget (2.5) or with a value over its channel's absolute
+    // bound (2.8) is kept uncompressed: RAW16 (2.6) when its binary16 rounding is
+    // within the bounds, or RAW segments (2.7) when smaller and within the bounds.
+    struct Work {
+        LineEncoder enc, enc3;
+        std::vector<float> xh;
+    };
+    auto choose = [&](Work &w, uint64_t l, const float *xl, uint64_t &sz) -> uint8_t {
+        sz = raw_size;
+        if (!all_finite(xl, W)) return kModeRaw;
+        const int ch = (int)(l / (uint64_t)H);
+        const Bounds bd{(double)rel, abs_err ? (double)abs_err[ch] : 0.0, budget > 0};
+        w.enc.tau = tol ? (double)tol[ch] : 0.0;
+        const int64_t seg = w.enc.encode(xl);
+        if (seg >= 0 && (bd.use_rel || bd.eps > 0.0)) {
+            rebuild(w.enc, xl, w.xh);
+            const auto [nrel, nabs] = bd.count(w.xh, xl, W);
+            if ((bd.use_rel && nrel >= budget) || nabs > 0) {
+                uint8_t mode = kModeRaw;
+                if (raw16 && raw16_ok(xl, W, bd)) { mode = kModeRaw16; sz = raw16_size; }
+                if (rawseg && encode_rawseg(w.enc, w.xh, w.enc3, xl, bd)) {
+                    const uint64_t s3 = round_up16(4 + 8 * (uint64_t)w.enc3.segs.size() + w.enc3.deltas.size());
+                    if (s3 < sz) {
+                        std::vector<float> xh3;
+                        rebuild(w.enc3, xl, xh3);
+                        const auto [r3, a3] = bd.count(xh3, xl, W);
+                        if ((!bd.use_rel || r3 < budget) && a3 == 0) { mode = kModeSegRaw; sz = s3; }
+                    }
+                }
+                return mode;
+            }
+        }
+        if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; return kModeSeg; }
+        return kModeRaw;
+    };
+    // pass 1: per-line mode and size
+    std::vector<uint8_t> mode(L);
     std::vector<uint32_t> dir(L + 1);
     std::vector<uint64_t> line_size(L);
-    // a line over the error budget: RAW16 (2.6) if allowed, or RAW segments (2.7)
-    // when that is smaller and within the budget; 3 = mode-3 line
-    auto over_budget = [&](LineEncoder &enc, LineEncoder &enc3, std::vector<uint8_t> &flag, const float *xl,
-                           uint64_t &sz) -> uint8_t {
-        uint8_t kind = 0;
-        sz = raw_size;
-        if (raw16 && raw16_ok(xl, W, rel)) { sz = raw16_size; kind = 2; }
-        if (rawseg && encode_rawseg(enc, enc3, xl, rel, flag)) {
-            const uint64_t s3 = round_up16(4 + 8 * (uint64_t)enc3.segs.size() + enc3.deltas.size());
-            if (s3 < sz && bad_values(enc3, xl, rel) < budget) { sz = s3; kind = 3; }
-        }
-        return kind;
-    };
     parallel_lines([&](uint64_t l0, uint64_t l1) {
-        LineEncoder enc(W, A, la, rm), enc3(W, A, la, rm);
-        std::vector<uint8_t> flag;
-        for (uint64_t l = l0; l < l1; l++) {
-            const float *xl = x + l * (uint64_t)W;
-            uint64_t sz = raw_size;
-            is_seg[l] = 0;
-            if (all_finite(xl, W)) {
-                int64_t seg = enc.encode(xl);
-                if (seg >= 0 && budget > 0 && bad_values(enc, xl, rel) >= budget) {  // FORMAT.md 2.5
-                    seg = -1;
-                    is_seg[l] = over_budget(enc, enc3, flag, xl, sz);
-                }
-                if (seg >= 0 && (uint64_t)seg < raw_size) { sz = (uint64_t)seg; is_seg[l] = 1; }
-            }
-            line_size[l] = sz;
-        }
+        Work w{LineEncoder(W, A, la, rm), LineEncoder(W, A, la, rm), {}};
+        for (uint64_t l = l0; l < l1; l++) mode[l] = choose(w, l, x + l * (uint64_t)W, line_size[l]);
     });
     uint64_t cur = 0;
     for (uint64_t l = 0; l < L; l++) {
@@ -373,47 +401,38 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     memcpy(out + kPayloadOff, &payload_off, 8);
     memcpy(out + kTotal, &total, 8);
     memcpy(out + dir_off, dir.data(), 4 * (L + 1));
-    // pass 2: payloads
+    // pass 2: payloads (the choice is deterministic: recomputed per line)
     parallel_lines([&](uint64_t l0, uint64_t l1) {
-    LineEncoder enc(W, A, la, rm), enc3(W, A, la, rm);
-    std::vector<uint8_t> flag;
-    for (uint64_t l = l0; l < l1; l++) {
-        const float *xl = x + l * (uint64_t)W;
-        uint8_t *p = out + payload_off + dir[l];
-        if (!is_seg[l]) {
-            p[0] = kModeRaw;
-            memcpy(p + 16, xl, 4 * (size_t)W);
-            continue;
-        }
-        if (is_seg[l] == 2) {
-            p[0] = kModeRaw16;
-            for (int k = 0; k < W; k++) {
-                const uint16_t h = f32_to_f16(xl[k]);
-                memcpy(p + 16 + 2 * (size_t)k, &h, 2);
+        Work w{LineEncoder(W, A, la, rm), LineEncoder(W, A, la, rm), {}};
+        for (uint64_t l = l0; l < l1; l++) {
+            const float *xl = x + l * (uint64_t)W;
+            uint8_t *p = out + payload_off + dir[l];
+            p[0] = mode[l];
+            if (mode[l] == kModeRaw) {
+                memcpy(p + 16, xl, 4 * (size_t)W);
+                continue;
             }
-            continue;
-        }
-        enc.encode(xl);
-        uint8_t mode = kModeSeg;
-        if (is_seg[l] == 3) {  // FORMAT.md 2.7: rebuild the RAW-segment line (deterministic)
+            if (mode[l] == kModeRaw16) {
+                for (int k = 0; k < W; k++) {
+                    const uint16_t h = f32_to_f16(xl[k]);
+                    memcpy(p + 16 + 2 * (size_t)k, &h, 2);
+                }
+                continue;
+            }
             uint64_t sz;
-            over_budget(enc, enc3, flag, xl, sz);
-            std::swap(enc.segs, enc3.segs);
-            std::swap(enc.deltas, enc3.deltas);
-            mode = kModeSegRaw;
+            choose(w, l, xl, sz);
+            const LineEncoder &e = mode[l] == kModeSegRaw ? w.enc3 : w.enc;
+            const uint16_t nseg = (uint16_t)e.segs.size();
+            memcpy(p + 2, &nseg, 2);
+            for (int s = 0; s < nseg; s++) {
+                const Seg &g = e.segs[s];
+                memcpy(p + 4 + 4 * s, &g.len, 2);
+                p[4 + 4 * s + 2] = g.kind;
+                p[4 + 4 * s + 3] = g.emin_b;
+                memcpy(p + 4 + 4 * (size_t)nseg + 4 * s, &g.head, 4);
+            }
+            memcpy(p + 4 + 8 * (size_t)nseg, e.deltas.data(), e.deltas.size());
         }
-        const uint16_t nseg = (uint16_t)enc.segs.size();
-        p[0] = mode;
-        memcpy(p + 2, &nseg, 2);
-        for (int s = 0; s < nseg; s++) {
-            const Seg &g = enc.segs[s];
-            memcpy(p + 4 + 4 * s, &g.len, 2);
-            p[4 + 4 * s + 2] = g.kind;
-            p[4 + 4 * s + 3] = g.emin_b;
-            memcpy(p + 4 + 4 * (size_t)nseg + 4 * s, &g.head, 4);
-        }
-        memcpy(p + 4 + 8 * (size_t)nseg, enc.deltas.data(), enc.deltas.size());
-    }
     });
     return SPP_OK;
 }

@@ -46,7 +46,8 @@ class spp_cosmo_params(C.Structure):
 
 class spp_deepcam_params(C.Structure):
     _fields_ = [("lookahead", C.c_int), ("repeat_min", C.c_int), ("rel_err", C.c_float), ("err_budget", C.c_int),
-                ("raw16", C.c_int), ("raw_segments", C.c_int)]
+                ("raw16", C.c_int), ("raw_segments", C.c_int), ("repeat_tol", C.c_void_p),
+                ("max_abs_err", C.c_void_p)]
 
 
 class spp_decode_opts(C.Structure):
@@ -140,10 +141,13 @@ def spp_deepcam_max_encoded_size(Cc: int, H: int, W: int) -> int:
 
 
 def spp_encode_deepcam(x: np.ndarray, lookahead: int = 0, repeat_min: int = 0, rel_err: float = 0.0,
-                       err_budget: int = 0, raw16: bool = False, raw_segments: bool = False) -> np.ndarray:
+                       err_budget: int = 0, raw16: bool = False, raw_segments: bool = False, repeat_tol=None,
+                       max_abs_err=None) -> np.ndarray:
     """fp32 [C, H, W] -> encoded uint8 stream (FORMAT.md 2); nonzero knobs go
     through spp_encode_deepcam_ex (0 = the FORMAT.md 2.4 default; err_budget
-    > 0 = the FORMAT.md 2.5 error budget at relative error rel_err)."""
+    > 0 = the FORMAT.md 2.5 error budget at relative error rel_err;
+    repeat_tol / max_abs_err = the FORMAT.md 2.8 per-channel fp32[C] REPEAT
+    tolerance and absolute error bound)."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     if a.ndim != 3:
         raise ValueError("x must be [C, H, W]")
@@ -151,9 +155,15 @@ def spp_encode_deepcam(x: np.ndarray, lookahead: int = 0, repeat_min: int = 0, r
     cap = spp_deepcam_max_encoded_size(Cc, H, W)
     dst = np.empty(max(cap, 64), dtype=np.uint8)
     size = C.c_size_t(0)
-    if lookahead or repeat_min or rel_err or err_budget or raw16 or raw_segments:
+    rt = None if repeat_tol is None else np.ascontiguousarray(repeat_tol, dtype=np.float32)
+    me = None if max_abs_err is None else np.ascontiguousarray(max_abs_err, dtype=np.float32)
+    for arr in (rt, me):
+        if arr is not None and arr.shape != (Cc,):
+            raise ValueError("per-channel knobs are fp32[C]")
+    if lookahead or repeat_min or rel_err or err_budget or raw16 or raw_segments or rt is not None or me is not None:
         prm = spp_deepcam_params(int(lookahead), int(repeat_min), float(rel_err), int(err_budget), int(bool(raw16)),
-                                 int(bool(raw_segments)))
+                                 int(bool(raw_segments)), None if rt is None else rt.ctypes.data,
+                                 None if me is None else me.ctypes.data)
         _check(load().spp_encode_deepcam_ex(a.ctypes.data, Cc, H, W, C.byref(prm), dst.ctypes.data, dst.size,
                                             C.byref(size)), "spp_encode_deepcam_ex")
     else:

@@ -111,6 +111,37 @@ def test_deepcam_encoder_matches_oracle_bytes(spp, orc):
         assert a.size == b.size and np.array_equal(a, b)
 
 
+@pytest.mark.parametrize("knobs", [
+    dict(repeat_tol=0.02), dict(max_abs_err=0.003), dict(repeat_tol=0.02, max_abs_err=0.003, raw16=True),
+    dict(repeat_tol=0.01, max_abs_err=0.002, raw_segments=True, err_budget=4),
+    dict(max_abs_err=0.001, raw16=True, raw_segments=True, err_budget=16, rel_err=0.05)])
+def test_deepcam_tolerances_match_oracle_bytes(spp, orc, knobs):
+    """FORMAT.md 2.8 per-channel REPEAT tolerance and absolute bound (values as
+    fractions of each channel's std; one channel with both knobs at 0): the
+    product encoder writes the oracle's bytes."""
+    from synth import deepcam_stats, gen_deepcam
+    x = gen_deepcam(2007, H=24)
+    _, rstd = deepcam_stats(x)
+    kw = dict(knobs)
+    for k in ("repeat_tol", "max_abs_err"):
+        if k in kw:
+            v = (kw[k] / rstd).astype(np.float32)
+            v[5] = 0.0
+            kw[k] = v
+    a = spp.spp_encode_deepcam(x, **kw)
+    b = orc.deepcam_encode(x, **kw)
+    assert a.size == b.size and np.array_equal(a, b)
+
+
+def test_deepcam_tolerance_argument_errors(spp):
+    x = np.zeros((2, 2, 16), dtype=np.float32)
+    for bad in (np.float32([0.1, -1.0]), np.float32([np.inf, 0.0]), np.float32([np.nan, 0.0])):
+        for k in ("repeat_tol", "max_abs_err"):
+            with pytest.raises(spp.SppError) as e:
+                spp.spp_encode_deepcam(x, **{k: bad})
+            assert e.value.code == spp.SPP_ERR_INVALID_ARG
+
+
 def test_encoder_argument_errors(spp):
     with pytest.raises(spp.SppError) as e:
         spp.spp_encode_cosmo(-np.ones((4, 2, 2, 2), dtype=np.int16))

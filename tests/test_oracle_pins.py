@@ -795,3 +795,117 @@ def test_deepcam_segment_alignment(orc):
         orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=3), 0, W)
     with pytest.raises(orc.OracleError):
         orc.deepcam_decode_line(fmt.build_deepcam_stream(1, 1, W, [line], A=0), 0, W)
+
+
+# --------------------------------------------------------------------------
+# FORMAT.md 2.8: per-channel REPEAT tolerance ("all neighbouring values
+# are similar", reading S15) and absolute error bound
+
+def _repeat_bound_ok(x_line, xh_line, segs, tau):
+    """Every REPEAT position within tau of x, the head x at the segment start;
+    DIFF positions obey the S19 bound (_check_bound)."""
+    pos = 0
+    for s in segs:
+        ln = s["len"]
+        if s["kind"] == 0:
+            assert s["head"].view(np.uint32) == x_line[pos].view(np.uint32)
+            assert np.all(xh_line[pos:pos + ln].view(np.uint32) == x_line[pos].view(np.uint32))
+            assert np.all(np.abs(x_line[pos:pos + ln].astype(np.float64) - np.float64(x_line[pos])) <= tau)
+        else:
+            _check_bound(x_line[pos:pos + ln], xh_line[pos:pos + ln], [s])
+        pos += ln
+
+
+def test_deepcam_repeat_tolerance_closed_forms(orc):
+    """A line of c + noise with |noise| <= tau/2 is ONE REPEAT segment of its
+    first value at tolerance tau and not at tau = 0; two noisy plateaus meeting
+    at an aligned position are two REPEAT segments whose heads are the plateau
+    starts; a plateau meeting at an unaligned position ends on the previous
+    aligned position (FORMAT.md 2.4 alignment) and the rest is DIFF/REPEAT."""
+    rng = np.random.default_rng(28)
+    W = 1152
+    tau = np.float32(0.01)
+    noisy = lambda c, n: (np.float64(c) + rng.uniform(-0.005, 0.005, n)).astype(np.float32)
+    flat = noisy(5.0, W)
+    steps = np.concatenate([noisy(10.0, 576), noisy(20.0, 576)])          # 576 = 16 * 36
+    off = np.concatenate([noisy(10.0, 500), noisy(20.0, 652)])            # 500 is not a multiple of 36
+    x = np.stack([flat, steps, off])[None]
+    b0 = orc.deepcam_encode(x)
+    b1 = orc.deepcam_encode(x, repeat_tol=np.float32([tau]))
+    h0, h1 = fmt.deepcam_header(b0), fmt.deepcam_header(b1)
+    assert all(s["kind"] == 1 for s in fmt.deepcam_line(b0, h0, 0)["segs"])     # tau = 0: no identical run
+    l0 = fmt.deepcam_line(b1, h1, 0)
+    assert l0["nseg"] == 1 and l0["segs"][0]["kind"] == 0 and l0["segs"][0]["head"] == flat[0]
+    l1 = fmt.deepcam_line(b1, h1, 1)
+    assert [(s["len"], s["kind"]) for s in l1["segs"]] == [(576, 0), (576, 0)]
+    assert l1["segs"][1]["head"] == steps[576]
+    l2 = fmt.deepcam_line(b1, h1, 2)
+    assert (l2["segs"][0]["len"], l2["segs"][0]["kind"]) == (468, 0)        # floor(500 / 36) * 36
+    for l in range(3):
+        _repeat_bound_ok(x[0, l], orc.deepcam_decode_line(b1, l, W), fmt.deepcam_line(b1, h1, l)["segs"], float(tau))
+    assert b1.size < b0.size
+
+
+def test_deepcam_repeat_tolerance_zero_is_default_and_bound(orc):
+    """tau = eps = 0 on every channel writes the default stream byte for byte;
+    with per-channel tau > 0 every REPEAT value is within its channel's tau and
+    every DIFF value obeys the S19 bound (checked exactly)."""
+    from synth import deepcam_stats, gen_deepcam
+    x = gen_deepcam(2005, H=12, W=288)
+    C, H, W = x.shape
+    b0 = orc.deepcam_encode(x)
+    z = np.zeros(C, np.float32)
+    assert np.array_equal(orc.deepcam_encode(x, repeat_tol=z, max_abs_err=z), b0)
+    _, rstd = deepcam_stats(x)
+    tau = (0.05 / rstd).astype(np.float32)
+    b = orc.deepcam_encode(x, repeat_tol=tau)
+    h = fmt.deepcam_header(b)
+    nrep = 0
+    for l in range(C * H):
+        c, y = divmod(l, H)
+        info = fmt.deepcam_line(b, h, l)
+        xh = orc.deepcam_decode_line(b, l, W)
+        if info["mode"] == 0:
+            assert np.array_equal(xh.view(np.uint32), x[c, y].view(np.uint32))
+            continue
+        nrep += sum(s["kind"] == 0 for s in info["segs"])
+        _repeat_bound_ok(x[c, y], xh, info["segs"], float(tau[c]))
+    assert nrep > 0 and b.size < b0.size
+
+
+@pytest.mark.parametrize("raw16,rawseg", [(False, False), (True, False), (False, True)])
+def test_deepcam_absolute_bound(orc, raw16, rawseg):
+    """max_abs_err: exactly the lines whose default SEG encoding has a value with
+    |x̂ - x| > eps_c (counted with numpy on the oracle's decode) are kept
+    uncompressed (RAW, RAW16 when its binary16 values are within both bounds,
+    or RAW segments), every other line is untouched, and every decoded value of
+    the final stream is within eps_c (exact, binary64)."""
+    from synth import deepcam_stats, gen_deepcam
+    x = gen_deepcam(2006, H=16, W=288)
+    C, H, W = x.shape
+    _, rstd = deepcam_stats(x)
+    eps = (0.002 / rstd).astype(np.float32)
+    eps[3] = 0.0                                                # a channel without a bound
+    b0 = orc.deepcam_encode(x)
+    b1 = orc.deepcam_encode(x, max_abs_err=eps, raw16=raw16, raw_segments=rawseg)
+    h0, h1 = fmt.deepcam_header(b0), fmt.deepcam_header(b1)
+    x64 = x.astype(np.float64)
+    switched = 0
+    for l in range(C * H):
+        c, y = divmod(l, H)
+        i0, i1 = fmt.deepcam_line(b0, h0, l), fmt.deepcam_line(b1, h1, l)
+        xh0 = orc.deepcam_decode_line(b0, l, W).astype(np.float64)
+        over = eps[c] > 0 and bool((np.abs(xh0 - x64[c, y]) > np.float64(eps[c])).any())
+        if i0["mode"] == 1 and over:
+            assert i1["mode"] in ((0, 2, 3) if (raw16 or rawseg) else (0,))
+            if not raw16:
+                assert i1["mode"] != 2
+            if not rawseg:
+                assert i1["mode"] != 3
+            switched += 1
+        else:
+            assert i1 == i0
+        xh1 = orc.deepcam_decode_line(b1, l, W).astype(np.float64)
+        if eps[c] > 0:
+            assert np.all(np.abs(xh1 - x64[c, y]) <= np.float64(eps[c]))
+    assert switched > 0
