@@ -75,6 +75,10 @@ def lib():
         L.orc_deepcam_encode_s.restype = I
         L.orc_deepcam_encode_t.argtypes = [P, I, I, I, I, I, I, C.c_float, I, I, I, P, P, P, SZ, C.POINTER(SZ)]
         L.orc_deepcam_encode_t.restype = I
+        L.orc_label_max_encoded_size.argtypes = [I, I, I]; L.orc_label_max_encoded_size.restype = SZ
+        L.orc_label_encode_mask.argtypes = [P, I, I, P, SZ, C.POINTER(SZ)]; L.orc_label_encode_mask.restype = I
+        L.orc_label_encode_vector.argtypes = [P, I, P, SZ, C.POINTER(SZ)]; L.orc_label_encode_vector.restype = I
+        L.orc_label_decode.argtypes = [P, SZ, I, I, I, P]; L.orc_label_decode.restype = I
         L.orc_f16_to_f32.argtypes = [C.c_uint16]; L.orc_f16_to_f32.restype = C.c_float
         L.orc_deepcam_align.argtypes = [I]; L.orc_deepcam_align.restype = I
         _lib = L
@@ -188,4 +192,32 @@ def deepcam_decode(stream: np.ndarray, shape, shift=None, scale=None, out: str =
     _check(lib().orc_deepcam_decode(_p(s), s.size, None if sh is None else _p(sh),
                                     None if sc is None else _p(sc), OUT[out], _p(o), Cc, H, W),
            "deepcam_decode")
+    return o
+
+
+# ---------------------------------------------------------------- labels (FORMAT.md 3)
+def label_encode_mask(m: np.ndarray) -> np.ndarray:
+    a = np.ascontiguousarray(m, dtype=np.uint8)
+    assert a.ndim == 2
+    H, W = a.shape
+    cap = lib().orc_label_max_encoded_size(1, H, W)
+    dst = np.zeros(cap, dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(lib().orc_label_encode_mask(_p(a), H, W, _p(dst), cap, C.byref(size)), "label_encode_mask")
+    return dst[: size.value].copy()
+
+
+def label_encode_vector(v: np.ndarray) -> np.ndarray:
+    a = np.ascontiguousarray(v, dtype=np.float32).ravel()
+    cap = lib().orc_label_max_encoded_size(2, 1, a.size)
+    dst = np.zeros(cap, dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(lib().orc_label_encode_vector(_p(a), a.size, _p(dst), cap, C.byref(size)), "label_encode_vector")
+    return dst[: size.value].copy()
+
+
+def label_decode(stream: np.ndarray, kind: int, H: int, W: int) -> np.ndarray:
+    s = np.ascontiguousarray(stream, dtype=np.uint8)
+    o = np.empty((H, W), dtype=np.uint8) if kind == 1 else np.empty(W, dtype=np.float32)
+    _check(lib().orc_label_decode(_p(s), s.size, int(kind), int(H), int(W), _p(o)), "label_decode")
     return o

@@ -911,6 +911,118 @@ int orc_deepcam_encode_t(const float *x, int C, int H, int W, int A, int lookahe
     return rc;
 }
 
+/* ---------------- labels (FORMAT.md 3; "lossless compression of the labels") */
+/* Plain definitions: a mask row is coded as its maximal runs of equal values
+ * (or verbatim when that is not smaller); decoding is the identity. */
+size_t orc_label_max_encoded_size(int kind, int H, int W) {
+    if (W < 1 || H < 1) return 0;
+    if (kind == 2) return (size_t)up16(32 + 4 * (uint64_t)W);
+    return (size_t)(32 + up16(4 * ((uint64_t)H + 1)) + (uint64_t)H * up16(16 + (uint64_t)W));
+}
+
+int orc_label_encode_mask(const uint8_t *m, int H, int W, uint8_t *dst, size_t cap, size_t *size) {
+    if (!m || !size || H < 1 || W < 1 || H > 65535 || W > 65535) return ORC_EINVAL;
+    uint64_t P = 32 + up16(4 * ((uint64_t)H + 1));
+    /* pass 1: row sizes */
+    uint64_t pay = 0;
+    for (int y = 0; y < H; y++) {
+        const uint8_t *r = m + (uint64_t)y * W;
+        uint64_t nrun = 1;
+        for (int x = 1; x < W; x++) if (r[x] != r[x - 1]) nrun++;
+        uint64_t run_size = up16(4 + 3 * nrun), raw_size = up16(16 + (uint64_t)W);
+        pay += run_size < raw_size ? run_size : raw_size;
+    }
+    uint64_t total = P + pay;
+    *size = (size_t)total;
+    if (total - P > 0xFFFFFFFFull) return ORC_EINVAL;
+    if (!dst || cap < total) return ORC_ESMALL;
+    memset(dst, 0, (size_t)total);
+    wr32(dst, 0x4C505053u); wr16(dst + 4, 1); wr16(dst + 6, 1);
+    wr16(dst + 8, (uint16_t)H); wr16(dst + 10, (uint16_t)W); wr64(dst + 16, total);
+    uint64_t cur = 0;
+    for (int y = 0; y < H; y++) {
+        wr32(dst + 32 + 4 * (uint64_t)y, (uint32_t)cur);
+        const uint8_t *r = m + (uint64_t)y * W;
+        uint8_t *p = dst + P + cur;
+        uint64_t nrun = 1;
+        for (int x = 1; x < W; x++) if (r[x] != r[x - 1]) nrun++;
+        uint64_t run_size = up16(4 + 3 * nrun), raw_size = up16(16 + (uint64_t)W);
+        if (run_size < raw_size) {
+            p[0] = 1; wr16(p + 2, (uint16_t)nrun);
+            int k = 0, start = 0;
+            for (int x = 1; x <= W; x++) {
+                if (x == W || r[x] != r[x - 1]) {          /* run [start, x) ends */
+                    wr16(p + 4 + 2 * (uint64_t)k, (uint16_t)(x - start));
+                    p[4 + 2 * nrun + (uint64_t)k] = r[start];
+                    k++;
+                    start = x;
+                }
+            }
+            cur += run_size;
+        } else {
+            p[0] = 0;
+            memcpy(p + 16, r, (size_t)W);
+            cur += raw_size;
+        }
+    }
+    wr32(dst + 32 + 4 * (uint64_t)H, (uint32_t)cur);
+    return ORC_OK;
+}
+
+int orc_label_encode_vector(const float *v, int n, uint8_t *dst, size_t cap, size_t *size) {
+    if (!v || !size || n < 1 || n > 65535) return ORC_EINVAL;
+    uint64_t total = up16(32 + 4 * (uint64_t)n);
+    *size = (size_t)total;
+    if (!dst || cap < total) return ORC_ESMALL;
+    memset(dst, 0, (size_t)total);
+    wr32(dst, 0x4C505053u); wr16(dst + 4, 1); wr16(dst + 6, 2);
+    wr16(dst + 8, 1); wr16(dst + 10, (uint16_t)n); wr64(dst + 16, total);
+    for (int i = 0; i < n; i++) wr32(dst + 32 + 4 * (uint64_t)i, bits_of_f32(v[i]));
+    return ORC_OK;
+}
+
+/* Sequential decoder of one label stream: kind 1 -> u8 [H][W], kind 2 -> f32 [W]. */
+int orc_label_decode(const uint8_t *src, size_t size, int kind, int H, int W, void *out) {
+    if (!src || !out || size < 32 || rd32(src) != 0x4C505053u || rd16(src + 4) != 1) return ORC_ECORRUPT;
+    if (rd16(src + 6) != kind || rd16(src + 8) != H || rd16(src + 10) != W || H < 1 || W < 1) return ORC_ECORRUPT;
+    uint64_t total = rd64(src + 16);
+    if (total > size || (total & 15)) return ORC_ECORRUPT;
+    if (kind == 2) {
+        if (H != 1 || total < 32 + 4 * (uint64_t)W) return ORC_ECORRUPT;
+        for (int i = 0; i < W; i++) ((float *)out)[i] = f32_of_bits(rd32(src + 32 + 4 * (uint64_t)i));
+        return ORC_OK;
+    }
+    if (kind != 1) return ORC_ECORRUPT;
+    uint64_t P = 32 + up16(4 * ((uint64_t)H + 1));
+    if (P > total) return ORC_ECORRUPT;
+    uint8_t *m = (uint8_t *)out;
+    for (int y = 0; y < H; y++) {
+        uint32_t a = rd32(src + 32 + 4 * (uint64_t)y), b = rd32(src + 32 + 4 * (uint64_t)y + 4);
+        if (b < a || (a & 15) || (b & 15) || b > total - P || b - a < 16) return ORC_ECORRUPT;
+        const uint8_t *p = src + P + a;
+        uint64_t len = b - a;
+        uint8_t *r = m + (uint64_t)y * W;
+        if (p[0] == 0) {
+            if (16 + (uint64_t)W > len) return ORC_ECORRUPT;
+            memcpy(r, p + 16, (size_t)W);
+        } else if (p[0] == 1) {
+            uint64_t nrun = rd16(p + 2);
+            if (nrun < 1 || nrun > (uint64_t)W || 4 + 3 * nrun > len) return ORC_ECORRUPT;
+            uint64_t x = 0;
+            for (uint64_t k = 0; k < nrun; k++) {
+                uint64_t l = rd16(p + 4 + 2 * k);
+                if (l < 1 || x + l > (uint64_t)W) return ORC_ECORRUPT;
+                for (uint64_t j = 0; j < l; j++) r[x + j] = p[4 + 2 * nrun + k];
+                x += l;
+            }
+            if (x != (uint64_t)W) return ORC_ECORRUPT;
+        } else {
+            return ORC_ECORRUPT;
+        }
+    }
+    return ORC_OK;
+}
+
 /* ---------------- array helpers for the Python tests ---------------------- */
 void orc_f32_to_f16_array(const float *in, int64_t n, uint16_t *out) {
     for (int64_t i = 0; i < n; i++) out[i] = orc_f32_to_f16(in[i]);

@@ -22,7 +22,7 @@ import numpy as np
 from scipy import special
 
 __all__ = ["gen_cosmo", "gen_deepcam", "COSMO_PRESETS", "DEEPCAM_CHANNELS",
-           "deepcam_stats"]
+           "deepcam_stats", "gen_deepcam_labels", "gen_cosmo_labels"]
 
 # name -> (lam, sigma, rho_c); paper = calibrated to P:98 (|U|~558, G~36,944)
 COSMO_PRESETS = {
@@ -169,3 +169,37 @@ def deepcam_stats(x: np.ndarray):
     std = m.std(axis=1)
     std[std == 0] = 1.0
     return mean.astype(np.float32), (1.0 / std).astype(np.float32)
+
+
+def gen_deepcam_labels(seed: int, H: int = 768, W: int = 1152) -> np.ndarray:
+    """uint8 [H, W] per-pixel class mask shaped like DeepCAM's segmentation
+    labels (PAPER.md P:56 semantic segmentation of extreme weather; classes as
+    in the MLPerf DeepCAM dataset: 0 background, 1 tropical cyclone, 2
+    atmospheric river): a few cyclone discs and a few long, thin, meandering
+    river bands on a background that covers most of the image."""
+    rng = np.random.default_rng(seed)
+    yy, xx = np.mgrid[0:H, 0:W].astype(np.float64)
+    m = np.zeros((H, W), dtype=np.uint8)
+    for _ in range(int(rng.integers(1, 4))):                   # atmospheric rivers
+        x0, x1 = np.sort(rng.uniform(0, W, 2))
+        x1 = max(x1, x0 + 0.2 * W)
+        y0 = rng.uniform(0.1, 0.9) * H
+        amp, lam, ph = rng.uniform(0.02, 0.1) * H, rng.uniform(0.2, 0.6) * W, rng.uniform(0, 2 * np.pi)
+        slope = rng.uniform(-0.3, 0.3)
+        thick = rng.uniform(0.008, 0.025) * H
+        yc = y0 + slope * (xx - x0) + amp * np.sin(2 * np.pi * xx / lam + ph)
+        m[(np.abs(yy - yc) < thick) & (xx >= x0) & (xx < x1)] = 2
+    for _ in range(int(rng.integers(1, 6))):                   # tropical cyclones
+        cy, cx = rng.uniform(0.1, 0.9) * H, rng.uniform(0, W)
+        r = rng.uniform(0.01, 0.025) * H
+        m[np.hypot(yy - cy, xx - cx) < r] = 1
+    return m
+
+
+def gen_cosmo_labels(seed: int) -> np.ndarray:
+    """fp32 [4]: the four cosmological parameters a CosmoFlow sample is
+    labelled with, drawn uniformly from plausible ranges."""
+    rng = np.random.default_rng(seed)
+    lo = np.array([0.25, 0.70, 0.90, 0.60])
+    hi = np.array([0.35, 0.90, 1.00, 0.80])
+    return (lo + (hi - lo) * rng.random(4)).astype(np.float32)

@@ -101,3 +101,25 @@ def build_deepcam_stream(C, H, W, lines, A=1):
     for ln in lines:
         body += ln
     return np.frombuffer(bytes(body), dtype=np.uint8).copy()
+
+
+def label_header(b: np.ndarray):
+    """FORMAT.md 3 label stream header and (kind 1) row directory."""
+    raw = bytes(b[:32])
+    magic, ver, kind, H, W, _res, total = struct.unpack_from("<IHHHHIQ", raw, 0)
+    d = dict(magic=magic, ver=ver, kind=kind, H=H, W=W, total=total)
+    if kind == 1:
+        d["dir"] = np.frombuffer(bytes(b[32:32 + 4 * (H + 1)]), dtype="<u4")
+        d["payload_off"] = 32 + ((4 * (H + 1) + 15) // 16) * 16
+    return d
+
+
+def label_row(b, hdr, y):
+    a, e = int(hdr["dir"][y]), int(hdr["dir"][y + 1])
+    p = bytes(b[hdr["payload_off"] + a: hdr["payload_off"] + e])
+    if p[0] == 0:
+        return dict(mode=0, size=len(p))
+    nrun = struct.unpack_from("<H", p, 2)[0]
+    lens = np.frombuffer(p[4:4 + 2 * nrun], dtype="<u2")
+    vals = np.frombuffer(p[4 + 2 * nrun:4 + 3 * nrun], dtype=np.uint8)
+    return dict(mode=1, size=len(p), nrun=nrun, lens=lens, vals=vals)

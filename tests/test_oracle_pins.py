@@ -909,3 +909,71 @@ def test_deepcam_absolute_bound(orc, raw16, rawseg):
         if eps[c] > 0:
             assert np.all(np.abs(xh1 - x64[c, y]) <= np.float64(eps[c]))
     assert switched > 0
+
+
+# --------------------------------------------------------------------------
+# Labels (FORMAT.md 3): lossless coding.  Pinned by the identity
+# (decode(encode(m)) == m) and by brute-force run-length sets from numpy.
+
+def _runs(row):
+    """maximal runs of equal values (numpy brute force)"""
+    cut = np.flatnonzero(np.diff(row.astype(np.int16))) + 1
+    starts = np.concatenate([[0], cut])
+    ends = np.concatenate([cut, [row.size]])
+    return (ends - starts), row[starts]
+
+
+def _masks():
+    from synth import gen_deepcam_labels
+    rng = np.random.default_rng(31)
+    alt = np.zeros((2, 64), np.uint8)
+    alt[:, 1::2] = 1
+    one_change = np.zeros((3, 1152), np.uint8)
+    one_change[:, 700:] = 255
+    return [gen_deepcam_labels(1), gen_deepcam_labels(2, H=64, W=256),
+            rng.integers(0, 256, (5, 37), dtype=np.uint8), np.zeros((4, 9), np.uint8),
+            np.full((1, 1), 7, np.uint8), alt, one_change, rng.integers(0, 3, (6, 7), dtype=np.uint8)]
+
+
+@pytest.mark.parametrize("mi", range(8))
+def test_label_mask_lossless_and_layout(orc, mi):
+    m = _masks()[mi]
+    H, W = m.shape
+    b = orc.label_encode_mask(m)
+    assert np.array_equal(orc.label_decode(b, 1, H, W), m)                 # lossless (P:175)
+    h = fmt.label_header(b)
+    assert (h["magic"], h["ver"], h["kind"], h["H"], h["W"]) == (0x4C505053, 1, 1, H, W)
+    assert h["total"] == b.size and b.size % 16 == 0
+    up16 = lambda v: (v + 15) // 16 * 16
+    for y in range(H):
+        lens, vals = _runs(m[y])
+        r = fmt.label_row(b, h, y)
+        run_size, raw_size = up16(4 + 3 * lens.size), up16(16 + W)
+        assert r["mode"] == (1 if run_size < raw_size else 0)
+        assert r["size"] == min(run_size, raw_size)
+        if r["mode"] == 1:
+            assert r["nrun"] == lens.size and np.array_equal(r["lens"], lens) and np.array_equal(r["vals"], vals)
+
+
+def test_label_vector_bitexact(orc):
+    v = np.float32([0.3, -0.0, np.inf, 1e-42, -7.5])
+    v = np.concatenate([v, np.frombuffer(np.uint32([0x7FC12345]).tobytes(), np.float32)])   # NaN payload
+    b = orc.label_encode_vector(v)
+    h = fmt.label_header(b)
+    assert (h["kind"], h["H"], h["W"], h["total"]) == (2, 1, v.size, 32 + 32)
+    assert np.array_equal(orc.label_decode(b, 2, 1, v.size).view(np.uint32), v.view(np.uint32))
+
+
+def test_label_decoder_rejects_corruption(orc):
+    m = _masks()[1]
+    b = orc.label_encode_mask(m)
+    h = fmt.label_header(b)
+    bad = [b.copy() for _ in range(4)]
+    bad[0][0] ^= 1                                                  # magic
+    bad[1][6] = 2                                                   # kind
+    row = h["payload_off"] + int(h["dir"][0])
+    bad[2][row + 4] ^= 0x7F                                          # first run length: sum != W
+    bad[3][row] = 5                                                 # unknown row mode
+    for c in bad:
+        with pytest.raises(RuntimeError):
+            orc.label_decode(c, 1, *m.shape)
