@@ -253,6 +253,37 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
 /* Number of decode launches and copies the last spp_decode_host call enqueued. */
 int spp_pipeline_last_launches(const spp_pipeline *p);
 
+/* ------------------------------------------------------------------------ */
+/* Labels: lossless label coding (FORMAT.md 3; "For both
+ * applications, we use lossless compression of the labels").  DeepCAM labels
+ * are per-pixel class masks (P:56 semantic segmentation), coded per row as
+ * maximal runs of one class or verbatim; CosmoFlow labels are the four
+ * cosmological parameters, kept as binary32.  One label stream per
+ * sample, independent of the sample stream. */
+typedef enum { SPP_LABEL_MASK = 1, SPP_LABEL_VECTOR = 2 } spp_label_kind;
+
+/* Upper bound of an encoded label stream: kind MASK, H x W; kind VECTOR, W values (H = 1). */
+size_t spp_label_max_encoded_size(int kind, int H, int W);
+
+/* mask: host u8 [H][W] row-major class values (any 0..255).  Lossless;
+ * deterministic.  H, W in 1..65535.  dst/dst_capacity/encoded_size as the
+ * sample encoders (SPP_ERR_BUFFER_TOO_SMALL reports the required size). */
+spp_status spp_encode_label_mask(const uint8_t *mask, int H, int W, void *dst, size_t dst_capacity,
+                                 size_t *encoded_size);
+
+/* v: host fp32 [n], n in 1..65535, stored verbatim (bit-exact, NaN payloads included). */
+spp_status spp_encode_label_vector(const float *v, int n, void *dst, size_t dst_capacity, size_t *encoded_size);
+
+/* Decode n label streams resident in HBM (one kernel launch on `stream`):
+ *   kind      : SPP_LABEL_MASK -> d_dst u8 [n][H][W]; SPP_LABEL_VECTOR -> d_dst fp32 [n][W] (H must be 1)
+ *   d_src     : DEVICE array of n DEVICE pointers, each 16-B aligned
+ *   src_bytes : optional device u64[n] bounding each stream's reads (NULL = trust the header)
+ *   status    : optional device word, as spp_decode_opts.status (a stream whose header does not match
+ *               kind/H/W, or a malformed row, sets SPP_ERR_CORRUPT | sample << 8)
+ * Host-checkable errors (n < 0, null pointers, bad kind/dims) return SPP_ERR_INVALID_ARG. */
+spp_status spp_decode_labels(int kind, const void *const *d_src, const uint64_t *src_bytes, int n, void *d_dst,
+                             int H, int W, uint32_t *status, spp_stream_t stream);
+
 const char *spp_status_string(spp_status s);
 
 /* Library build identification: "spp <version> sm_100a". */

@@ -13,7 +13,7 @@ from . import spp
 from .spp import (FMT, OUT, SppError, spp_decode_batch, spp_decode_host, spp_decode_opts_init,
                   spp_encode_cosmo, spp_encode_deepcam, spp_stream_info, spp_version)
 
-__all__ = ["spp", "Decoder", "HostPipeline", "SppError", "spp_encode_cosmo", "spp_encode_deepcam",
+__all__ = ["spp", "Decoder", "HostPipeline", "LabelDecoder", "SppError", "spp_encode_cosmo", "spp_encode_deepcam",
            "spp_decode_batch", "spp_decode_host", "spp_decode_opts_init", "spp_stream_info", "spp_version",
            "sample_shape"]
 
@@ -105,6 +105,48 @@ class Decoder:
         if v:
             self.status.zero_()
             raise SppError(v & 0xFF, f"sample {v >> 8}")
+
+
+class LabelDecoder:
+    """Device-resident batch decode of label streams through ``spp_decode_labels``
+    (FORMAT.md 3; PAPER.md P:175 lossless labels).  kind "mask": dims (H, W),
+    output u8 [n, H, W]; kind "vector": dims (W,), output fp32 [n, W]."""
+
+    def __init__(self, kind: str, dims, device=None):
+        import torch
+        self.torch = torch
+        spp.load()
+        if kind not in spp.LABEL_KIND:
+            raise ValueError("kind is 'mask' or 'vector'")
+        self.kind = kind
+        self.dims = tuple(int(d) for d in dims)
+        self.H, self.W = (self.dims if kind == "mask" else (1, self.dims[-1]))
+        self.device = torch.device(device or "cuda")
+        self.status = torch.zeros(1, dtype=torch.int32, device=self.device)
+
+    def alloc_out(self, n: int):
+        t = self.torch
+        if self.kind == "mask":
+            return t.empty((n, self.H, self.W), dtype=t.uint8, device=self.device)
+        return t.empty((n, self.W), dtype=t.float32, device=self.device)
+
+    def decode(self, srcs, out=None, n: int | None = None, src_bytes=None, stream=None):
+        t = self.torch
+        ptrs = srcs if isinstance(srcs, t.Tensor) and srcs.dtype == t.int64 else \
+            t.tensor([s.data_ptr() for s in srcs], dtype=t.int64, device=self.device)
+        n = int(ptrs.numel()) if n is None else n
+        if out is None:
+            out = self.alloc_out(n)
+        st = (stream or t.cuda.current_stream()).cuda_stream
+        spp.spp_decode_labels(self.kind, ptrs.data_ptr(), n, out.data_ptr(), self.H, self.W, self.status.data_ptr(),
+                              0 if src_bytes is None else src_bytes.data_ptr(), st)
+        return out
+
+    def check_status(self):
+        v = int(self.status.item()) & 0xFFFFFFFF
+        if v:
+            self.status.zero_()
+            raise SppError(v & 0xFF, f"label sample {v >> 8}")
 
 
 class HostPipeline:

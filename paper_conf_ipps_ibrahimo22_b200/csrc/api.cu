@@ -103,6 +103,16 @@ spp_status spp_decode_batch(spp_format fmt, const void *const *d_src, int n, voi
     return deepcam_decode(d_src, n, d_dst, o, st);
 }
 
+spp_status spp_decode_labels(int kind, const void *const *d_src, const uint64_t *src_bytes, int n, void *d_dst,
+                             int H, int W, uint32_t *status, spp_stream_t stream) {
+    if (n < 0 || (kind != SPP_LABEL_MASK && kind != SPP_LABEL_VECTOR)) return SPP_ERR_INVALID_ARG;
+    if (H < 1 || W < 1 || H > 65535 || W > 65535 || (kind == SPP_LABEL_VECTOR && H != 1)) return SPP_ERR_INVALID_ARG;
+    if (n == 0) return SPP_OK;
+    if (!d_src || !d_dst) return SPP_ERR_INVALID_ARG;
+    if (kind == SPP_LABEL_VECTOR && (reinterpret_cast<uintptr_t>(d_dst) & 3) != 0) return SPP_ERR_INVALID_ARG;
+    return labels_decode(kind, d_src, src_bytes, n, d_dst, H, W, status, reinterpret_cast<cudaStream_t>(stream));
+}
+
 spp_status spp_stream_info(spp_format fmt, const void *src, size_t src_bytes, int64_t info[4]) {
     if (!src || !info) return SPP_ERR_INVALID_ARG;
     const uint8_t *b = static_cast<const uint8_t *>(src);

@@ -1,0 +1,184 @@
+// labels.cu — GPU decode of the lossless label streams (FORMAT.md 3; PAPER.md
+// P:175 "For both applications, we use lossless compression of the labels").
+//
+//   KL  kl_decode_mask  persistent warps, one mask row at a time (rows are
+//                       independent, like DeepCAM data lines): a RUN row's
+//                       run starts (warp scan of the run lengths) are set in a
+//                       per-warp bitmap of 1,024 positions; lane l owns 32
+//                       consecutive positions, so the run of position p is
+//                       (starts before the lane) + popc(bits <= p) - 1, and the
+//                       lane writes its 32 class bytes with two 16-B stores.
+//                       RAW rows are copied with 16-B loads/stores.
+//   KL  kl_decode_vec   one thread per value (CosmoFlow's 4 parameters per
+//                       sample): binary32 copied verbatim.
+// Output: masks u8 [n][H][W]; vectors fp32 [n][W].  Corrupt streams set the
+// status word (first error wins) and never read outside [src, src + total).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "spp_format.h"
+#include "spp_internal.h"
+
+namespace spp {
+namespace {
+
+constexpr uint32_t kLabelMagic = 0x4C505053u;  // "SPPL"
+constexpr int kLabelHeader = 32;
+constexpr int kKlWarps = 8;  // warps per CTA
+
+// header check shared by both kinds: returns total (0 if invalid)
+__device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t limit, uint32_t kind, uint32_t H,
+                                                    uint32_t W) {
+    if (b == nullptr || (reinterpret_cast<uintptr_t>(b) & 15) != 0 || limit < (uint64_t)kLabelHeader) return 0;
+    const uint4 h0 = *reinterpret_cast<const uint4 *>(b);
+    const uint4 h1 = *reinterpret_cast<const uint4 *>(b + 16);
+    const uint64_t total = (uint64_t)h1.y << 32 | h1.x;
+    const bool ok = h0.x == kLabelMagic && (h0.y & 0xFFFFu) == kVersion && (h0.y >> 16) == kind &&
+                    (h0.z & 0xFFFFu) == H && (h0.z >> 16) == W && total <= limit && (total & 15) == 0 &&
+                    total >= (uint64_t)kLabelHeader;
+    return ok ? total : 0;
+}
+
+__global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *const *__restrict__ src,
+                                                                   const uint64_t *__restrict__ src_bytes, int n,
+                                                                   uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
+                                                                   uint32_t *__restrict__ status) {
+    __shared__ uint32_t bitmap[kKlWarps][32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t *bm = bitmap[warp];
+    const uint64_t T = (uint64_t)n * H;
+    const uint64_t NW = (uint64_t)gridDim.x * kKlWarps, gw = (uint64_t)blockIdx.x * kKlWarps + warp;
+    const uint64_t g0 = gw * T / NW, g1 = (gw + 1) * T / NW;
+    const uint64_t P = kLabelHeader + ((4ull * (H + 1) + 15) & ~15ull);
+    int64_t cur_s = -1;
+    const uint8_t *b = nullptr;
+    uint64_t total = 0;
+    const bool vec16 = (W & 15) == 0;  // rows start 16-B aligned in dst
+    for (uint64_t g = g0; g < g1; g++) {
+        const int64_t s = (int64_t)(g / H);
+        const uint32_t y = (uint32_t)(g - (uint64_t)s * H);
+        if (s != cur_s) {
+            cur_s = s;
+            b = static_cast<const uint8_t *>(src[s]);
+            total = label_header_ok(b, src_bytes ? src_bytes[s] : ~0ull, SPP_LABEL_MASK, H, W);
+            if (total && P > total) total = 0;
+            if (!total && lane == 0) report(status, SPP_ERR_CORRUPT, s);
+        }
+        if (!total) continue;
+        const uint32_t *dir = reinterpret_cast<const uint32_t *>(b + kLabelHeader);
+        const uint32_t da = __ldg(dir + y), db = __ldg(dir + y + 1);
+        uint8_t *row = dst + g * (uint64_t)W;
+        bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= total - P && db - da >= 16;
+        const uint8_t *p = b + P + da;
+        const uint64_t bytes = ok ? db - da : 0;
+        const uint32_t mode = ok ? __ldg(p) : 0xFFu;
+        if (ok && mode == 0) {  // verbatim row
+            ok = 16ull + W <= bytes;
+            if (ok) {
+                if (vec16) {
+                    const uint4 *s4 = reinterpret_cast<const uint4 *>(p + 16);
+                    for (uint32_t k = lane; k < W / 16; k += kWarp) reinterpret_cast<uint4 *>(row)[k] = __ldg(s4 + k);
+                } else {
+                    for (uint32_t k = lane; k < W; k += kWarp) row[k] = __ldg(p + 16 + k);
+                }
+            }
+        } else if (ok && mode == 1) {  // maximal runs
+            const uint32_t nrun = __ldg(reinterpret_cast<const uint16_t *>(p + 2));
+            ok = nrun >= 1 && nrun <= W && 4ull + 3ull * nrun <= bytes;
+            const uint16_t *lens = reinterpret_cast<const uint16_t *>(p + 4);
+            const uint8_t *vals = p + 4 + 2 * nrun;
+            // pass 1: validate the run lengths (len >= 1, sum = W)
+            uint32_t carry = 0;
+            bool bad = false;
+            for (uint32_t r0 = 0; ok && r0 < nrun; r0 += kWarp) {
+                const uint32_t r = r0 + lane;
+                const uint32_t len = r < nrun ? __ldg(lens + r) : 0u;
+                bad |= r < nrun && len == 0;
+                carry += __reduce_add_sync(0xffffffffu, len);
+            }
+            ok = ok && !__any_sync(0xffffffffu, bad) && carry == W;
+            // pass 2: 1,024 positions at a time, lane l owns [c0 + 32 l, c0 + 32 l + 32)
+            for (uint32_t c0 = 0; ok && c0 < W; c0 += 32 * kWarp) {
+                bm[lane] = 0;
+                __syncwarp();
+                uint32_t before = 0, run_end = 0;
+                for (uint32_t r0 = 0; r0 < nrun && run_end <= c0 + 32 * kWarp; r0 += kWarp) {
+                    const uint32_t r = r0 + lane;
+                    const uint32_t len = r < nrun ? __ldg(lens + r) : 0u;
+                    const uint32_t incl = warp_incl_scan(len, lane);
+                    const uint32_t st = run_end + incl - len;
+                    if (r < nrun && st >= c0 && st < c0 + 32 * kWarp)
+                        atomicOr(&bm[(st - c0) >> 5], 1u << (st & 31));
+                    before += __popc(__ballot_sync(0xffffffffu, r < nrun && st < c0));
+                    run_end += __shfl_sync(0xffffffffu, incl, 31);
+                }
+                __syncwarp();
+                const uint32_t word = bm[lane];
+                const uint32_t c = __popc(word);
+                const uint32_t base = before + warp_incl_scan(c, lane) - c;  // starts before this lane's positions
+                const uint32_t p0 = c0 + 32 * lane;
+                if (p0 < W) {
+                    uint32_t out[8];
+#pragma unroll
+                    for (int k = 0; k < 8; k++) out[k] = 0;
+#pragma unroll
+                    for (int j = 0; j < 32; j++) {
+                        const uint32_t idx = base + __popc(word & (0xFFFFFFFFu >> (31 - j))) - 1;  // run of p0 + j
+                        const uint32_t v = p0 + j < W ? __ldg(vals + min(idx, nrun - 1)) : 0u;
+                        out[j >> 2] |= v << (8 * (j & 3));
+                    }
+                    if (vec16 && p0 + 32 <= W) {
+                        reinterpret_cast<uint4 *>(row + p0)[0] = make_uint4(out[0], out[1], out[2], out[3]);
+                        reinterpret_cast<uint4 *>(row + p0)[1] = make_uint4(out[4], out[5], out[6], out[7]);
+                    } else {
+                        for (int j = 0; j < 32 && p0 + j < W; j++) row[p0 + j] = (uint8_t)(out[j >> 2] >> (8 * (j & 3)));
+                    }
+                }
+                __syncwarp();
+            }
+        } else {
+            ok = false;
+        }
+        if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, s);
+    }
+}
+
+__global__ void kl_decode_vec(const void *const *__restrict__ src, const uint64_t *__restrict__ src_bytes, int n,
+                              uint32_t W, float *__restrict__ dst, uint32_t *__restrict__ status) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (uint64_t)n * W) return;
+    const uint64_t s = i / W;
+    const uint32_t k = (uint32_t)(i - s * W);
+    const uint8_t *b = static_cast<const uint8_t *>(src[s]);
+    const uint64_t total = label_header_ok(b, src_bytes ? src_bytes[s] : ~0ull, SPP_LABEL_VECTOR, 1, W);
+    if (!total || total < kLabelHeader + 4ull * W) {
+        if (k == 0) report(status, SPP_ERR_CORRUPT, (int64_t)s);
+        return;
+    }
+    dst[i] = __ldg(reinterpret_cast<const float *>(b + kLabelHeader) + k);
+}
+
+}  // namespace
+
+spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src_bytes, int n, void *d_dst,
+                         int H, int W, uint32_t *status, cudaStream_t stream) {
+    DeviceProps dp;
+    spp_status st = current_device_props(&dp);
+    if (st != SPP_OK) return st;
+    if (kind == SPP_LABEL_VECTOR) {
+        const uint64_t total = (uint64_t)n * W;
+        kl_decode_vec<<<(unsigned)((total + 255) / 256), 256, 0, stream>>>(d_src, src_bytes, n, (uint32_t)W,
+                                                                           static_cast<float *>(d_dst), status);
+    } else {
+        const uint64_t rows = (uint64_t)n * H;
+        const uint64_t ctas = std::min<uint64_t>((uint64_t)dp.sms * 8, (rows + kKlWarps - 1) / kKlWarps);
+        kl_decode_mask<<<(unsigned)std::max<uint64_t>(1, ctas), kKlWarps * kWarp, 0, stream>>>(
+            d_src, src_bytes, n, (uint32_t)H, (uint32_t)W, static_cast<uint8_t *>(d_dst), status);
+    }
+    return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
+}
+
+}  // namespace spp

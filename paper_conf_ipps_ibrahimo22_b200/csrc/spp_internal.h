@@ -52,6 +52,10 @@ spp_status set_smem_attr(int smem, const DeviceProps &dp) {
     return SPP_OK;
 }
 
+// Labels (labels.cu, FORMAT.md 3)
+spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src_bytes, int n, void *d_dst, int H,
+                         int W, uint32_t *status, cudaStream_t stream);
+
 inline size_t out_elem_bytes(int out) { return out == SPP_OUT_F32 ? 4 : 2; }
 
 }  // namespace spp

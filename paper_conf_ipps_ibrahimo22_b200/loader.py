@@ -123,6 +123,11 @@ class DecodeLoader:
     depth     : output slots in the ring (>= 2: one in use, one being decoded)
     cuda_graph: capture each slot's decode once and replay it (device source)
     check     : read the device status word every `check` batches (0: at epoch end only)
+    labels    : optional (LabelDecoder, EncodedShard) of the samples' lossless label
+                streams (FORMAT.md 3), the shard HBM-resident (labels are small:
+                ~20 KB per DeepCAM mask, 48 B per CosmoFlow vector); each batch's labels
+                are decoded on the same stream right after its samples and the
+                iterator yields (batch, labels, indices) instead of (batch, indices)
 
     Each complete pass advances the epoch by one (``set_epoch`` overrides it),
     so consecutive passes see different permutations.
@@ -130,7 +135,7 @@ class DecodeLoader:
 
     def __init__(self, decoder: Decoder, shard: EncodedShard, batch_size: int, sampler: EpochSampler,
                  source: str = "device", depth: int = 2, cuda_graph: bool = True, drop_last: bool = True,
-                 chunk: int = 16, check: int = 0):
+                 chunk: int = 16, check: int = 0, labels=None):
         import torch
         self.torch = torch
         if depth < 2:
@@ -154,6 +159,18 @@ class DecodeLoader:
         self.launches = 0       # libspp kernel launches enqueued by this loader
         self.batches_done = 0
         self.pipe = None
+        self.lab = None
+        if labels is not None:
+            ldec, lshard = labels
+            if lshard.device_buf is None or len(lshard) != len(shard):
+                raise ValueError("labels: an HBM-resident shard with one label stream per sample")
+            self.lab = ldec
+            self.lab_shard = lshard
+            self.lab_out = [ldec.alloc_out(self.B) for _ in range(depth)]
+            self.lab_ptr_host = [torch.zeros(self.B, dtype=torch.int64, pin_memory=True) for _ in range(depth)]
+            self.lab_ptr_dev = [torch.zeros(self.B, dtype=torch.int64, device=dev) for _ in range(depth)]
+            self.lab_copied = [torch.cuda.Event() for _ in range(depth)]
+            self.lab_copied_pending = [False] * depth
         if source == "device":
             self.ptr_host = [torch.zeros(self.B, dtype=torch.int64, pin_memory=True) for _ in range(depth)]
             self.ptr_dev = [torch.zeros(self.B, dtype=torch.int64, device=dev) for _ in range(depth)]
@@ -209,7 +226,19 @@ class DecodeLoader:
                 srcs = [self.shard.host_view(int(i)) for i in idx]
                 self.pipe.decode(srcs, self.out[s], stream=self.stream)
                 self.launches += self.pipe.launches()
+            if self.lab is not None:
+                self._decode_labels(s, idx, len(idx))
             self.ready[s].record(self.stream)
+
+    def _decode_labels(self, s: int, idx: np.ndarray, n: int):
+        if self.lab_copied_pending[s]:
+            self.lab_copied[s].synchronize()    # the slot's previous pointer upload has been consumed
+        self.lab_ptr_host[s].numpy()[:n] = self.lab_shard.device_ptrs(idx)
+        self.lab_ptr_dev[s].copy_(self.lab_ptr_host[s], non_blocking=True)
+        self.lab_copied[s].record(self.stream)
+        self.lab_copied_pending[s] = True
+        self.lab.decode(self.lab_ptr_dev[s], out=self.lab_out[s], n=n, stream=self.stream)
+        self.launches += 1
 
     def dec_launches(self) -> int:
         from . import spp
@@ -239,7 +268,11 @@ class DecodeLoader:
             s = k % self.depth
             consumer.wait_event(self.ready[s])
             n = len(self._batches[k])
-            yield (self.out[s] if n == self.B else self.out[s][:n]), self._batches[k]
+            batch = self.out[s] if n == self.B else self.out[s][:n]
+            if self.lab is not None:
+                yield batch, (self.lab_out[s] if n == self.B else self.lab_out[s][:n]), self._batches[k]
+            else:
+                yield batch, self._batches[k]
             # the consumer has enqueued its work on batch k: the slot is free after that work
             consumer = t.cuda.current_stream(self.dec.device)
             self.free[s].record(consumer)
@@ -251,6 +284,8 @@ class DecodeLoader:
                 self._enqueue(k + self.depth)
         self.stream.synchronize()
         self.dec.check_status()
+        if self.lab is not None:
+            self.lab.check_status()
         self.epoch += 1
 
     def close(self):

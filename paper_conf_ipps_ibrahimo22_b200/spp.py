@@ -31,7 +31,10 @@ EXPORTS = (
     "spp_stream_info", "spp_decode_opts_init", "spp_decode_workspace_size", "spp_decoded_sample_bytes",
     "spp_decode_batch", "spp_decode_launches", "spp_pipeline_create", "spp_pipeline_destroy", "spp_decode_host",
     "spp_pipeline_last_launches", "spp_status_string", "spp_version",
+    "spp_label_max_encoded_size", "spp_encode_label_mask", "spp_encode_label_vector", "spp_decode_labels",
 )
+SPP_LABEL_MASK, SPP_LABEL_VECTOR = 1, 2
+LABEL_KIND = {"mask": SPP_LABEL_MASK, "vector": SPP_LABEL_VECTOR}
 
 
 class SppError(RuntimeError):
@@ -88,6 +91,10 @@ def load() -> C.CDLL:
         "spp_decode_host": ([P, P, P, I, P, C.POINTER(spp_decode_opts), P], I),
         "spp_pipeline_last_launches": ([P], I),
         "spp_status_string": ([I], C.c_char_p),
+        "spp_label_max_encoded_size": ([I, I, I], SZ),
+        "spp_encode_label_mask": ([P, I, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_encode_label_vector": ([P, I, P, SZ, C.POINTER(SZ)], I),
+        "spp_decode_labels": ([I, P, P, I, P, I, I, P, P], I),
         "spp_version": ([], C.c_char_p),
     }
     for name, (args, res) in sig.items():
@@ -228,3 +235,38 @@ def spp_decode_host(handle: int, h_ptrs: Sequence[int], sizes: Sequence[int], d_
 
 def spp_pipeline_last_launches(handle: int) -> int:
     return int(load().spp_pipeline_last_launches(handle))
+
+
+# ---------------------------------------------------------------- labels (FORMAT.md 3)
+def spp_label_max_encoded_size(kind: str, H: int, W: int) -> int:
+    return int(load().spp_label_max_encoded_size(LABEL_KIND[kind], H, W))
+
+
+def spp_encode_label_mask(mask: np.ndarray) -> np.ndarray:
+    """u8 [H, W] class mask -> lossless label stream (FORMAT.md 3)."""
+    a = np.ascontiguousarray(mask, dtype=np.uint8)
+    if a.ndim != 2:
+        raise ValueError("mask must be [H, W]")
+    H, W = a.shape
+    dst = np.empty(max(spp_label_max_encoded_size("mask", H, W), 32), dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(load().spp_encode_label_mask(a.ctypes.data, H, W, dst.ctypes.data, dst.size, C.byref(size)),
+           "spp_encode_label_mask")
+    return dst[: size.value].copy()
+
+
+def spp_encode_label_vector(v: np.ndarray) -> np.ndarray:
+    """fp32 [n] -> lossless label stream (FORMAT.md 3, binary32 verbatim)."""
+    a = np.ascontiguousarray(v, dtype=np.float32).ravel()
+    dst = np.empty(max(spp_label_max_encoded_size("vector", 1, a.size), 32), dtype=np.uint8)
+    size = C.c_size_t(0)
+    _check(load().spp_encode_label_vector(a.ctypes.data, a.size, dst.ctypes.data, dst.size, C.byref(size)),
+           "spp_encode_label_vector")
+    return dst[: size.value].copy()
+
+
+def spp_decode_labels(kind: str, d_src_ptrs: int, n: int, d_dst: int, H: int, W: int, status: int = 0,
+                      src_bytes: int = 0, stream: int = 0):
+    """Raw call: device pointer table of n label streams -> u8 [n][H][W] (mask) or fp32 [n][W] (vector)."""
+    _check(load().spp_decode_labels(LABEL_KIND[kind], d_src_ptrs, src_bytes or None, n, d_dst, H, W, status or None,
+                                    stream), "spp_decode_labels")

@@ -1,0 +1,127 @@
+"""GPU decode of the lossless label streams (FORMAT.md 3; "For
+both applications, we use lossless compression of the labels") against the
+identity (the masks / vectors themselves) and the oracle's decoder, bit for
+bit; corrupt streams reported; labels delivered with their samples by the
+loader (the paper's DALI pipeline role)."""
+import struct
+
+import numpy as np
+import pytest
+
+from tests import fmt
+from tests.test_gpu_parity import _to_dev
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_ibrahimo22_b200 import build
+    build.build()
+    return torch.device("cuda:0")
+
+
+def _decode(kind, bufs, dims, src_bytes=False):
+    from paper_conf_ipps_ibrahimo22_b200 import LabelDecoder
+    d = LabelDecoder(kind, dims)
+    srcs = [_to_dev(b) for b in bufs]
+    sb = torch.tensor([b.size for b in bufs], dtype=torch.int64, device="cuda") if src_bytes else None
+    out = d.decode(srcs, src_bytes=sb)
+    torch.cuda.synchronize()
+    return out.cpu().numpy(), int(d.status.item())
+
+
+@pytest.mark.parametrize("H,W", [(768, 1152), (5, 37), (3, 2100), (1, 1), (4, 1024)])
+def test_label_masks_lossless(dev, orc, H, W):
+    """Paper-shaped DeepCAM masks (cyclone discs, river bands), random masks
+    (verbatim rows), constant masks, W not a multiple of 16, W over the 1,024-
+    position chunk; mixed in one batch, bit-exact vs the masks and the oracle."""
+    from synth import gen_deepcam_labels
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(H * 7 + W)
+    masks = [gen_deepcam_labels(5000 + i, H=H, W=W) for i in range(6)]
+    masks += [rng.integers(0, 256, (H, W), dtype=np.uint8), np.full((H, W), 2, np.uint8),
+              (rng.random((H, W)) < 0.5).astype(np.uint8)]
+    bufs = [spp.spp_encode_label_mask(m) for m in masks]
+    for b, m in zip(bufs, masks):
+        assert np.array_equal(orc.label_decode(b, 1, H, W), m)
+    for sb in (False, True):
+        got, st = _decode("mask", bufs, (H, W), src_bytes=sb)
+        assert st == 0
+        assert np.array_equal(got, np.stack(masks))
+
+
+def test_label_vectors_bitexact(dev, orc):
+    from synth import gen_cosmo_labels
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    vs = [gen_cosmo_labels(i) for i in range(63)]
+    vs.append(np.frombuffer(np.uint32([0x7FC12345, 0x80000000, 0x00000001, 0x7F800000]).tobytes(), np.float32))
+    bufs = [spp.spp_encode_label_vector(v) for v in vs]
+    got, st = _decode("vector", bufs, (4,))
+    assert st == 0
+    assert np.array_equal(got.view(np.uint32), np.stack(vs).view(np.uint32))
+    for b, v in zip(bufs, vs):
+        assert np.array_equal(orc.label_decode(b, 2, 1, 4).view(np.uint32), v.view(np.uint32))
+
+
+def test_label_corruption_detected(dev):
+    from synth import gen_deepcam_labels
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    m = gen_deepcam_labels(9, H=32, W=256)
+    good = spp.spp_encode_label_mask(m)
+    h = fmt.label_header(good)
+    row = h["payload_off"] + int(h["dir"][3])
+    bad = [good.copy() for _ in range(5)]
+    bad[0][6] = 2                                           # kind
+    bad[1][10:12] = np.frombuffer(struct.pack("<H", 255), np.uint8)  # W
+    bad[2][row + 4] ^= 0x40                                  # a run length: sum != W
+    bad[3][row] = 7                                         # row mode
+    bad[4] = good[: good.size // 2].copy()                  # truncated (caught by src_bytes)
+    for i, c in enumerate(bad):
+        _, st = _decode("mask", [good, c, good], (32, 256), src_bytes=True)
+        assert st == (3 | (1 << 8)), (i, st)
+
+
+@pytest.mark.parametrize("source", ["device", "host"])
+def test_loader_delivers_labels(dev, orc, source):
+    """DecodeLoader with labels: every batch's decoded samples AND labels match
+    the oracle / the original masks for the sampled indices (DeepCAM masks);
+    CosmoFlow parameter vectors on the host-source path."""
+    from synth import gen_cosmo, gen_cosmo_labels, gen_deepcam, gen_deepcam_labels, deepcam_stats
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, LabelDecoder, spp
+    from paper_conf_ipps_ibrahimo22_b200.loader import DecodeLoader, EncodedShard, EpochSampler
+    if source == "device":
+        xs = [gen_deepcam(2400 + i, H=16) for i in range(6)]
+        ms = [gen_deepcam_labels(2400 + i, H=16) for i in range(6)]
+        bufs = [spp.spp_encode_deepcam(x) for x in xs]
+        mean, rstd = deepcam_stats(xs[0])
+        dec = Decoder("deepcam", xs[0].shape)
+        dec.set_normalisation(mean, rstd)
+        lab = (LabelDecoder("mask", ms[0].shape), EncodedShard([spp.spp_encode_label_mask(m) for m in ms],
+                                                               device_resident=True))
+        want = lambda i: orc.deepcam_decode(bufs[i], xs[0].shape, mean, rstd, "f16")
+    else:
+        xs = [gen_cosmo(2500 + i, n=32) for i in range(6)]
+        ms = [gen_cosmo_labels(2500 + i) for i in range(6)]
+        bufs = [spp.spp_encode_cosmo(x) for x in xs]
+        dec = Decoder("cosmo", xs[0].shape)
+        lab = (LabelDecoder("vector", (4,)), EncodedShard([spp.spp_encode_label_vector(v) for v in ms],
+                                                          device_resident=True))
+        want = lambda i: orc.cosmo_direct(xs[i], 1, "f16")
+    shard = EncodedShard(bufs, device_resident=(source == "device"))
+    loader = DecodeLoader(dec, shard, batch_size=2, sampler=EpochSampler(6, seed=3), source=source, labels=lab)
+    seen = 0
+    for _ in range(2):
+        for batch, labels, idx in loader:
+            got, gl = batch.cpu().numpy(), labels.cpu().numpy()
+            for j, i in enumerate(idx):
+                assert np.array_equal(got[j].view(np.uint16), want(int(i)).view(np.uint16))
+                assert np.array_equal(gl[j].view(np.uint8 if source == "device" else np.uint32),
+                                      ms[int(i)].view(np.uint8 if source == "device" else np.uint32))
+                seen += 1
+    assert seen == 12
+    loader.close()

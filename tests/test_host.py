@@ -142,6 +142,26 @@ def test_deepcam_tolerance_argument_errors(spp):
             assert e.value.code == spp.SPP_ERR_INVALID_ARG
 
 
+def test_label_encoders_match_oracle_bytes(spp, orc):
+    """FORMAT.md 3 (P:175 lossless labels): product label encoders write the
+    oracle's bytes; argument errors."""
+    from synth import gen_cosmo_labels, gen_deepcam_labels
+    rng = np.random.default_rng(8)
+    for m in [gen_deepcam_labels(11), gen_deepcam_labels(12, H=7, W=37), rng.integers(0, 256, (3, 50), dtype=np.uint8),
+              np.zeros((1, 1), np.uint8), (rng.random((9, 64)) < 0.3).astype(np.uint8)]:
+        a, b = spp.spp_encode_label_mask(m), orc.label_encode_mask(m)
+        assert a.size == b.size and np.array_equal(a, b)
+    v = gen_cosmo_labels(3)
+    assert np.array_equal(spp.spp_encode_label_vector(v), orc.label_encode_vector(v))
+    lib = spp.load()
+    size = ctypes.c_size_t(0)
+    m = np.zeros((2, 2), np.uint8)
+    assert lib.spp_encode_label_mask(m.ctypes.data, 0, 2, None, 0, ctypes.byref(size)) == spp.SPP_ERR_INVALID_ARG
+    assert lib.spp_encode_label_mask(m.ctypes.data, 2, 2, None, 0, ctypes.byref(size)) == spp.SPP_ERR_BUFFER_TOO_SMALL
+    assert lib.spp_decode_labels(3, None, None, 1, None, 1, 1, None, None) == spp.SPP_ERR_INVALID_ARG
+    assert lib.spp_decode_labels(2, None, None, 1, None, 2, 4, None, None) == spp.SPP_ERR_INVALID_ARG
+
+
 def test_encoder_argument_errors(spp):
     with pytest.raises(spp.SppError) as e:
         spp.spp_encode_cosmo(-np.ones((4, 2, 2, 2), dtype=np.int16))
