@@ -76,6 +76,9 @@ constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
+#ifndef SPP_KC_FIXUP
+#define SPP_KC_FIXUP 0  // 1: branch-free hot pass + per-lane cold fix-up loop in the expansion
+#endif
 #ifndef SPP_KC_DIAG_NOCOLD
 #define SPP_KC_DIAG_NOCOLD 0
 #endif
@@ -108,16 +111,6 @@ constexpr bool kAllLanesRelease = SPP_KC_ALL_LANES_RELEASE;  // every consumer l
 #endif
 constexpr int kColdSlots = SPP_KC_COLD_SLOTS;             // LUT rows per thread per tile fetched ahead
 constexpr int kColdSlotBytes = (kColdLA + 1) * kConsumers * kColdSlots * 8;
-// Dense slabs (most keys beyond the shared-memory prefix, e.g. C5 lambda >= 16):
-// a slab visit whose first key tile shows many threads with more than
-// kColdSlots cold keys takes up to kMaxColdSlots slots per thread, carved from
-// the end of the hot region (a shorter prefix, but every cold row fetched one
-// tile ahead instead of in place).  SPP_KC_DENSE=0 disables it.
-#ifndef SPP_KC_DENSE
-#define SPP_KC_DENSE 1
-#endif
-constexpr int kMaxColdSlots = SPP_KC_DENSE ? 8 : kColdSlots;
-constexpr uint32_t kDenseSlotBytes = (kColdLA + 1) * kConsumers * 8;  // per slot per thread, both tiles in flight
 constexpr int kSmemBytes = kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes + 2 * kKeyStages * 8;
 
 size_t meta_offset(int n) { return round_up16((size_t)n * kFuStride * sizeof(float)); }
@@ -419,8 +412,7 @@ struct KeyRing {
     uint64_t *full;    // kKeyStages, completed by the TMA transaction count
     uint64_t *empty;   // kKeyStages, one arrival per warp
     uint32_t count;
-    uint32_t cold;     // shared address of the per-thread cold-row slots (this slab visit)
-    uint32_t ncs;      // cold-row slots per thread per tile (this slab visit; kColdSlots or a dense setting)
+    uint32_t cold;     // shared address of the per-thread cold-row slots
 };
 
 __device__ __forceinline__ Keys8 keys_from_smem(const uint8_t *stage, uint32_t kwb) {
@@ -582,7 +574,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
 #pragma unroll
     for (int i = 0; i <= kColdLA; i++) cj[i] = 0u;
     auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k of this thread for tile t
-        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * ring.ncs + k) * 8;
+        return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * kColdSlots + k) * 8;
     };
     auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
@@ -619,8 +611,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
 #endif
             uint32_t m = cold;
 #pragma unroll
-            for (int i = 0; i < kMaxColdSlots; i++) {
-                if (m && (uint32_t)i < ring.ncs) {
+            for (int i = 0; i < kColdSlots; i++) {
+                if (m) {
                     const uint32_t j = __ffs(m) - 1;
                     cp_async8(slot_addr(t, i), sv.lut + 8ull * min(k.get_dyn(j), Gm1));
                     m &= m - 1;
@@ -673,6 +665,33 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 k0 = keys_from_smem(stage, kwb);
             }
             E e[8];
+#if SPP_KC_FIXUP
+            // Hot pass, branch-free: every position reads the prefix (a cold key's
+            // clamped read is replaced below).  Then this lane's cold positions (the
+            // power-law tail: ~1% of voxels on C2) are fixed up one by one, so
+            // the warp runs the cold-entry code once per cold key of its busiest lane
+            // instead of once per position that has a cold key in any lane.
+            uint32_t cm = 0;
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                const uint32_t g = k0.get(j);
+                cm |= (g >= n_hot ? 1u : 0u) << j;
+                e[j] = lds_entry<OUT>(hot_base + min(g, n_hot - 1u) * EB);
+            }
+            for (uint32_t m = cm; m; m &= m - 1) {
+                const uint32_t j = __ffs(m) - 1;
+                const uint32_t g = k0.get_dyn(j);
+                bad |= g > Gm1;
+                const uint32_t si = __popc(cm & ((1u << j) - 1u));  // rank among the tile's cold keys
+                const bool pre = !ESC || kEscPrefetch != 0 || ((cmask >> j) & 1u);  // fetched ahead at classify
+                const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
+                                                                  : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);
+                const E en = make_entry<OUT, true>(lv, fu, bad);
+#pragma unroll
+                for (int jj = 0; jj < 8; jj++)
+                    if ((uint32_t)jj == j) e[jj] = en;
+            }
+#else
 #pragma unroll
             for (int j = 0; j < 8; j++) {
 #if SPP_KC_DIAG_NOCOLD  // timing diagnostic only (wrong output): every key treated as hot
@@ -686,11 +705,12 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     bad |= g > Gm1;
                     const uint32_t si = __popc(cmask & ((1u << j) - 1u));  // rank among the tile's cold keys
                     const bool pre = !ESC || kEscPrefetch != 0 || ((cmask >> j) & 1u);  // fetched ahead at classify
-                    const uint2 lv = pre && si < ring.ncs ? lds_u2(slot_addr(t, si))
+                    const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
                                                                : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);  // rare
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }
             }
+#endif
             store8<OUT>(out_s, N, slab_v0 + q, e);
         }
         __syncwarp();
@@ -770,22 +790,6 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
     }
 }
 
-// number of consumer threads whose predicate is true (named barrier 1 with a
-// popc reduction; all consumer threads take part)
-__device__ __forceinline__ uint32_t bar_red_popc_consumers(bool pred) {
-    uint32_t r;
-    asm volatile(
-        "{\n"
-        ".reg .pred p;\n"
-        "setp.ne.u32 p, %1, 0;\n"
-        "barrier.cta.red.popc.u32 %0, 1, %2, p;\n"
-        "}\n"
-        : "=r"(r)
-        : "r"((uint32_t)pred), "n"(kConsumers)
-        : "memory");
-    return r;
-}
-
 // CTA-wide barrier of the threads that run the item loop: all of them, or the
 // consumer warps only when the producer warp has split off (named barrier 1)
 template <bool SPLIT>
@@ -809,8 +813,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
     uint32_t hot_base = region;
     uint64_t *bars =
         reinterpret_cast<uint64_t *>(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes + kColdSlotBytes);
-    const uint32_t cold_fixed = smem_u32(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes);
-    KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0, cold_fixed, (uint32_t)kColdSlots};
+    KeyRing ring{smem_raw + kHotBytes + kUCap * 4, bars, bars + kKeyStages, 0,
+                 smem_u32(smem_raw + kHotBytes + kUCap * 4 + kKeyStages * kStageBytes)};
     if (VEC && threadIdx.x == 0) {
         for (int i = 0; i < kKeyStages; i++) {
             mbar_init(&ring.full[i], 1);
@@ -885,36 +889,6 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) kc_expand(const void *co
                     // for its resolved keys)
                     const uint32_t rk = ESC && kEscPrefetch == 2 && sv.kw == kEscaped ? kRkBytes : 0u;
                     n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes - rk) / EB), amort);
-                    ring.cold = cold_fixed;
-                    ring.ncs = kColdSlots;
-                    if constexpr (kSplit && SPP_KC_DENSE) {
-                        if (sv.G > n_hot && sv.kw != kEscaped && fu.in_smem) {
-                            // probe: this segment's first key tile (already streamed by the
-                            // producer): how many threads hold more cold keys than kColdSlots
-                            const uint32_t gt = ring.count;
-                            mbar_wait(&ring.full[gt % kKeyStages], (gt / kKeyStages) & 1u);
-                            const uint32_t kwb = (uint32_t)sv.kw;
-                            const uint64_t q = a + 8ull * threadIdx.x;
-                            uint32_t c = 0;
-                            if (q < e) {
-                                const Keys8 k = keys_from_smem(ring.buf + (gt % kKeyStages) * kStageBytes, kwb);
-#pragma unroll
-                                for (int j = 0; j < 8; j++) c += (q + j < e && k.get(j) >= n_hot) ? 1u : 0u;
-                            }
-                            const uint32_t over = bar_red_popc_consumers(c > (uint32_t)kColdSlots);
-                            // slots per thread from the overflow rate at kColdSlots (measured on
-                            // C5 presets: lambda 2 ~0.2%, lambda 16 6-15%, lambda 64 45-65%)
-                            const uint32_t ncs = over * 100u < 1u * kConsumers ? (uint32_t)kColdSlots
-                                                 : over * 100u < 8u * kConsumers ? 4u
-                                                 : over * 100u < 25u * kConsumers ? 6u : 8u;
-                            if (ncs > (uint32_t)kColdSlots) {
-                                const uint32_t slot_bytes = ncs * kDenseSlotBytes;
-                                ring.ncs = ncs;
-                                ring.cold = region + (uint32_t)kRegionBytes - slot_bytes;
-                                n_hot = min(min(sv.G, ((uint32_t)kRegionBytes - fu_bytes - slot_bytes) / EB), amort);
-                            }
-                        }
-                    }
 #pragma unroll 1
                     for (uint32_t g0 = threadIdx.x; g0 < n_hot; g0 += 4 * kLoopThreads) {
                         uint2 lv[4];

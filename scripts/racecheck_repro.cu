@@ -1,0 +1,131 @@
+// racecheck_repro.cu — minimal reproducer for the compute-sanitizer racecheck
+// reports on KD's input ring: a producer refills a shared
+// slot by 1-D TMA after every consumer lane has read it and arrived on the
+// slot's "empty" mbarrier, which the producer waits on (release/acquire).
+// The same protocol is run in variants that add, one at a time, what KD does
+// beyond KC's (racecheck-clean) key ring:
+//   0  one producer thread, blocking try_wait on "empty", no cluster (KC-like)
+//   1  as 0, launched as a cluster of 2 CTAs (KD needs it for st.async)
+//   2  as 1, plus a 16-B st.async record on the slot's "full" barrier (KD's line record)
+//   3  as 2, the producer polls "empty" with test_wait (KD's producer loop)
+// Every variant is correctly ordered by the PTX memory model (mbarrier
+// arrive = release, try_wait/test_wait = acquire; the TMA write is issued after
+// the acquire).  build: nvcc -gencode arch=compute_100a,code=sm_100a -o /tmp/rr scripts/racecheck_repro.cu
+// run:   compute-sanitizer --tool racecheck /tmp/rr <variant>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
+
+constexpr int kSlots = 2, kSlotBytes = 1024, kIters = 64;
+
+__device__ __forceinline__ uint32_t sa(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t c) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sa(b)), "r"(c) : "memory");
+}
+__device__ __forceinline__ void expect_tx(uint64_t *b, uint32_t n) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sa(b)), "r"(n) : "memory");
+}
+__device__ __forceinline__ void arrive(uint64_t *b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sa(b)) : "memory");
+}
+__device__ __forceinline__ void wait(uint64_t *b, uint32_t ph) {
+    asm volatile("{\n.reg .pred p;\nW_%=:\nmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n@!p bra W_%=;\n}\n" ::"r"(
+                     sa(b)),
+                 "r"(ph)
+                 : "memory");
+}
+__device__ __forceinline__ bool test(uint64_t *b, uint32_t ph) {
+    uint32_t r;
+    asm volatile("{\n.reg .pred p;\nmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\nselp.u32 %0, 1, 0, p;\n}\n"
+                 : "=r"(r)
+                 : "r"(sa(b)), "r"(ph)
+                 : "memory");
+    return r;
+}
+__device__ __forceinline__ void tma(void *d, const void *s, uint32_t n, uint64_t *b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(sa(d)),
+                 "l"(s), "r"(n), "r"(sa(b))
+                 : "memory");
+}
+__device__ __forceinline__ void st_async(void *d, uint4 v, uint64_t *b) {
+    asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(sa(d)),
+                 "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(sa(b))
+                 : "memory");
+}
+
+template <int V>
+__global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out) {
+    __shared__ __align__(128) uint8_t slot[kSlots][kSlotBytes];
+    __shared__ __align__(16) uint4 rec[kSlots];
+    __shared__ uint64_t full[kSlots], empty[kSlots];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < kSlots; i++) {
+            mbar_init(&full[i], 1);
+            mbar_init(&empty[i], 32);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (warp == 1) {  // producer: lane 0
+        if (lane != 0) return;
+        for (int i = 0; i < kIters; i++) {
+            const int s = i % kSlots;
+            if (i >= kSlots) {
+                const uint32_t ph = ((i / kSlots) - 1) & 1;
+                if (V >= 3) {
+                    while (!test(&empty[s], ph)) {
+                    }
+                } else {
+                    wait(&empty[s], ph);
+                }
+            }
+            expect_tx(&full[s], kSlotBytes + (V >= 2 ? 16 : 0));
+            if (V >= 2) st_async(&rec[s], make_uint4(i, 0, 0, 0), &full[s]);
+            tma(slot[s], src + (size_t)i * kSlotBytes, kSlotBytes, &full[s]);
+        }
+        return;
+    }
+    uint32_t acc = 0;  // consumer warp
+    for (int i = 0; i < kIters; i++) {
+        const int s = i % kSlots;
+        wait(&full[s], (i / kSlots) & 1);
+        const uint32_t *w = reinterpret_cast<const uint32_t *>(slot[s]);
+        for (int k = lane; k < kSlotBytes / 4; k += 32) acc += w[k];
+        if (V >= 2) acc += rec[s].x;
+        __syncwarp();
+        arrive(&empty[s]);
+    }
+    out[blockIdx.x * 32 + lane] = acc;
+}
+
+int main(int argc, char **argv) {
+    const int v = argc > 1 ? atoi(argv[1]) : 0;
+    uint8_t *src;
+    uint32_t *out;
+    cudaMalloc(&src, (size_t)kIters * kSlotBytes);
+    cudaMemset(src, 1, (size_t)kIters * kSlotBytes);
+    cudaMalloc(&out, 2 * 32 * 4);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2);
+    cfg.blockDim = dim3(64);
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = v >= 1 ? 1 : 0;
+    cudaError_t e = v == 0   ? cudaLaunchKernelEx(&cfg, ring<0>, (const uint8_t *)src, out)
+                    : v == 1 ? cudaLaunchKernelEx(&cfg, ring<1>, (const uint8_t *)src, out)
+                    : v == 2 ? cudaLaunchKernelEx(&cfg, ring<2>, (const uint8_t *)src, out)
+                             : cudaLaunchKernelEx(&cfg, ring<3>, (const uint8_t *)src, out);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    uint32_t h[64];
+    cudaMemcpy(h, out, sizeof(h), cudaMemcpyDeviceToHost);
+    uint64_t sum = 0;
+    for (int i = 0; i < 64; i++) sum += h[i];
+    printf("variant %d: %s, checksum %llu\n", v, cudaGetErrorString(e), (unsigned long long)sum);
+    return e == cudaSuccess ? 0 : 1;
+}
