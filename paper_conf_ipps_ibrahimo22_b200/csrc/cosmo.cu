@@ -76,9 +76,6 @@ constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
-#ifndef SPP_KC_FIXUP
-#define SPP_KC_FIXUP 0  // 1: branch-free hot pass + per-lane cold fix-up loop in the expansion
-#endif
 #ifndef SPP_KC_DIAG_NOCOLD
 #define SPP_KC_DIAG_NOCOLD 0
 #endif
@@ -665,33 +662,6 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 k0 = keys_from_smem(stage, kwb);
             }
             E e[8];
-#if SPP_KC_FIXUP
-            // Hot pass, branch-free: every position reads the prefix (a cold key's
-            // clamped read is replaced below).  Then this lane's cold positions (the
-            // power-law tail: ~1% of voxels on C2) are fixed up one by one, so
-            // the warp runs the cold-entry code once per cold key of its busiest lane
-            // instead of once per position that has a cold key in any lane.
-            uint32_t cm = 0;
-#pragma unroll
-            for (int j = 0; j < 8; j++) {
-                const uint32_t g = k0.get(j);
-                cm |= (g >= n_hot ? 1u : 0u) << j;
-                e[j] = lds_entry<OUT>(hot_base + min(g, n_hot - 1u) * EB);
-            }
-            for (uint32_t m = cm; m; m &= m - 1) {
-                const uint32_t j = __ffs(m) - 1;
-                const uint32_t g = k0.get_dyn(j);
-                bad |= g > Gm1;
-                const uint32_t si = __popc(cm & ((1u << j) - 1u));  // rank among the tile's cold keys
-                const bool pre = !ESC || kEscPrefetch != 0 || ((cmask >> j) & 1u);  // fetched ahead at classify
-                const uint2 lv = pre && si < (uint32_t)kColdSlots ? lds_u2(slot_addr(t, si))
-                                                                  : ld_ro_u2_keep(sv.lut + 8ull * min(g, Gm1), pol);
-                const E en = make_entry<OUT, true>(lv, fu, bad);
-#pragma unroll
-                for (int jj = 0; jj < 8; jj++)
-                    if ((uint32_t)jj == j) e[jj] = en;
-            }
-#else
 #pragma unroll
             for (int j = 0; j < 8; j++) {
 #if SPP_KC_DIAG_NOCOLD  // timing diagnostic only (wrong output): every key treated as hot
@@ -710,7 +680,6 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     e[j] = make_entry<OUT, true>(lv, fu, bad);
                 }
             }
-#endif
             store8<OUT>(out_s, N, slab_v0 + q, e);
         }
         __syncwarp();

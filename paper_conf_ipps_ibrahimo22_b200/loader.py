@@ -43,8 +43,8 @@ class EncodedShard:
         if not buffers:
             raise ValueError("empty shard")
         self.sizes = np.array([int(b.size) for b in buffers], dtype=np.int64)
-        if np.any(self.sizes % 16) or np.any(self.sizes < 64):
-            raise ValueError("encoded samples are whole 16-B multiples of at least 64 bytes")
+        if np.any(self.sizes % 16) or np.any(self.sizes < 32):
+            raise ValueError("encoded streams are whole 16-B multiples of at least 32 bytes")
         slots = (self.sizes + _ALIGN - 1) // _ALIGN * _ALIGN
         self.offsets = np.zeros(len(buffers), dtype=np.int64)
         self.offsets[1:] = np.cumsum(slots)[:-1]

@@ -28,7 +28,14 @@ def run(fmt_name, bufs, dims, shift=None, scale=None, **kw):
 
 
 case = sys.argv[1] if len(sys.argv) > 1 else "deepcam"
-if case == "deepcam":
+if case in ("deepcam_default", "deepcam_bigline"):
+    # racecheck isolation: the default stream (no line longer than one ring slot)
+    # vs a stream with RAW lines (each takes the whole ring)
+    y = gen_deepcam(2001, H=192)
+    mean, rstd = deepcam_stats(y)
+    b = spp.spp_encode_deepcam(y) if case == "deepcam_default" else spp.spp_encode_deepcam(y, err_budget=4)
+    print(case, spp.spp_stream_info("deepcam", b), run("deepcam", [b, b], y.shape, mean, rstd, out="f16"))
+elif case == "deepcam":
     y = gen_deepcam(2001)
     mean, rstd = deepcam_stats(y)
     d = spp.spp_encode_deepcam(y)
