@@ -10,6 +10,7 @@
 //   3  as 2, the producer polls "empty" with test_wait (KD's producer loop)
 //   4  KD's protocol: a producer warp, lane k serving consumer warp k (two)
 //   5  as 4, plus lines that take the whole ring (KD's RAW / oversize lines)
+//   6  as 4 with a blocking try_wait per producer lane instead of test_wait
 // Every variant is correctly ordered by the PTX memory model (mbarrier
 // arrive = release, try_wait/test_wait = acquire; the TMA write is issued after
 // the acquire).  build: nvcc -gencode arch=compute_100a,code=sm_100a -o /tmp/rr scripts/racecheck_repro.cu
@@ -65,6 +66,7 @@ __device__ __forceinline__ void st_async(void *d, uint4 v, uint64_t *b) {
 template <int V>
 __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out) {
     constexpr int NC = V >= 4 ? 2 : 1;  // consumer warps
+    constexpr bool BLOCKING = V == 6;   // V6: V4 with a blocking try_wait per producer lane
     __shared__ __align__(128) uint8_t slot[NC][kSlots][kSlotBytes];
     __shared__ __align__(16) uint4 rec[NC][kSlots];
     __shared__ uint64_t full[NC][kSlots], empty[NC][kSlots];
@@ -78,7 +80,7 @@ __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    auto is_big = [](int i) { return V >= 5 && (i % 4) == 3; };
+    auto is_big = [](int i) { return V == 5 && (i % 4) == 3; };
     if (warp == NC) {  // producer
         if (V < 4) {
             if (lane != 0) return;
@@ -108,7 +110,10 @@ __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out
                 const bool big = is_big(i);
                 bool ready = true;
                 for (int j = 0; j < kSlots; j++)
-                    if ((big || j == s) && ((used >> j) & 1u)) ready = ready && test(&empty[lane][j], (par >> j) & 1u);
+                    if ((big || j == s) && ((used >> j) & 1u)) {
+                        if (BLOCKING) wait(&empty[lane][j], (par >> j) & 1u);
+                        else ready = ready && test(&empty[lane][j], (par >> j) & 1u);
+                    }
                 if (ready) {
                     const uint32_t bytes = big ? kSlots * kSlotBytes : kSlotBytes;
                     expect_tx(&full[lane][s], bytes + 16);
@@ -168,7 +173,8 @@ int main(int argc, char **argv) {
                     : v == 2 ? cudaLaunchKernelEx(&cfg, ring<2>, (const uint8_t *)src, out)
                     : v == 3 ? cudaLaunchKernelEx(&cfg, ring<3>, (const uint8_t *)src, out)
                     : v == 4 ? cudaLaunchKernelEx(&cfg, ring<4>, (const uint8_t *)src, out)
-                             : cudaLaunchKernelEx(&cfg, ring<5>, (const uint8_t *)src, out);
+                    : v == 5 ? cudaLaunchKernelEx(&cfg, ring<5>, (const uint8_t *)src, out)
+                             : cudaLaunchKernelEx(&cfg, ring<6>, (const uint8_t *)src, out);
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     uint32_t h[128];
     cudaMemcpy(h, out, sizeof(h), cudaMemcpyDeviceToHost);
