@@ -43,9 +43,6 @@ __device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes, uint6
     asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes), "l"(pol)
                  : "memory");
 }
-__device__ __forceinline__ void prefetch_l1(const void *p) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
-}
 __device__ __forceinline__ uint2 ld_ro_u2_keep(const void *p, uint64_t pol) {
     uint2 r;
     asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));

@@ -76,9 +76,6 @@ constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
-#ifndef SPP_KC_PF_L1
-#define SPP_KC_PF_L1 0  // 1: L1 prefetch of the LUT rows of cold keys beyond the per-thread slots
-#endif
 #ifndef SPP_KC_DIAG_NOCOLD
 #define SPP_KC_DIAG_NOCOLD 0
 #endif
@@ -618,11 +615,6 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                     m &= m - 1;
                 }
             }
-#if SPP_KC_PF_L1
-            // cold keys beyond the slots (dense slabs): pull their LUT rows into L1
-            // now, so the in-place read at expansion, one tile later, hits L1
-            for (; m; m &= m - 1) prefetch_l1(sv.lut + 8ull * min(k.get_dyn(__ffs(m) - 1), Gm1));
-#endif
         }
         cp_async_commit();
         return cold | escw;

@@ -904,6 +904,9 @@ constexpr int kWsWarps = SPP_KD_WS_WPC + 1;
 #ifndef SPP_KD_PROD_SLEEP_NS
 #define SPP_KD_PROD_SLEEP_NS 100  // producer back-off when no slot was free this round
 #endif
+#ifndef SPP_KD_PROD_SERIAL
+#define SPP_KD_PROD_SERIAL 0
+#endif
 #ifndef SPP_KD_PROD_REACQUIRE
 #define SPP_KD_PROD_REACQUIRE 0  // measured -3% on C4 and racecheck still flags the refills (profiles/r02b)
 #endif
@@ -1010,13 +1013,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             if (active) {
                 const bool big = e_flags & kFlagBig;
                 const bool glob = e_flags & kFlagGlobal;
-                bool ready;
-                if (!big) {
-                    ready = !((used >> s) & 1u) || mbar_test(&empty[s], (par >> s) & 1u);
-                } else {  // an oversize line takes the whole ring: every slot must be free
-                    ready = true;
-                    for (uint32_t i = 0; i < kWsNs; i++)
-                        ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
+                bool ready = false;
+                auto test_slots = [&]() {
+                    if (!big) {
+                        ready = !((used >> s) & 1u) || mbar_test(&empty[s], (par >> s) & 1u);
+                    } else {  // an oversize line takes the whole ring: every slot must be free
+                        ready = true;
+                        for (uint32_t i = 0; i < kWsNs; i++)
+                            ready = ready && (!((used >> i) & 1u) || mbar_test(&empty[i], (par >> i) & 1u));
+                    }
+                };
+                if constexpr (SPP_KD_PROD_SERIAL) {
+                    // one lane at a time: compute-sanitizer's racecheck does not see the
+                    // acquire of an mbarrier test issued by several lanes of a warp on
+                    // different barriers (scripts/racecheck_repro.cu variants 4 vs 3/7)
+                    for (int kk = 0; kk < wpc; kk++)
+                        if (kk == k) test_slots();
+                } else {
+                    test_slots();
                 }
                 if (ready && SPP_KD_PROD_REACQUIRE) {
                     // the phases just found complete by test_wait are taken again with

@@ -11,6 +11,8 @@
 //   4  KD's protocol: a producer warp, lane k serving consumer warp k (two)
 //   5  as 4, plus lines that take the whole ring (KD's RAW / oversize lines)
 //   6  as 4 with a blocking try_wait per producer lane instead of test_wait
+//   7  as 4 with each lane's test_wait issued while it is the only active lane
+//   8  as 4 with one producer WARP per consumer (lane 0 of each producer warp)
 // Every variant is correctly ordered by the PTX memory model (mbarrier
 // arrive = release, try_wait/test_wait = acquire; the TMA write is issued after
 // the acquire).  build: nvcc -gencode arch=compute_100a,code=sm_100a -o /tmp/rr scripts/racecheck_repro.cu
@@ -67,6 +69,7 @@ template <int V>
 __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out) {
     constexpr int NC = V >= 4 ? 2 : 1;  // consumer warps
     constexpr bool BLOCKING = V == 6;   // V6: V4 with a blocking try_wait per producer lane
+    constexpr bool SERIAL = V == 7;     // V7: V4 with the lanes' empty-barrier tests taken one lane at a time
     __shared__ __align__(128) uint8_t slot[NC][kSlots][kSlotBytes];
     __shared__ __align__(16) uint4 rec[NC][kSlots];
     __shared__ uint64_t full[NC][kSlots], empty[NC][kSlots];
@@ -81,6 +84,23 @@ __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out
     }
     __syncthreads();
     auto is_big = [](int i) { return V == 5 && (i % 4) == 3; };
+    if (V == 8 && warp >= NC) {  // one producer warp per consumer, lane 0
+        if (lane != 0) return;
+        const int c = warp - NC;
+        uint32_t used = 0, par = 0;
+        for (int i = 0, s = 0; i < kIters; i++, s = (s + 1) % kSlots) {
+            if ((used >> s) & 1u) {
+                while (!test(&empty[c][s], (par >> s) & 1u)) {
+                }
+            }
+            expect_tx(&full[c][s], kSlotBytes + 16);
+            st_async(&rec[c][s], make_uint4(i, 0, 0, 0), &full[c][s]);
+            tma(slot[c][s], src + (size_t)i * kSlotBytes, kSlotBytes, &full[c][s]);
+            par ^= (1u << s) & used;
+            used |= 1u << s;
+        }
+        return;
+    }
     if (warp == NC) {  // producer
         if (V < 4) {
             if (lane != 0) return;
@@ -111,8 +131,14 @@ __global__ void ring(const uint8_t *__restrict__ src, uint32_t *__restrict__ out
                 bool ready = true;
                 for (int j = 0; j < kSlots; j++)
                     if ((big || j == s) && ((used >> j) & 1u)) {
-                        if (BLOCKING) wait(&empty[lane][j], (par >> j) & 1u);
-                        else ready = ready && test(&empty[lane][j], (par >> j) & 1u);
+                        if (BLOCKING) {
+                            wait(&empty[lane][j], (par >> j) & 1u);
+                        } else if (SERIAL) {
+                            for (int k = 0; k < NC; k++)
+                                if (k == lane) ready = ready && test(&empty[lane][j], (par >> j) & 1u);
+                        } else {
+                            ready = ready && test(&empty[lane][j], (par >> j) & 1u);
+                        }
                     }
                 if (ready) {
                     const uint32_t bytes = big ? kSlots * kSlotBytes : kSlotBytes;
@@ -160,7 +186,7 @@ int main(int argc, char **argv) {
     cudaMemset(out, 0, 2 * 64 * 4);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(2);
-    cfg.blockDim = dim3(v >= 4 ? 96 : 64);
+    cfg.blockDim = dim3(v == 8 ? 128 : (v >= 4 ? 96 : 64));
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 2;
@@ -174,7 +200,9 @@ int main(int argc, char **argv) {
                     : v == 3 ? cudaLaunchKernelEx(&cfg, ring<3>, (const uint8_t *)src, out)
                     : v == 4 ? cudaLaunchKernelEx(&cfg, ring<4>, (const uint8_t *)src, out)
                     : v == 5 ? cudaLaunchKernelEx(&cfg, ring<5>, (const uint8_t *)src, out)
-                             : cudaLaunchKernelEx(&cfg, ring<6>, (const uint8_t *)src, out);
+                    : v == 6 ? cudaLaunchKernelEx(&cfg, ring<6>, (const uint8_t *)src, out)
+                    : v == 7 ? cudaLaunchKernelEx(&cfg, ring<7>, (const uint8_t *)src, out)
+                             : cudaLaunchKernelEx(&cfg, ring<8>, (const uint8_t *)src, out);
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     uint32_t h[128];
     cudaMemcpy(h, out, sizeof(h), cudaMemcpyDeviceToHost);

@@ -769,3 +769,28 @@ def test_host_pipeline_coalesced_runs(dev, fmt_name):
         for j, i in enumerate(order):
             assert torch.equal(out[j].view(torch.int16), ref[i].view(torch.int16)), (max_chunk, j)
         pipe.close()
+
+
+@pytest.mark.parametrize("rs", [False, True])
+def test_deepcam_tolerance_streams(dev, orc, rs):
+    """FORMAT.md 2.8 streams (per-channel REPEAT tolerance and absolute bound,
+    alone and with RAW16 lines / RAW segments): decoded bit-exact on both W = 1152
+    KD instances; every value of a bounded channel within its bound."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    x = gen_deepcam(2013, H=48)
+    mean, rstd = deepcam_stats(x)
+    tau, eps = (0.02 / rstd).astype(np.float32), (0.005 / rstd).astype(np.float32)
+    bufs = [spp.spp_encode_deepcam(x, repeat_tol=tau), spp.spp_encode_deepcam(x, max_abs_err=eps),
+            spp.spp_encode_deepcam(x, repeat_tol=tau, max_abs_err=eps, raw16=True, err_budget=8),
+            spp.spp_encode_deepcam(x, repeat_tol=tau, max_abs_err=eps, raw_segments=True, err_budget=8)]
+    got, st = _decode("deepcam", bufs, x.shape, out="f16", shift=mean, scale=rstd, raw_segments=rs)
+    assert st == 0
+    for g, b in zip(got, bufs):
+        _same_bits(g, _dc_ref(orc, b, x.shape, mean, rstd, "f16"))
+    got, st = _decode("deepcam", bufs, x.shape, out="f32", raw_segments=rs)
+    assert st == 0
+    for k, (g, b) in enumerate(zip(got, bufs)):
+        _same_bits(g, _dc_ref(orc, b, x.shape, None, None, "f32"))
+        if k >= 1:
+            assert np.all(np.abs(g.astype(np.float64) - x) <= eps[:, None, None].astype(np.float64))
