@@ -191,7 +191,9 @@ typedef struct {
                                 (spp_encode_deepcam_ex raw_segments = 1): W = 1152 batches use the
                                 KD instance that decodes them (and FORMAT.md 2.6 RAW16 lines) in one
                                 warp pass.  0 (default): the mode-1 instance, on which those lines
-                                take the general line path (same bits, slower).  Other values -> SPP_ERR_INVALID_ARG. */
+                                take the general line path (same bits, slower).  Other values -> SPP_ERR_INVALID_ARG.
+                                spp_decode_host reads each sample's header flags (FORMAT.md 2.1 bit 0, set
+                                by the encoders when such lines exist) and selects this instance itself. */
 } spp_decode_opts;
 
 /* Fill opts with defaults for fmt and the given dims (out = F16, transform = 1). */

@@ -872,7 +872,7 @@ int orc_deepcam_encode_t(const float *x, int C, int H, int W, int A, int lookahe
     else if (!dst || cap < total) rc = ORC_ESMALL;
     if (rc == ORC_OK) {
         memset(dst, 0, (size_t)total);
-        wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);
+        wr32(dst, 0x44505053u); wr16(dst + 4, 1); wr16(dst + 6, 0);   /* flags: bit 0 set below (FORMAT.md 2.1) */
         wr16(dst + 8, (uint16_t)C); wr16(dst + 10, (uint16_t)H); wr16(dst + 12, (uint16_t)W);
         wr16(dst + 14, (uint16_t)A);
         wr32(dst + 16, (uint32_t)L);
@@ -903,6 +903,7 @@ int orc_deepcam_encode_t(const float *x, int C, int H, int W, int A, int lookahe
                 }
                 memcpy(p + 4 + 8 * (uint64_t)ns, mode == 1 ? c.deltas : c.deltas2, (size_t)(mode == 1 ? c.nd : c.nd2));
             }
+            if (mode == 2 || mode == 3) wr16(dst + 6, 1);     /* an extended line mode is present */
             cur += sz;
         }
         wr32(dst + dir_off + 4 * L, (uint32_t)cur);

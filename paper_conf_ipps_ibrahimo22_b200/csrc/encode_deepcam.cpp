@@ -392,6 +392,9 @@ extern "C" spp_status spp_encode_deepcam_ex(const float *x, int C, int H, int W,
     uint16_t u16;
     u32 = spp::kDeepcamMagic; memcpy(out, &u32, 4);
     u16 = spp::kVersion; memcpy(out + 4, &u16, 2);
+    // flags bit 0 (FORMAT.md 2.1): the stream holds RAW16 / mode-3 lines (2.6 / 2.7)
+    u16 = std::any_of(mode.begin(), mode.end(), [](uint8_t m) { return m == kModeRaw16 || m == kModeSegRaw; }) ? 1 : 0;
+    memcpy(out + 6, &u16, 2);
     u16 = (uint16_t)C; memcpy(out + kC, &u16, 2);
     u16 = (uint16_t)H; memcpy(out + kH, &u16, 2);
     u16 = (uint16_t)W; memcpy(out + kW, &u16, 2);

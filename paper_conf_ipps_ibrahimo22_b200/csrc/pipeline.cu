@@ -166,6 +166,16 @@ spp_status spp_decode_host(spp_pipeline *p, const void *const *h_src, const size
             cudaStreamWaitEvent(st, p->copied[slot], 0) != cudaSuccess)
             return SPP_ERR_CUDA;
         o.src_bytes = ds;
+        // the host holds the headers: a DeepCAM chunk with extended line modes
+        // (header flags bit 0, FORMAT.md 2.1) takes the KD instance that decodes
+        // them in one pass, whatever opts->raw_segments says
+        o.raw_segments = opts->raw_segments;
+        if (p->fmt == SPP_FMT_DEEPCAM && !o.raw_segments)
+            for (int j = 0; j < k; j++) {
+                uint16_t flags;
+                memcpy(&flags, static_cast<const uint8_t *>(h_src[i + j]) + 6, 2);
+                if (flags & 1u) o.raw_segments = 1;
+            }
         spp_status r = spp_decode_batch(p->fmt, dp, k, static_cast<uint8_t *>(d_dst) + (size_t)i * out_bytes, &o,
                                         stream);
         if (r != SPP_OK) return r;

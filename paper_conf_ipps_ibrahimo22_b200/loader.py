@@ -55,6 +55,11 @@ class EncodedShard:
         for i, b in enumerate(buffers):
             o = int(self.offsets[i])
             h[o:o + int(self.sizes[i])] = np.asarray(b, dtype=np.uint8)
+        # DeepCAM streams whose header flags (FORMAT.md 2.1 bit 0) announce RAW16 /
+        # RAW-segment lines: the loader then selects the KD instance that decodes
+        # them in one pass (opts.raw_segments)
+        self.extended_line_modes = any(bytes(np.asarray(b[:4], np.uint8)) == b"SPPD" and int(b[6]) & 1
+                                       for b in buffers)
         self.device_buf = None
         if device_resident:
             self.device_buf = self.host.to(device or "cuda", non_blocking=False)
@@ -147,6 +152,9 @@ class DecodeLoader:
         if sampler.n != len(shard):
             raise ValueError("sampler size != shard size")
         self.dec, self.shard, self.B, self.sampler = decoder, shard, int(batch_size), sampler
+        if decoder.fmt == "deepcam" and shard.extended_line_modes and not decoder.opts.raw_segments:
+            decoder.opts.raw_segments = 1
+            decoder.version += 1
         self.source, self.depth, self.drop_last, self.check = source, depth, drop_last, check
         self.use_graph = cuda_graph and source == "device"
         dev = decoder.device

@@ -222,3 +222,26 @@ def test_loader_graphs_follow_decoder_buffers(dev, orc):
                 got = batch.cpu().numpy()
                 for j, i in enumerate(idx):
                     _same_bits(got[j], orc.deepcam_decode(bufs[int(i)], xs[0].shape, sh, sc, "f16"))
+
+
+def test_host_pipeline_selects_extended_mode_instance(dev, orc):
+    """a stream with RAW-segment / RAW16 lines decoded through
+    spp_decode_host with opts.raw_segments = 0 (the caller forgot the flag): the
+    pipeline reads the header flags (FORMAT.md 2.1 bit 0) and picks the one-pass
+    instance itself; the result is bit-exact either way."""
+    from synth import deepcam_stats, gen_deepcam
+    from paper_conf_ipps_ibrahimo22_b200 import Decoder, HostPipeline, spp
+    xs = [gen_deepcam(2600 + i, H=32) for i in range(3)]
+    bufs = [spp.spp_encode_deepcam(x, err_budget=1, raw_segments=True, raw16=True) for x in xs]
+    assert all(int(b[6]) & 1 for b in bufs)
+    mean, rstd = deepcam_stats(xs[0])
+    dec = Decoder("deepcam", xs[0].shape)            # raw_segments left at 0
+    dec.set_normalisation(mean, rstd)
+    pipe = HostPipeline(dec, slot_bytes=max(b.size for b in bufs) * 2 + 4096, nslots=2, max_chunk=2)
+    out = dec.alloc_out(3)
+    pipe.decode([torch.from_numpy(b).pin_memory() for b in bufs], out)
+    torch.cuda.synchronize()
+    dec.check_status()
+    pipe.close()
+    for g, b in zip(out.cpu().numpy(), bufs):
+        _same_bits(g, _dc_ref(orc, b, xs[0].shape, mean, rstd, "f16"))

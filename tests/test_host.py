@@ -133,6 +133,19 @@ def test_deepcam_tolerances_match_oracle_bytes(spp, orc, knobs):
     assert a.size == b.size and np.array_equal(a, b)
 
 
+def test_deepcam_header_flags_extended_modes(spp, orc):
+    """FORMAT.md 2.1 flags bit 0 is set iff some line is mode 2 (RAW16) or 3 (RAW
+    segments), by both encoders (the hint spp_decode_host / the loader use)."""
+    from synth import gen_deepcam
+    x = gen_deepcam(2009, H=16)
+    for kw in (dict(), dict(err_budget=1), dict(err_budget=1, raw16=True), dict(err_budget=1, raw_segments=True)):
+        for b in (spp.spp_encode_deepcam(x, **kw), orc.deepcam_encode(x, **kw)):
+            h = fmt.deepcam_header(b)
+            modes = {fmt.deepcam_line(b, h, l)["mode"] for l in range(h["L"])}
+            flags = int(b[6]) | (int(b[7]) << 8)
+            assert flags == (1 if modes & {2, 3} else 0), (kw, modes, flags)
+
+
 def test_deepcam_tolerance_argument_errors(spp):
     x = np.zeros((2, 2, 16), dtype=np.float32)
     for bad in (np.float32([0.1, -1.0]), np.float32([np.inf, 0.0]), np.float32([np.nan, 0.0])):
