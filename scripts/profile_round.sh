@@ -5,7 +5,7 @@
 # Outputs land in gpurun_out/; summarise here with scripts/ncu_summary.py and
 # scripts/launch_summary.py into profiles/.
 set -u
-R=${1:-r01}
+R=${1:-r02}
 mkdir -p gpurun_out
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${R}_launches.csv \
     python bench.py --steps 20 --warmup 3 --e2e-steps 1 --cpu-seconds 1 --secondary none \
