@@ -977,3 +977,125 @@ def test_label_decoder_rejects_corruption(orc):
     for c in bad:
         with pytest.raises(RuntimeError):
             orc.label_decode(c, 1, *m.shape)
+
+
+# --------------------------------------------------------------------------
+# FORMAT.md 2.4 encoder POLICY, characterised independently of the oracle's
+# code: for every segment the oracle wrote, numpy / brute force recompute what
+# 2.4 prescribes (identical runs, the emin rule, the nearest code over all 256
+# bytes, where the segment must end) from the text of FORMAT.md alone.
+
+_MAG = np.array([(b & 15) if (b >> 4) & 7 == 0 else (16 + (b & 15)) << (((b >> 4) & 7) - 1) for b in range(128)],
+                dtype=np.float64)
+
+
+def _nearest_code(t):
+    """2.4: the code value nearest to t, ties toward the smaller magnitude (brute force over all codes)."""
+    vals = np.concatenate([_MAG, -_MAG[1:]])          # every distinct code value
+    d = np.abs(vals - t)
+    best = d.min()
+    cand = vals[d == best]
+    return cand[np.argmin(np.abs(cand))]
+
+
+def _policy_check_line(x, A, segs, deltas, lookahead=64, repeat_min=16, stats=None):
+    W = x.size
+    stats = {} if stats is None else stats
+    bits = x.view(np.uint32)
+
+    def rep(i):
+        r = 1
+        while i + r < W and bits[i + r] == bits[i]:
+            r += 1
+        return r if i + r == W else (r // A) * A
+
+    def simulate(i, emin, jmax):
+        """closed loop from head i at emin; returns (positions coded, overflow position or None, codes)"""
+        h = x[i]
+        unit = np.float32(2.0 ** emin)
+        S, prev, codes = 0, h, []
+        for j in range(i + 1, jmax):
+            if j % A == 0 and rep(j) >= repeat_min:
+                return j, None, codes
+            t = (np.float64(x[j]) - np.float64(prev)) / 2.0 ** emin
+            if abs(t) > 1984.5:
+                return j, j, codes
+            k = _nearest_code(t)
+            if abs(S + k) > 1983 * 1984:
+                return j, j, codes
+            S += int(k)
+            prev = np.float32(h + np.float32(S) * unit)      # the product is exact: one rounding
+            codes.append(k)
+        return jmax, None, codes
+
+    pos, dp = 0, 0
+    for s in segs:
+        i, ln = pos, s["len"]
+        assert i % A == 0 and s["head"].view(np.uint32) == bits[i]
+        if rep(i) >= repeat_min:
+            assert s["kind"] == 0 and ln == rep(i)
+        else:
+            assert s["kind"] == 1
+            m = np.max(np.abs(np.diff(x[i:min(i + lookahead, W)].astype(np.float64))), initial=0.0)
+            e0 = -149 if m == 0 else int(min(96, max(-149, np.ceil(np.log2(m / 1984.0)))))
+            if m > 0 and 2.0 ** (e0 - 1) * 1984.0 >= m:           # exact ceil of log2 (no float fuzz)
+                e0 -= 1
+            e = s["emin"]
+            assert e >= e0
+            for e_low in range(e0, e):                            # a lower emin overflows within A positions
+                _, ov, _ = simulate(i, e_low, W)
+                assert ov is not None and (ov // A) * A == i
+            end, ov, codes = simulate(i, e, W)
+            if ov is None:
+                assert ln == end - i                              # stopped at W or at a REPEAT start
+                stats["stop"] = stats.get("stop", 0) + 1
+            else:
+                assert ln == (ov // A) * A - i and ln > 0         # overflow: cut at the aligned position
+                stats["overflow"] = stats.get("overflow", 0) + 1
+            stats["emin_raised"] = stats.get("emin_raised", 0) + (e > e0)
+            got = [(-1 if b & 0x80 else 1) * _MAG[b & 127] for b in deltas[dp:dp + ln - 1]]
+            assert got == [float(c) for c in codes[:ln - 1]]
+            dp += ln - 1
+        pos += ln
+    assert pos == W
+
+
+@pytest.mark.parametrize("W,seed", [(64, 1), (37, 2), (1152, 3), (256, 4)])
+def test_deepcam_encoder_policy_characterisation(orc, W, seed):
+    """Lines with smooth stretches, noise, abrupt jumps (forcing overflow splits
+    and emin increments), identical runs at aligned and unaligned positions,
+    subnormal and huge magnitudes; every SEG line's segmentation, emin and codes
+    match FORMAT.md 2.4 recomputed from scratch."""
+    rng = np.random.default_rng(seed)
+    C, H = 1, 12
+    x = np.empty((C, H, W), np.float32)
+    t = np.linspace(0, 6, W)
+    for y in range(H):
+        base = np.sin(t * (1 + y % 3)) * 10.0 ** (y % 5 - 2) + rng.standard_normal(W) * 10.0 ** (y % 4 - 4)
+        if y % 3 == 0:
+            base[W // 3: W // 3 + 20] = base[W // 3]                # identical run (unaligned start)
+        if y % 4 == 1:
+            base[2 * W // 3:] += 1e4                                 # abrupt jump
+        if y == 7:
+            base = base * 1e-40                                      # subnormal range
+        x[0, y] = base.astype(np.float32)
+    # closed-loop overflow inside the first A positions at the window's emin (Δ = 1950
+    # quantises to 1920, then Δ = 1984 gives t = 2014 > 1984.5): 2.4 raises emin
+    x[0, 2, :] = np.float32(3934 + 1000 * np.arange(W) - 2000)
+    x[0, 2, :3] = np.float32([0, 1950, 3934])
+    A = orc.lib().orc_deepcam_align(W)
+    b = orc.deepcam_encode(x)
+    h = fmt.deepcam_header(b)
+    checked, stats = 0, {}
+    for l in range(C * H):
+        info = fmt.deepcam_line(b, h, l)
+        if info["mode"] != 1:
+            continue
+        _policy_check_line(x[0, l], A, info["segs"], info["delta"], stats=stats)
+        checked += 1
+    assert checked >= H // 2
+    assert stats.get("stop", 0) > 0, stats
+    if A > 1:
+        assert stats.get("emin_raised", 0) > 0, stats               # (with A = 1 2.4 never raises emin)
+    if W >= 256:
+        assert stats.get("overflow", 0) > 0, stats                   # overflow splits exercised
