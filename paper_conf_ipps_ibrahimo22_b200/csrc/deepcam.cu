@@ -124,6 +124,26 @@ __device__ __forceinline__ float code_f_byte(uint32_t b) {
     return __uint_as_float(((b & 0x80u) << 24) | ((b & 0x7Fu) << 19));
 }
 
+// Inclusive warp scans whose shuffle also yields the "source lane in range"
+// predicate (shfl.sync.up's second destination), so each step is SHFL + one
+// predicated add (no separate lane >= d compare / select).
+__device__ __forceinline__ uint32_t scan_incl_u32(uint32_t v) {
+#pragma unroll
+    for (int d = 1; d < kWarp; d <<= 1)
+        asm("{\n.reg .u32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, 0, 0xffffffff;\n@p add.u32 %0, %0, t;\n}\n"
+            : "+r"(v)
+            : "r"(d));
+    return v;
+}
+__device__ __forceinline__ float scan_incl_f32(float v) {  // exact here: sums of codes (see callers)
+#pragma unroll
+    for (int d = 1; d < kWarp; d <<= 1)
+        asm("{\n.reg .f32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, 0, 0xffffffff;\n@p add.rn.f32 %0, %0, t;\n}\n"
+            : "+f"(v)
+            : "r"(d));
+    return v;
+}
+
 // per-segment packed info written in place of the descriptor:
 //   bits 0..21  byte base a + 2^21 (DIFF: the delta byte of position p is dl[a + p];
 //               RAW segment: its value is the binary32 at dl + a + 4p), any W <= 65535
@@ -630,11 +650,10 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
 // one bitmap word (one warp OR-reduction) and every lane fetches its segment's
 // parameters by shuffle.  Falls back to the shared-memory tables otherwise.
 template <int OUT, bool RAWSEG>  // RAWSEG: a mode-3 line (FORMAT.md 2.7); mode-1 lines run without its code
-__device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
-                                                    uint32_t nbw, float shv, float scv, uint8_t *row, uint8_t *rowbuf,
-                                                    int lane) {
+__device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t hdr, uint32_t bytes, uint32_t W,
+                                                    uint32_t *bbits, uint32_t nbw, float shv, float scv, uint8_t *row,
+                                                    uint8_t *rowbuf, uint32_t rep_s, int lane) {
     constexpr int VPL = 36;
-    const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
     // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
     // it never has more than 32 segments, so the fallback sees only mode 1
@@ -655,7 +674,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     }
     const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : (kind == kRawSeg ? 4u * len : 0u);
     const uint32_t pk = len | (dlen << 16);
-    const uint32_t inc = warp_incl_scan(pk, lane);
+    const uint32_t inc = scan_incl_u32(pk);
     const uint32_t ex = inc - pk;
     const uint32_t st = ex & 0xFFFFu, db = ex >> 16;
     const uint32_t blk = st / VPL;
@@ -679,12 +698,10 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
     const uint32_t skind = (d >> 22) & 3u, seb = d >> 24;
     const bool raw = RAWSEG && skind == kRawSeg;
     const bool rep = skind == kRepeat || raw;  // RAW lanes run the chain on zero codes, then take their values
+    // a REPEAT / RAW lane reads a constant block of 0x80 bytes (code -0: S = -0
+    // keeps h exact) instead of the delta area: same loads, no selects
     Bytes<VPL> bt;
-    bt.load(dl_s + (uint32_t)(rep ? 0 : a + (int)p0));
-    if (rep) {
-#pragma unroll
-        for (int k = 0; k < VPL / 4; k++) bt.w[k] = 0x80808080u;  // code -0: S = -0 keeps h exact
-    }
+    bt.load(rep ? rep_s : dl_s + (uint32_t)(a + (int)p0));
     if (flag) bt.w[0] = (bt.w[0] & 0xFFFFFF00u) | 0x80u;  // the head has no delta byte
     // codes of the lane's 36 positions as fp16 pairs (value = code * 2^-18),
     // then two exact fp32 prefix chains (positions 0..17 and 18..35) fed by
@@ -704,12 +721,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t bytes
                             fadd_h(hv[(HALF + i) >> 1], (HALF + i) & 1, pp[i - 1].y));
     const float totA = pp[HALF - 1].x;
     const float lt = totA + pp[HALF - 1].y;  // lane total
-    float P = lt;
-#pragma unroll
-    for (int dd = 1; dd < kWarp; dd <<= 1) {
-        const float y = __shfl_up_sync(0xffffffffu, P, dd);
-        if (lane >= dd) P += y;
-    }
+    const float P = scan_incl_f32(lt);        // exact: multiples of 2^-18 far below 2^6
     const float P_excl = P - lt;
     const uint32_t mle = word & le_mask;
     const float base = __shfl_sync(0xffffffffu, P_excl, 31 - __clz(mle));
@@ -937,6 +949,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     const uint32_t ctl_off = (kWsNs * cap + rowb + 4 * nwords + 15u) & ~15u;  // 16-B aligned: info[] is read as uint4
     auto ctl = [&](int w) { return reinterpret_cast<uint64_t *>(smem_raw + (size_t)w * warp_bytes + ctl_off); };
 
+    if (warp == wpc && lane < 12)  // 48 B of 0x80 after the warps' regions: REPEAT lanes' code bytes
+        reinterpret_cast<uint32_t *>(smem_raw + (size_t)wpc * warp_bytes)[lane] = 0x80808080u;
     if (warp == wpc && lane < wpc) {
         uint64_t *c = ctl(lane);
         for (uint32_t i = 0; i < kWsNs; i++) {
@@ -1097,17 +1111,21 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     const uint32_t info_s = smem_u32(full + 2 * kWsNs);
     const uint32_t nbw = (W / VPL + 31) / 32;
     const uint32_t nsb = nwords / 2;  // words of the start bitmap (and of its prefix counts)
+    const uint32_t rep_s = smem_u32(smem_raw + (size_t)wpc * warp_bytes);  // 48 B of 0x80 (producer-filled)
     uint32_t fph = 0;  // bit s: parity of slot s's next full phase
     uint32_t s = 0;
-    for (uint64_t g = g_begin; g < g_end; g++, s = s + 1 == kWsNs ? 0u : s + 1) {
+    const uint32_t nlines = (uint32_t)(g_end - g_begin);  // < 2^32: lines of one warp
+    const uint64_t row_bytes = (uint64_t)W * ob;
+    uint8_t *row = dst + g_begin * row_bytes;
+    for (uint32_t it = 0; it < nlines; it++, row += row_bytes, s = s + 1 == kWsNs ? 0u : s + 1) {
         mbar_wait(&full[s], (fph >> s) & 1u);
         fph ^= 1u << s;
         const uint4 inf = lds_u4(info_s + 16u * s);
         const uint32_t bytes = inf.x, flags = inf.y, al = flags >> 16;
-        uint8_t *row = dst + g * (uint64_t)W * ob;
         if (flags & kFlagGlobal) {
             // record only: release the slot at once, decode the line from HBM
             mbar_arrive(&empty[s]);
+            const uint64_t g = g_begin + it;
             const uint8_t *src = reinterpret_cast<const uint8_t *>((uint64_t)inf.w << 32 | inf.z);
             const uint32_t c = (uint32_t)(g % L) / H;
             const float shv = shift ? __ldg(shift + c) : 0.f, scv = scale ? __ldg(scale + c) : 1.f;
@@ -1118,26 +1136,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
         if (bytes) {
             uint8_t *buf = (flags & kFlagBig) ? base : base + s * cap;
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
+            const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);  // mode (byte 0) and nseg (bytes 2-3)
+            const uint32_t mode = hdr & 0xFFu;
             bool ok;
-            if (RAWSEG && buf[0] == kModeRaw16) {
+            if (RAWSEG && mode == kModeRaw16) {
                 if constexpr (RAWSEG && VPL == 36)
                     ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, rowbuf, lane);
-            } else if (VEC && al == (uint32_t)VPL && (buf[0] == kModeSeg || (RAWSEG && buf[0] == kModeSegRaw))) {
+            } else if (VEC && al == (uint32_t)VPL && (mode == kModeSeg || (RAWSEG && mode == kModeSegRaw))) {
                 if constexpr (VPL == 36) {
-                    if (!RAWSEG || buf[0] == kModeSeg)
-                        ok = decode_line_onepass<OUT, false>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
+                    if (!RAWSEG || mode == kModeSeg)
+                        ok = decode_line_onepass<OUT, false>(buf, hdr, bytes, W, sbits, nbw, shv, scv, row, rowbuf,
+                                                             rep_s, lane);
                     else
-                        ok = decode_line_onepass<OUT, true>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
+                        ok = decode_line_onepass<OUT, true>(buf, hdr, bytes, W, sbits, nbw, shv, scv, row, rowbuf,
+                                                            rep_s, lane);
                 }
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
             } else {
                 ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nsb, shv, scv, row, lane);
             }
-            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / L));
+            if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)((g_begin + it) / L));
         }
         __syncwarp();
         // every lane releases: its own reads of the slot and of info[s] precede its arrival
-        if (flags & kFlagBig) {
+        if (__builtin_expect(flags & kFlagBig, 0)) {
             for (uint32_t i = 0; i < kWsNs; i++) mbar_arrive(&empty[i]);  // the line took the whole ring
         } else {
             mbar_arrive(&empty[s]);
@@ -1169,8 +1191,8 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
     // consumer warps per CTA: as many as fit two CTAs per SM (else one)
     int wpc = SPP_KD_WS_WPC;
     auto fits = [&](int w, int ctas) {
-        return (size_t)w * warp_bytes <= (size_t)dp.smem_optin &&
-               (size_t)ctas * ((size_t)w * warp_bytes + dp.smem_reserved) <= (size_t)dp.smem_per_sm;
+        return (size_t)w * warp_bytes + 64 <= (size_t)dp.smem_optin &&
+               (size_t)ctas * ((size_t)w * warp_bytes + 64 + dp.smem_reserved) <= (size_t)dp.smem_per_sm;
     };
     while (wpc > 1 && !fits(wpc, 2)) wpc--;
     if (!fits(wpc, 2)) {
@@ -1178,7 +1200,7 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
         while (wpc > 1 && !fits(wpc, 1)) wpc--;
     }
     if (!fits(wpc, 1)) return SPP_ERR_UNSUPPORTED;
-    const int smem = wpc * (int)warp_bytes;
+    const int smem = wpc * (int)warp_bytes + 64;  // + the constant REPEAT code block
     auto kern = kd_decode_ws<OUT, VEC, VPL, RAWSEG>;
     if (set_smem_attr<kd_decode_ws<OUT, VEC, VPL, RAWSEG>>(smem, dp) != SPP_OK) return SPP_ERR_CUDA;
     int occ = 0;

@@ -121,14 +121,24 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                 const uint32_t base = before + warp_incl_scan(c, lane) - c;  // starts before this lane's positions
                 const uint32_t p0 = c0 + 32 * lane;
                 if (p0 < W) {
+                    // the run of p0, then one fill per run starting inside the window
+                    // (a mask row has a handful of runs: usually none starts here)
+                    uint32_t idx = base + (word & 1u) - 1;
+                    uint32_t v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
                     uint32_t out[8];
 #pragma unroll
-                    for (int k = 0; k < 8; k++) out[k] = 0;
+                    for (int k = 0; k < 8; k++) out[k] = v;
+                    for (uint32_t w = word & ~1u; w; w &= w - 1) {
+                        const uint32_t j = __ffs(w) - 1;  // a run starts at p0 + j: bytes j.. take its value
+                        idx++;
+                        v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
 #pragma unroll
-                    for (int j = 0; j < 32; j++) {
-                        const uint32_t idx = base + __popc(word & (0xFFFFFFFFu >> (31 - j))) - 1;  // run of p0 + j
-                        const uint32_t v = p0 + j < W ? __ldg(vals + min(idx, nrun - 1)) : 0u;
-                        out[j >> 2] |= v << (8 * (j & 3));
+                        for (int k = 0; k < 8; k++) {
+                            // bytes 4k..4k+3 at or after j
+                            const int sh = (int)j - 4 * k;
+                            const uint32_t m = sh <= 0 ? 0xFFFFFFFFu : (sh >= 4 ? 0u : 0xFFFFFFFFu << (8 * sh));
+                            out[k] = (out[k] & ~m) | (v & m);
+                        }
                     }
                     if (vec16 && p0 + 32 <= W) {
                         reinterpret_cast<uint4 *>(row + p0)[0] = make_uint4(out[0], out[1], out[2], out[3]);
