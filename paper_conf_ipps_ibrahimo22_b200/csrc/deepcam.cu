@@ -650,9 +650,10 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
 // one bitmap word (one warp OR-reduction) and every lane fetches its segment's
 // parameters by shuffle.  Falls back to the shared-memory tables otherwise.
 template <int OUT, bool RAWSEG>  // RAWSEG: a mode-3 line (FORMAT.md 2.7); mode-1 lines run without its code
-__device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t hdr, uint32_t bytes, uint32_t W,
-                                                    uint32_t *bbits, uint32_t nbw, float shv, float scv, uint8_t *row,
-                                                    uint8_t *rowbuf, uint32_t rep_s, int lane) {
+__device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t buf_s, uint32_t hdr, uint32_t bytes,
+                                                    uint32_t W, uint32_t *bbits, uint32_t nbw, float shv, float scv,
+                                                    uint8_t *row, uint8_t *rowbuf, uint32_t rowbuf_s, uint32_t rep_s,
+                                                    int lane) {
     constexpr int VPL = 36;
     const uint32_t nseg = hdr >> 16;
     // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
@@ -661,28 +662,25 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t hdr, 
     if (nseg > (uint32_t)kWarp)
         return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, rowbuf, lane);
     if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
-    const uint32_t dl_s = smem_u32(buf + 4 + 8 * nseg);
+    const uint32_t dl_s = buf_s + 4 + 8 * nseg;
     const bool have = (uint32_t)lane < nseg;
-    uint32_t len = 0, kind = 0, eb = 0;
-    float hs = 0.f;
-    if (have) {
-        const uint32_t d = reinterpret_cast<const uint32_t *>(buf + 4)[lane];
-        len = d & 0xFFFFu;
-        kind = (d >> 16) & 0xFFu;
-        eb = d >> 24;
-        hs = reinterpret_cast<const float *>(buf + 4 + 4 * nseg)[lane];
-    }
-    const uint32_t dlen = (kind == kDiff && len > 0) ? len - 1 : (kind == kRawSeg ? 4u * len : 0u);
+    // lanes past nseg read the (in-slot) neighbouring words and discard them
+    const uint32_t dw = lds_u32(buf_s + 4 + 4 * (uint32_t)lane);
+    const float hs = lds_f32(buf_s + 4 + 4 * nseg + 4 * (uint32_t)lane);
+    const uint32_t len = have ? dw & 0xFFFFu : 0u, kind = have ? (dw >> 16) & 0xFFu : 0u, eb = dw >> 24;
+    const uint32_t dlen = kind == kDiff ? len - (len > 0) : (kind == kRawSeg ? 4u * len : 0u);
     const uint32_t pk = len | (dlen << 16);
     const uint32_t inc = scan_incl_u32(pk);
     const uint32_t ex = inc - pk;
     const uint32_t st = ex & 0xFFFFu, db = ex >> 16;
     const uint32_t blk = st / VPL;
-    bool bad = have && (len == 0 || kind > max_kind || (kind == kDiff && (eb < (uint32_t)kEminBMin || eb > (uint32_t)kEminBMax)) ||
-                        st + len > W || blk * VPL != st);
+    // validation without short-circuit branches (FORMAT.md 2.1 / 2.7 rules)
+    const uint32_t bad_lane = (uint32_t)have & ((uint32_t)(len == 0) | (uint32_t)(kind > max_kind) |
+                                                ((uint32_t)(kind == kDiff) & ((uint32_t)(eb < (uint32_t)kEminBMin) |
+                                                                              (uint32_t)(eb > (uint32_t)kEminBMax))) |
+                                                (uint32_t)(st + len > W) | (uint32_t)(blk * VPL != st));
     const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-    bad = __any_sync(0xffffffffu, bad) || (tot & 0xFFFFu) != W || 4u + 8u * nseg + (tot >> 16) > bytes;
-    if (bad) return false;
+    if (__any_sync(0xffffffffu, bad_lane) | ((tot & 0xFFFFu) != W) | (4u + 8u * nseg + (tot >> 16) > bytes)) return false;
     const uint32_t word = __reduce_or_sync(0xffffffffu, have ? 1u << blk : 0u);  // head lanes
     // DIFF: the code of position p is delta byte a + p; RAW: its value is at bytes a + 4p
     const int a_s = kind == kRawSeg ? (int)db - 4 * (int)st : (int)db - (int)st - 1;
@@ -750,7 +748,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t hdr, 
         for (int i = 0; i < VPL; i++) y[i] = __fmul_rn(__fadd_rn(lds_f32_any(va + 4u * i), -shv), scv);
     }
     row_buffer_acquire(lane);
-    stage_vpl<OUT, VPL>(smem_u32(rowbuf) + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
+    stage_vpl<OUT, VPL>(rowbuf_s + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
     row_buffer_release<OUT>(row, rowbuf, W, lane);
     return true;
 }
@@ -1112,6 +1110,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     const uint32_t nbw = (W / VPL + 31) / 32;
     const uint32_t nsb = nwords / 2;  // words of the start bitmap (and of its prefix counts)
     const uint32_t rep_s = smem_u32(smem_raw + (size_t)wpc * warp_bytes);  // 48 B of 0x80 (producer-filled)
+    const uint32_t base_s = smem_u32(base), rowbuf_s = smem_u32(rowbuf);      // shared addresses, hoisted
     uint32_t fph = 0;  // bit s: parity of slot s's next full phase
     uint32_t s = 0;
     const uint32_t nlines = (uint32_t)(g_end - g_begin);  // < 2^32: lines of one warp
@@ -1134,9 +1133,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             continue;
         }
         if (bytes) {
-            uint8_t *buf = (flags & kFlagBig) ? base : base + s * cap;
+            const uint32_t boff = (flags & kFlagBig) ? 0u : s * cap;
+            uint8_t *buf = base + boff;
+            const uint32_t buf_s = base_s + boff;
             const float shv = __uint_as_float(inf.z), scv = __uint_as_float(inf.w);
-            const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);  // mode (byte 0) and nseg (bytes 2-3)
+            const uint32_t hdr = lds_u32(buf_s);  // mode (byte 0) and nseg (bytes 2-3)
             const uint32_t mode = hdr & 0xFFu;
             bool ok;
             if (RAWSEG && mode == kModeRaw16) {
@@ -1145,11 +1146,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             } else if (VEC && al == (uint32_t)VPL && (mode == kModeSeg || (RAWSEG && mode == kModeSegRaw))) {
                 if constexpr (VPL == 36) {
                     if (!RAWSEG || mode == kModeSeg)
-                        ok = decode_line_onepass<OUT, false>(buf, hdr, bytes, W, sbits, nbw, shv, scv, row, rowbuf,
-                                                             rep_s, lane);
+                        ok = decode_line_onepass<OUT, false>(buf, buf_s, hdr, bytes, W, sbits, nbw, shv, scv, row,
+                                                             rowbuf, rowbuf_s, rep_s, lane);
                     else
-                        ok = decode_line_onepass<OUT, true>(buf, hdr, bytes, W, sbits, nbw, shv, scv, row, rowbuf,
-                                                            rep_s, lane);
+                        ok = decode_line_onepass<OUT, true>(buf, buf_s, hdr, bytes, W, sbits, nbw, shv, scv, row,
+                                                            rowbuf, rowbuf_s, rep_s, lane);
                 }
                 else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
             } else {

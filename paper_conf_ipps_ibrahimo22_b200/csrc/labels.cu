@@ -28,6 +28,17 @@ namespace {
 constexpr uint32_t kLabelMagic = 0x4C505053u;  // "SPPL"
 constexpr int kLabelHeader = 32;
 constexpr int kKlWarps = 8;  // warps per CTA
+constexpr uint32_t kKlChunk = 4096;  // positions per bitmap pass (128 words per warp)
+
+// inclusive warp scan, the shuffle's in-range predicate guarding the add
+__device__ __forceinline__ uint32_t scan_u32(uint32_t v) {
+#pragma unroll
+    for (int d = 1; d < kWarp; d <<= 1)
+        asm("{\n.reg .u32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, 0, 0xffffffff;\n@p add.u32 %0, %0, t;\n}\n"
+            : "+r"(v)
+            : "r"(d));
+    return v;
+}
 
 // header check shared by both kinds: returns total (0 if invalid)
 __device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t limit, uint32_t kind, uint32_t H,
@@ -46,7 +57,7 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                                                                    const uint64_t *__restrict__ src_bytes, int n,
                                                                    uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
                                                                    uint32_t *__restrict__ status) {
-    __shared__ uint32_t bitmap[kKlWarps][32];
+    __shared__ uint32_t bitmap[kKlWarps][kKlChunk / 32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t *bm = bitmap[warp];
     const uint64_t T = (uint64_t)n * H;
@@ -90,61 +101,64 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
             ok = nrun >= 1 && nrun <= W && 4ull + 3ull * nrun <= bytes;
             const uint16_t *lens = reinterpret_cast<const uint16_t *>(p + 4);
             const uint8_t *vals = p + 4 + 2 * nrun;
-            // pass 1: validate the run lengths (len >= 1, sum = W)
-            uint32_t carry = 0;
-            bool bad = false;
-            for (uint32_t r0 = 0; ok && r0 < nrun; r0 += kWarp) {
-                const uint32_t r = r0 + lane;
-                const uint32_t len = r < nrun ? __ldg(lens + r) : 0u;
-                bad |= r < nrun && len == 0;
-                carry += __reduce_add_sync(0xffffffffu, len);
-            }
-            ok = ok && !__any_sync(0xffffffffu, bad) && carry == W;
-            // pass 2: 1,024 positions at a time, lane l owns [c0 + 32 l, c0 + 32 l + 32)
-            for (uint32_t c0 = 0; ok && c0 < W; c0 += 32 * kWarp) {
-                bm[lane] = 0;
+            // positions in chunks of kKlChunk: one pass over the runs sets the
+            // chunk's run starts in the warp's bitmap (and validates the lengths);
+            // lane l then owns the 32-position windows l, l + 32, ... of the chunk
+            for (uint32_t c0 = 0; ok && c0 < W; c0 += kKlChunk) {
+                for (uint32_t k = lane; k < kKlChunk / 32; k += kWarp) bm[k] = 0;
                 __syncwarp();
                 uint32_t before = 0, run_end = 0;
-                for (uint32_t r0 = 0; r0 < nrun && run_end <= c0 + 32 * kWarp; r0 += kWarp) {
+                bool bad = false;
+                for (uint32_t r0 = 0; r0 < nrun && (c0 == 0 || run_end <= c0 + kKlChunk); r0 += kWarp) {
                     const uint32_t r = r0 + lane;
                     const uint32_t len = r < nrun ? __ldg(lens + r) : 0u;
-                    const uint32_t incl = warp_incl_scan(len, lane);
+                    bad |= r < nrun && len == 0;
+                    const uint32_t incl = scan_u32(len);
                     const uint32_t st = run_end + incl - len;
-                    if (r < nrun && st >= c0 && st < c0 + 32 * kWarp)
-                        atomicOr(&bm[(st - c0) >> 5], 1u << (st & 31));
+                    if (r < nrun && st >= c0 && st < c0 + kKlChunk) atomicOr(&bm[(st - c0) >> 5], 1u << (st & 31));
                     before += __popc(__ballot_sync(0xffffffffu, r < nrun && st < c0));
                     run_end += __shfl_sync(0xffffffffu, incl, 31);
                 }
+                if (c0 == 0) ok = !__any_sync(0xffffffffu, bad) && run_end == W;  // the first pass saw every run
                 __syncwarp();
-                const uint32_t word = bm[lane];
-                const uint32_t c = __popc(word);
-                const uint32_t base = before + warp_incl_scan(c, lane) - c;  // starts before this lane's positions
-                const uint32_t p0 = c0 + 32 * lane;
-                if (p0 < W) {
-                    // the run of p0, then one fill per run starting inside the window
-                    // (a mask row has a handful of runs: usually none starts here)
-                    uint32_t idx = base + (word & 1u) - 1;
-                    uint32_t v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
-                    uint32_t out[8];
+                if (!ok) break;
+                uint32_t carry = before;
+                for (uint32_t w0 = 0; w0 < kKlChunk / 32 && c0 + 32 * w0 < W; w0 += kWarp) {
+                    const uint32_t word = bm[w0 + lane];
+                    const uint32_t c = __popc(word);
+                    const uint32_t incl = scan_u32(c);
+                    const uint32_t base = carry + incl - c;  // run starts before this lane's window
+                    carry += __shfl_sync(0xffffffffu, incl, 31);
+                    const uint32_t p0 = c0 + 32 * (w0 + lane);
+                    if (p0 < W) {
+                        // the run of p0, then one fill per run starting inside the window
+                        // (a mask row has a handful of runs: usually none starts here)
+                        uint32_t idx = base + (word & 1u) - 1;
+                        uint32_t v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
+                        uint32_t out[8];
 #pragma unroll
-                    for (int k = 0; k < 8; k++) out[k] = v;
-                    for (uint32_t w = word & ~1u; w; w &= w - 1) {
-                        const uint32_t j = __ffs(w) - 1;  // a run starts at p0 + j: bytes j.. take its value
-                        idx++;
-                        v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
+                        for (int k = 0; k < 8; k++) out[k] = v;
+                        for (uint32_t w = word & ~1u; w; w &= w - 1) {
+                            const uint32_t j = __ffs(w) - 1;  // a run starts at p0 + j: bytes j.. take its value
+                            idx++;
+                            v = __ldg(vals + min(idx, nrun - 1)) * 0x01010101u;
 #pragma unroll
-                        for (int k = 0; k < 8; k++) {
-                            // bytes 4k..4k+3 at or after j
-                            const int sh = (int)j - 4 * k;
-                            const uint32_t m = sh <= 0 ? 0xFFFFFFFFu : (sh >= 4 ? 0u : 0xFFFFFFFFu << (8 * sh));
-                            out[k] = (out[k] & ~m) | (v & m);
+                            for (int k = 0; k < 8; k++) {
+                                const int sh = (int)j - 4 * k;  // bytes 4k..4k+3 at or after j
+                                const uint32_t m = sh <= 0 ? 0xFFFFFFFFu : (sh >= 4 ? 0u : 0xFFFFFFFFu << (8 * sh));
+                                out[k] = (out[k] & ~m) | (v & m);
+                            }
                         }
-                    }
-                    if (vec16 && p0 + 32 <= W) {
-                        reinterpret_cast<uint4 *>(row + p0)[0] = make_uint4(out[0], out[1], out[2], out[3]);
-                        reinterpret_cast<uint4 *>(row + p0)[1] = make_uint4(out[4], out[5], out[6], out[7]);
-                    } else {
-                        for (int j = 0; j < 32 && p0 + j < W; j++) row[p0 + j] = (uint8_t)(out[j >> 2] >> (8 * (j & 3)));
+                        if (vec16 && p0 + 32 <= W) {
+                            reinterpret_cast<uint4 *>(row + p0)[0] = make_uint4(out[0], out[1], out[2], out[3]);
+                            reinterpret_cast<uint4 *>(row + p0)[1] = make_uint4(out[4], out[5], out[6], out[7]);
+                        } else {
+#pragma unroll
+                            for (int k = 0; k < 8; k++)
+#pragma unroll
+                                for (int bb = 0; bb < 4; bb++)
+                                    if (p0 + 4 * k + bb < W) row[p0 + 4 * k + bb] = (uint8_t)(out[k] >> (8 * bb));
+                        }
                     }
                 }
                 __syncwarp();
