@@ -765,8 +765,8 @@ def test_deepcam_decoder_rejects_corruption(orc):
 
 
 def test_deepcam_segment_alignment(orc):
-    """FORMAT.md 2.1/2.4: the encoder aligns segment starts to A (12 when
-    W % 384 == 0, 8 when W % 8 == 0, else 1) and decoders reject violations."""
+    """FORMAT.md 2.1/2.4: the encoder aligns segment starts to A (36 when
+    W = 1152, 8 when W % 8 == 0, else 1) and decoders reject violations."""
     rng = np.random.default_rng(33)
     for W, A in ((384, 8), (1152, 36), (64, 8), (200, 8), (37, 1)):
         x = np.cumsum(rng.standard_normal((1, 6, W)) * 0.05, axis=2).astype(np.float32)
