@@ -668,7 +668,8 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t buf_s
     const uint32_t dw = lds_u32(buf_s + 4 + 4 * (uint32_t)lane);
     const float hs = lds_f32(buf_s + 4 + 4 * nseg + 4 * (uint32_t)lane);
     const uint32_t len = have ? dw & 0xFFFFu : 0u, kind = have ? (dw >> 16) & 0xFFu : 0u, eb = dw >> 24;
-    const uint32_t dlen = kind == kDiff ? len - (len > 0) : (kind == kRawSeg ? 4u * len : 0u);
+    // delta bytes: len - 1 for DIFF, 4 len for a RAW segment (mode 3 only), none for REPEAT (selects, no branches)
+    const uint32_t dlen = (kind == kDiff ? len - (uint32_t)(len > 0) : 0u) + ((RAWSEG && kind == kRawSeg) ? 4u * len : 0u);
     const uint32_t pk = len | (dlen << 16);
     const uint32_t inc = scan_incl_u32(pk);
     const uint32_t ex = inc - pk;
