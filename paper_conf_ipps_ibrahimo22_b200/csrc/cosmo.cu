@@ -463,8 +463,8 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         bool staged;     // esp is in shared memory (at ssh)
         uint32_t ssh;
     };
-    auto esc_tile = [&](uint32_t t, uint32_t stg) {  // stg = (ring.count + t) % kKeyStages
-        const uint8_t *stage = ring.buf + stg * kStageBytes;
+    auto esc_tile = [&](uint32_t t) {
+        const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
         const uint64_t st = a + (uint64_t)t * kTileVox;
         const uint64_t rem = b - st;
         const uint32_t nvox = rem < (uint64_t)kTileVox ? (uint32_t)rem : (uint32_t)kTileVox;
@@ -556,17 +556,10 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         mbar_arrive_expect_tx(&ring.full[stg], bytes);
         bulk_g2s(ring.buf + stg * kStageBytes, sv.keys + st * kwb, bytes, &ring.full[stg]);
     };
-    auto wait_full = [&](uint32_t stg, uint32_t ph) { mbar_wait(&ring.full[stg], ph); };
-    // stage index and full-barrier parity of a tile, advanced incrementally (no
-    // division by the 5-stage ring size per tile)
-    struct StagePos {
-        uint32_t stg, ph;
-        __device__ __forceinline__ void next() {
-            if (++stg == (uint32_t)kKeyStages) {
-                stg = 0;
-                ph ^= 1u;
-            }
-        }
+    auto wait_full = [&](uint32_t t) {
+        const uint32_t gt = ring.count + t;
+        mbar_wait(&ring.full[gt % kKeyStages], (gt / kKeyStages) & 1u);
+        return ring.buf + (gt % kKeyStages) * kStageBytes;
     };
     // Cold rows: while tile t is expanded, the thread classifies its keys of
     // tile t + kColdLA and starts LDGSTS copies (cp.async) of its first
@@ -580,18 +573,18 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     auto slot_addr = [&](uint32_t t, uint32_t k) {  // slot k of this thread for tile t
         return ring.cold + ((((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * kColdSlots + k) * 8;
     };
-    auto classify = [&](uint32_t t, uint32_t stg) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
+    auto classify = [&](uint32_t t) -> uint32_t {  // tile t's keys are in smem (full barrier passed)
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         uint32_t cold = 0;
         Keys8 kres;
         uint32_t escw = 0;  // escaped tile: escape mask << 8 | first escape (tile-relative) << 16
         if (escd) {         // warp-collective (scan): inactive lanes take part with no keys
-            const uint8_t *stage = ring.buf + stg * kStageBytes;
+            const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
             const uint2 raw = q < b ? lds_u2(smem_u32(stage) + threadIdx.x * 8u) : make_uint2(0u, 0u);
             const uint32_t m = q < b ? esc_mask8(raw) : 0u;
             const uint32_t c = __popc(m);
             const uint32_t incl = warp_incl_scan(c, (int)lane);
-            const EscTile et = esc_tile(t, stg);
+            const EscTile et = esc_tile(t);
             const uint32_t wtot = __shfl_sync(0xffffffffu, incl, 31);
             if (lane == 0 && et.wact && wtot != et.wcnt) bad = 1u;  // the index disagrees with the low bytes
             const uint32_t r0 = et.wbase + incl - c;
@@ -606,7 +599,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             }
         }
         if (q < b) {
-            const uint8_t *stage = ring.buf + stg * kStageBytes;
+            const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
             const Keys8 k = escd ? kres : keys_from_smem(stage, kwb);
 #pragma unroll
             for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
@@ -631,24 +624,21 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
     if (!kProducerWarp && threadIdx.x == 0) {
         for (uint32_t t = 0; t < ntiles && t < (uint32_t)(kKeyStages - 1); t++) issue(t);
     }
-    StagePos cur{ring.count % kKeyStages, (ring.count / kKeyStages) & 1u};  // tile t
-    StagePos ahead = cur;                                                  // tile t + kColdLA
 #pragma unroll
     for (int i = 0; i < kColdLA; i++) {
         if ((uint32_t)i < ntiles) {
-            wait_full(ahead.stg, ahead.ph);
-            cj[i] = classify(i, ahead.stg);
+            wait_full(i);
+            cj[i] = classify(i);
         } else {
             cp_async_commit();
         }
-        ahead.next();
     }
 #pragma unroll 1
-    for (uint32_t t = 0; t < ntiles; t++, cur.next(), ahead.next()) {
+    for (uint32_t t = 0; t < ntiles; t++) {
         if (!kProducerWarp && threadIdx.x == 0 && t + kKeyStages - 1 < ntiles) issue(t + kKeyStages - 1);
         if (t + kColdLA < ntiles) {
-            wait_full(ahead.stg, ahead.ph);
-            cj[kColdLA] = classify(t + kColdLA, ahead.stg);
+            wait_full(t + kColdLA);
+            cj[kColdLA] = classify(t + kColdLA);
         } else {
             cp_async_commit();  // keep one group per iteration
         }
@@ -656,7 +646,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         const uint32_t cmask_all = cj[0], cmask = cmask_all & 0xFFu;  // cold mask (+ escapes, kw = 3)
 #pragma unroll
         for (int i = 0; i < kColdLA; i++) cj[i] = cj[i + 1];  // rotate (compile-time indices)
-        const uint8_t *stage = ring.buf + cur.stg * kStageBytes;
+        const uint8_t *stage = ring.buf + ((ring.count + t) % kKeyStages) * kStageBytes;
         const uint64_t q = a + (uint64_t)t * kTileVox + 8u * threadIdx.x;
         if (q < b) {
             Keys8 k0;
@@ -664,7 +654,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 if constexpr (kEscPrefetch == 2) {
                     k0.v = lds_u4(rk_base + (((ring.count + t) % (kColdLA + 1)) * kConsumers + threadIdx.x) * 16u);
                 } else {
-                    const EscTile et = esc_tile(t, cur.stg);
+                    const EscTile et = esc_tile(t);
                     k0 = esc_keys(lds_u2(smem_u32(stage) + threadIdx.x * 8u), (cmask_all >> 8) & 0xFFu,
                                   cmask_all >> 16, et);
                 }
@@ -695,7 +685,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
         __syncwarp();
         // this warp is done with the stage: every lane releases its own reads (kAllLanesRelease), or
         // lane 0 for the warp after __syncwarp (bar.warp.sync orders the other lanes' reads)
-        if (kAllLanesRelease || lane == 0) mbar_arrive(&ring.empty[cur.stg]);
+        if (kAllLanesRelease || lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);
     }
     cp_async_wait<0>();
     ring.count += ntiles;
