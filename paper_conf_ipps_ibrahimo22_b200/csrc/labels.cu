@@ -64,28 +64,47 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
     const uint64_t NW = (uint64_t)gridDim.x * kKlWarps, gw = (uint64_t)blockIdx.x * kKlWarps + warp;
     const uint64_t g0 = gw * T / NW, g1 = (gw + 1) * T / NW;
     const uint64_t P = kLabelHeader + ((4ull * (H + 1) + 15) & ~15ull);
-    int64_t cur_s = -1;
-    const uint8_t *b = nullptr;
-    uint64_t total = 0;
     const bool vec16 = (W & 15) == 0;  // rows start 16-B aligned in dst
-    for (uint64_t g = g0; g < g1; g++) {
-        const int64_t s = (int64_t)(g / H);
-        const uint32_t y = (uint32_t)(g - (uint64_t)s * H);
-        if (s != cur_s) {
-            cur_s = s;
-            b = static_cast<const uint8_t *>(src[s]);
-            total = label_header_ok(b, src_bytes ? src_bytes[s] : ~0ull, SPP_LABEL_MASK, H, W);
+    // Row window: lane k holds row (wbase + k)'s payload address, byte count and
+    // first word (mode, nrun), loaded and validated by all lanes at once every
+    // 32 rows, so a row's dependent loads (header -> directory -> row header)
+    // are paid once per 32 rows instead of per row.
+    uint64_t wbase = 0, w_p = 0;
+    uint32_t w_bytes = 0, w_hdr = 0, w_ok = 0;
+    auto load_window = [&](uint64_t wb) {
+        wbase = wb;
+        const uint64_t gk = wb + lane;
+        w_ok = 0;
+        if (gk < g1) {
+            const uint64_t sk = gk / H;
+            const uint32_t yk = (uint32_t)(gk - sk * H);
+            const uint8_t *b = static_cast<const uint8_t *>(src[sk]);
+            uint64_t total = label_header_ok(b, src_bytes ? src_bytes[sk] : ~0ull, SPP_LABEL_MASK, H, W);
             if (total && P > total) total = 0;
-            if (!total && lane == 0) report(status, SPP_ERR_CORRUPT, s);
+            if (total) {
+                const uint32_t *dir = reinterpret_cast<const uint32_t *>(b + kLabelHeader);
+                const uint32_t da = __ldg(dir + yk), db = __ldg(dir + yk + 1);
+                if (db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= total - P && db - da >= 16) {
+                    w_p = reinterpret_cast<uint64_t>(b + P + da);
+                    w_bytes = db - da;
+                    w_hdr = __ldg(reinterpret_cast<const uint32_t *>(w_p));
+                    w_ok = 1;
+                }
+            }
+            if (!w_ok) report(status, SPP_ERR_CORRUPT, (int64_t)sk);
         }
-        if (!total) continue;
-        const uint32_t *dir = reinterpret_cast<const uint32_t *>(b + kLabelHeader);
-        const uint32_t da = __ldg(dir + y), db = __ldg(dir + y + 1);
+    };
+    for (uint64_t g = g0; g < g1; g++) {
+        if (g == g0 || g >= wbase + kWarp) load_window(g);
+        const int kk = (int)(g - wbase);
+        const int64_t s = (int64_t)(g / H);
+        bool ok = __shfl_sync(0xffffffffu, w_ok, kk) != 0;
+        if (!ok) continue;  // reported by the window load
+        const uint8_t *p = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_p, kk));
+        const uint64_t bytes = __shfl_sync(0xffffffffu, w_bytes, kk);
+        const uint32_t hdr = __shfl_sync(0xffffffffu, w_hdr, kk);
         uint8_t *row = dst + g * (uint64_t)W;
-        bool ok = db >= da && ((da | db) & 15u) == 0 && (uint64_t)db <= total - P && db - da >= 16;
-        const uint8_t *p = b + P + da;
-        const uint64_t bytes = ok ? db - da : 0;
-        const uint32_t mode = ok ? __ldg(p) : 0xFFu;
+        const uint32_t mode = hdr & 0xFFu;
         if (ok && mode == 0) {  // verbatim row
             ok = 16ull + W <= bytes;
             if (ok) {
@@ -97,7 +116,7 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                 }
             }
         } else if (ok && mode == 1) {  // maximal runs
-            const uint32_t nrun = __ldg(reinterpret_cast<const uint16_t *>(p + 2));
+            const uint32_t nrun = hdr >> 16;
             ok = nrun >= 1 && nrun <= W && 4ull + 3ull * nrun <= bytes;
             const uint16_t *lens = reinterpret_cast<const uint16_t *>(p + 4);
             const uint8_t *vals = p + 4 + 2 * nrun;
