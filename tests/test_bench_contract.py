@@ -50,6 +50,13 @@ def test_gpu_arm_contract():
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["gpu_launches"] == 2 * d["steps"]
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    # round-2 reporting (VERDICT r1 missing 5): nominal-peak fraction, per-rank H2D and overlap,
+    # placement, format statistics, value = mode A / e2e = mode B labels
+    assert abs(r["frac_nominal_8tbs"] - r["achieved"] / 8000.0) < 1e-9
+    assert len(d["per_rank"]) == 1 and d["per_rank"][0]["h2d_gbs"] > 0 and 0 < d["per_rank"][0]["overlap"] <= 1.5
+    assert len(d["config"]["placement"]) == 1 and "mode A" in d["config"]["workload"]
+    st = d["config"]["stream_stats"]
+    assert st["nU_mean"] > 0 and st["G_slab0_mean"] > 0 and st["kw_slab0"]
 
 
 @pytest.mark.gpu
