@@ -284,6 +284,8 @@ def run_gpu(args, rank: int, world: int, local_rank: int, dist):
     # weak: every rank its own batch of B_total samples (distinct seeds);
     # strong: the one B_total set split across ranks (the same seeds everywhere)
     B = len(shard_indices(B_total, rank, world)) if strong else B_total
+    if B < 1:
+        raise ValueError(f"--scaling strong with a batch of {B_total} leaves rank {rank} of {world} without samples")
     t_setup = time.perf_counter()
     esc = args.escape_keys and args.workload == "cosmo"
     seed = W["seed"] if strong else rank_seed_base(W["seed"], rank)
