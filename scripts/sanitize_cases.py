@@ -67,3 +67,27 @@ for rs in (False, True):  # general line path / one-pass instance (opts.raw_segm
     print("deepcam raw segments ok", rs, run("deepcam", [r, r], y.shape, raw_segments=rs))
     print("deepcam raw segment in mode 1", rs, run("deepcam", [r, rm1], y.shape, raw_segments=rs))
     print("deepcam raw segment too long", rs, run("deepcam", [rlen, r], y.shape, out="f32", raw_segments=rs))
+# lossless labels (FORMAT.md 3): valid, wrong kind, bad run sum, truncated (src_bytes)
+from paper_conf_ipps_ibrahimo22_b200 import LabelDecoder  # noqa: E402
+from synth import gen_deepcam_labels  # noqa: E402
+m = gen_deepcam_labels(9, H=32, W=256)
+lb = spp.spp_encode_label_mask(m)
+hl = fmt.label_header(lb)
+lk = lb.copy(); lk[6] = 2
+ls = lb.copy(); ls[hl["payload_off"] + int(hl["dir"][3]) + 4] ^= 0x40
+lt = lb[: lb.size // 2].copy()
+
+
+def run_labels(bufs):
+    d = LabelDecoder("mask", m.shape)
+    srcs = [torch.from_numpy(b).cuda() for b in bufs]
+    sizes = torch.tensor([b.size for b in bufs], dtype=torch.int64, device="cuda")
+    d.decode(srcs, src_bytes=sizes)
+    torch.cuda.synchronize()
+    return int(d.status.item())
+
+
+print("labels ok", run_labels([lb, lb]))
+print("labels bad kind", run_labels([lb, lk]))
+print("labels bad run sum", run_labels([ls, lb]))
+print("labels truncated", run_labels([lb, lt]))
