@@ -2,7 +2,10 @@
 // P:175 "For both applications, we use lossless compression of the labels").
 //
 //   KL  kl_decode_mask  persistent warps, one mask row at a time (rows are
-//                       independent, like DeepCAM data lines): a RUN row's
+//                       independent, like DeepCAM data lines).  Rows of
+//                       <= 32 runs (W % 16 == 0, W <= 2048) are filled in
+//                       registers and leave by TMA bulk store
+//                       (kl_run_row_staged); other RUN rows: the row's
 //                       run starts (warp scan of the run lengths) are set in a
 //                       per-warp bitmap of 1,024 positions; lane l owns 32
 //                       consecutive positions, so the run of position p is
@@ -29,6 +32,8 @@ constexpr uint32_t kLabelMagic = 0x4C505053u;  // "SPPL"
 constexpr int kLabelHeader = 32;
 constexpr int kKlWarps = 8;  // warps per CTA
 constexpr uint32_t kKlChunk = 4096;  // positions per bitmap pass (128 words per warp)
+constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 16 words per lane)
+constexpr uint32_t kKlFastRuns = 32;  // staged RUN rows: one run per lane
 
 // inclusive warp scan, the shuffle's in-range predicate guarding the add
 __device__ __forceinline__ uint32_t scan_u32(uint32_t v) {
@@ -38,6 +43,71 @@ __device__ __forceinline__ uint32_t scan_u32(uint32_t v) {
             : "+r"(v)
             : "r"(d));
     return v;
+}
+
+__device__ __forceinline__ void bulk_wait_read_1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+
+// Staged RUN row (nrun <= 32, W % 16 == 0, W <= 2048; the paper's masks have
+// 1-5 runs per row): lane r holds run r (length, value); one warp scan gives
+// the run starts, each start sets one bit in the bitmap of the lane owning its
+// position (lane l owns words [wpl l, wpl l + wpl) of the row: <= 64
+// positions, two bitmap words); a popc scan of those words gives the run at
+// each lane's first position, and the lane's words are filled in registers,
+// written to the warp's staging row and leave with one TMA bulk store.
+template <int WPL>  // words (4 positions) per lane: W = 1152 -> 9
+__device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
+                                                  uint32_t magic, uint32_t *bm, uint32_t bm_s,
+                                                  uint8_t *stage, uint32_t stage_s, uint8_t *row, int lane) {
+    if (4ull + 3ull * nrun > bytes) return false;
+    const bool have = (uint32_t)lane < nrun;
+    const uint32_t len = have ? __ldg(reinterpret_cast<const uint16_t *>(p + 4) + lane) : 0u;
+    const uint32_t val = have ? __ldg(p + 4 + 2 * nrun + lane) : 0u;
+    const uint32_t incl = scan_u32(len), st = incl - len;
+    const bool bad = __any_sync(0xffffffffu, have && len == 0) || __shfl_sync(0xffffffffu, incl, 31) != W;
+    if (bad) return false;
+    constexpr uint32_t rlen = 4u * WPL;  // positions per lane
+    sts_u2(bm_s + 8u * (uint32_t)lane, make_uint2(0u, 0u));
+    __syncwarp();
+    if (have) {
+        const uint32_t o = __umulhi(st, magic);  // st / rlen (exact: st < 2^16, rlen <= 64)
+        const uint32_t b = st - o * rlen;
+        atomicOr(bm + 2 * o + (b >> 5), 1u << (b & 31));
+    }
+    __syncwarp();
+    const uint2 mm = lds_u2(bm_s + 8u * (uint32_t)lane);
+    const uint32_t c = __popc(mm.x) + __popc(mm.y);
+    const uint32_t before = scan_u32(c) - c;  // run starts before this lane's first position
+    uint32_t idx = before + (mm.x & 1u) - 1u;  // run of the first position (run 0 starts at 0)
+    uint64_t rest = ((uint64_t)mm.y << 32 | mm.x) & ~1ull;
+    uint32_t v = __shfl_sync(0xffffffffu, val, idx & 31) * 0x01010101u;
+    uint32_t out[WPL];
+#pragma unroll
+    for (int k = 0; k < WPL; k++) out[k] = v;
+    const uint32_t tmax = __reduce_max_sync(0xffffffffu, c - (mm.x & 1u));
+    for (uint32_t t = 0; t < tmax; t++) {  // one pass per run starting inside the lane's words
+        const bool has = rest != 0;
+        const uint32_t j = has ? (uint32_t)__ffsll((long long)rest) - 1u : 0u;
+        idx += has;
+        v = __shfl_sync(0xffffffffu, val, idx & 31) * 0x01010101u;
+        rest &= rest - 1;
+        if (has) {
+            const uint32_t kj = j >> 2, keep = 0xFFFFFFFFu >> (32 - 8 * (j & 3));  // bytes of word kj before j
+#pragma unroll
+            for (int k = 0; k < WPL; k++) {
+                const uint32_t m = (uint32_t)k > kj ? 0u : ((uint32_t)k == kj ? ((j & 3) ? keep : 0u) : 0xFFFFFFFFu);
+                out[k] = (out[k] & m) | (v & ~m);
+            }
+        }
+    }
+    const uint32_t lo = rlen * (uint32_t)lane;
+    const uint32_t nw = lo + rlen <= W ? (uint32_t)WPL : (lo < W ? (W - lo) / 4 : 0u);  // the last lanes: part / none
+#pragma unroll
+    for (int k = 0; k < WPL; k++)
+        if ((uint32_t)k < nw) sts_f32(stage_s + lo + 4u * k, __uint_as_float(out[k]));
+    fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
+    __syncwarp();
+    if (lane == 0) bulk_s2g(row, stage, W);
+    return true;
 }
 
 // header check shared by both kinds: returns total (0 if invalid)
@@ -53,13 +123,18 @@ __device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t l
     return ok ? total : 0;
 }
 
+template <int WPL>  // 0: no staged rows (W % 16 != 0, W > 2048 or an unaligned dst)
 __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *const *__restrict__ src,
                                                                    const uint64_t *__restrict__ src_bytes, int n,
                                                                    uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
                                                                    uint32_t *__restrict__ status) {
     __shared__ uint32_t bitmap[kKlWarps][kKlChunk / 32];
+    __shared__ __align__(128) uint8_t stage_rows[kKlWarps][2][kKlFastW];  // double-buffered staging rows
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t *bm = bitmap[warp];
+    const uint32_t bm_s = smem_u32(bm);
+    const uint32_t magic = 0xFFFFFFFFu / (4u * (WPL > 0 ? WPL : 1)) + 1u;
+    uint32_t nstaged = 0;  // rows this warp has stored by TMA (buffer nstaged & 1 next)
     const uint64_t T = (uint64_t)n * H;
     const uint64_t NW = (uint64_t)gridDim.x * kKlWarps, gw = (uint64_t)blockIdx.x * kKlWarps + warp;
     const uint64_t g0 = gw * T / NW, g1 = (gw + 1) * T / NW;
@@ -97,7 +172,6 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
     for (uint64_t g = g0; g < g1; g++) {
         if (g == g0 || g >= wbase + kWarp) load_window(g);
         const int kk = (int)(g - wbase);
-        const int64_t s = (int64_t)(g / H);
         bool ok = __shfl_sync(0xffffffffu, w_ok, kk) != 0;
         if (!ok) continue;  // reported by the window load
         const uint8_t *p = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_p, kk));
@@ -115,6 +189,13 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                     for (uint32_t k = lane; k < W; k += kWarp) row[k] = __ldg(p + 16 + k);
                 }
             }
+        } else if (WPL > 0 && ok && mode == 1 && (hdr >> 16) >= 1 && (hdr >> 16) <= kKlFastRuns) {
+            uint8_t *stage = stage_rows[warp][nstaged & 1];
+            if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
+            __syncwarp();
+            ok = kl_run_row_staged<(WPL > 0 ? WPL : 1)>(p, (uint32_t)bytes, hdr >> 16, W, magic, bm, bm_s, stage, smem_u32(stage),
+                                        row, lane);
+            nstaged += ok;
         } else if (ok && mode == 1) {  // maximal runs
             const uint32_t nrun = hdr >> 16;
             ok = nrun >= 1 && nrun <= W && 4ull + 3ull * nrun <= bytes;
@@ -185,8 +266,9 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
         } else {
             ok = false;
         }
-        if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, s);
+        if (!ok && lane == 0) report(status, SPP_ERR_CORRUPT, (int64_t)(g / H));
     }
+    if (lane == 0) bulk_wait_all();  // shared memory must outlive the last row stores
 }
 
 __global__ void kl_decode_vec(const void *const *__restrict__ src, const uint64_t *__restrict__ src_bytes, int n,
@@ -218,8 +300,23 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
     } else {
         const uint64_t rows = (uint64_t)n * H;
         const uint64_t ctas = std::min<uint64_t>((uint64_t)dp.sms * 8, (rows + kKlWarps - 1) / kKlWarps);
-        kl_decode_mask<<<(unsigned)std::max<uint64_t>(1, ctas), kKlWarps * kWarp, 0, stream>>>(
-            d_src, src_bytes, n, (uint32_t)H, (uint32_t)W, static_cast<uint8_t *>(d_dst), status);
+        // staged rows leave by TMA bulk store: 16-B aligned rows of a multiple of 16 bytes
+        const bool staged = (W % 16) == 0 && W <= (int)kKlFastW && (reinterpret_cast<uintptr_t>(d_dst) & 15) == 0;
+        const int wpl = staged ? (W / 4 + kWarp - 1) / kWarp : 0;
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, ctas);
+        uint8_t *dst = static_cast<uint8_t *>(d_dst);
+        switch (wpl) {
+#define SPP_KL_CASE(k)                                                                                            \
+    case k:                                                                                                       \
+        kl_decode_mask<k><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W, dst, \
+                                                                 status);                                         \
+        break;
+            SPP_KL_CASE(0) SPP_KL_CASE(1) SPP_KL_CASE(2) SPP_KL_CASE(3) SPP_KL_CASE(4) SPP_KL_CASE(5) SPP_KL_CASE(6)
+            SPP_KL_CASE(7) SPP_KL_CASE(8) SPP_KL_CASE(9) SPP_KL_CASE(10) SPP_KL_CASE(11) SPP_KL_CASE(12)
+            SPP_KL_CASE(13) SPP_KL_CASE(14) SPP_KL_CASE(15) SPP_KL_CASE(16)
+#undef SPP_KL_CASE
+            default: return SPP_ERR_INVALID_ARG;
+        }
     }
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }

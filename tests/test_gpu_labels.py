@@ -35,17 +35,36 @@ def _decode(kind, bufs, dims, src_bytes=False):
     return out.cpu().numpy(), int(d.status.item())
 
 
-@pytest.mark.parametrize("H,W", [(768, 1152), (5, 37), (3, 2100), (1, 1), (4, 1024)])
+def _runs_mask(rng, H, W):
+    """Row y has exactly min(y + 1, W) maximal runs (cut points drawn at random,
+    neighbouring runs of different classes): 1..H runs, across the 32-run
+    limit of the staged path."""
+    m = np.empty((H, W), np.uint8)
+    for y in range(H):
+        k = min(y + 1, W)
+        cuts = np.sort(rng.choice(np.arange(1, W), size=k - 1, replace=False)) if k > 1 else np.array([], int)
+        bounds = np.concatenate([[0], cuts, [W]])
+        v = int(rng.integers(0, 256))
+        for r in range(k):
+            m[y, bounds[r]:bounds[r + 1]] = v
+            v = (v + 1 + int(rng.integers(0, 255))) % 256
+    return m
+
+
+@pytest.mark.parametrize("H,W", [(768, 1152), (5, 37), (3, 2100), (1, 1), (4, 1024), (40, 1152), (40, 2048),
+                                 (36, 16), (40, 1040), (34, 48)])
 def test_label_masks_lossless(dev, orc, H, W):
     """Paper-shaped DeepCAM masks (cyclone discs, river bands), random masks
     (verbatim rows), constant masks, W not a multiple of 16, W over the 1,024-
-    position chunk; mixed in one batch, bit-exact vs the masks and the oracle."""
+    position chunk; rows of exactly 1..40 runs (the staged path takes <= 32 runs
+    with W % 16 == 0 and W <= 2048: 1152, 2048, 16, 1040 with a partial last
+    lane, 48); mixed in one batch, bit-exact vs the masks and the oracle."""
     from synth import gen_deepcam_labels
     from paper_conf_ipps_ibrahimo22_b200 import spp
     rng = np.random.default_rng(H * 7 + W)
     masks = [gen_deepcam_labels(5000 + i, H=H, W=W) for i in range(6)]
     masks += [rng.integers(0, 256, (H, W), dtype=np.uint8), np.full((H, W), 2, np.uint8),
-              (rng.random((H, W)) < 0.5).astype(np.uint8)]
+              (rng.random((H, W)) < 0.5).astype(np.uint8), _runs_mask(rng, H, W)]
     bufs = [spp.spp_encode_label_mask(m) for m in masks]
     for b, m in zip(bufs, masks):
         assert np.array_equal(orc.label_decode(b, 1, H, W), m)
