@@ -76,6 +76,9 @@ constexpr int kRegionBytes = kHotBytes + kUCap * 4;  // f(U) first, then the hot
 #define SPP_KC_STAGES 5
 #endif
 constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
+#ifndef SPP_KC_DIAG_LDG  // timing diagnostic only (wrong output): cold keys = one global 8-B load, no slots
+#define SPP_KC_DIAG_LDG 0
+#endif
 #ifndef SPP_KC_DIAG_NOCOLD
 #define SPP_KC_DIAG_NOCOLD 0
 #endif
@@ -603,7 +606,7 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
             const Keys8 k = escd ? kres : keys_from_smem(stage, kwb);
 #pragma unroll
             for (int j = 0; j < 8; j++) cold |= (k.get(j) >= n_hot ? 1u : 0u) << j;
-#if SPP_KC_DIAG_NOCOLD
+#if SPP_KC_DIAG_NOCOLD || SPP_KC_DIAG_LDG
             cold = 0;
 #endif
             uint32_t m = cold;
@@ -662,6 +665,19 @@ __device__ __forceinline__ void expand_keys_vec(const SlabView &sv, uint64_t sla
                 k0 = keys_from_smem(stage, kwb);
             }
             E e[8];
+#if SPP_KC_DIAG_LDG
+            if constexpr (OUT == SPP_OUT_F16 && !ESC) {
+#pragma unroll
+                for (int j = 0; j < 8; j++) {
+                    const uint32_t g = k0.get(j);
+                    e[j] = g < n_hot ? lds_entry<OUT>(hot_base + g * EB) : ld_ro_u2(sv.lut + 8ull * min(g, Gm1));
+                }
+                store8<OUT>(out_s, N, slab_v0 + q, e);
+                __syncwarp();
+                if (kAllLanesRelease || lane == 0) mbar_arrive(&ring.empty[(ring.count + t) % kKeyStages]);
+                continue;
+            }
+#endif
 #pragma unroll
             for (int j = 0; j < 8; j++) {
 #if SPP_KC_DIAG_NOCOLD  // timing diagnostic only (wrong output): every key treated as hot
