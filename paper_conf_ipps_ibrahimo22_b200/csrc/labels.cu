@@ -91,10 +91,11 @@ __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t byt
         v = __shfl_sync(0xffffffffu, val, idx & 31) * 0x01010101u;
         rest &= rest - 1;
         if (has) {
-            const uint32_t kj = j >> 2, keep = 0xFFFFFFFFu >> (32 - 8 * (j & 3));  // bytes of word kj before j
+            const uint32_t kj = j >> 2;
+            const uint32_t keep = (j & 3) ? 0xFFFFFFFFu >> (32 - 8 * (j & 3)) : 0u;  // bytes of word kj before j
 #pragma unroll
             for (int k = 0; k < WPL; k++) {
-                const uint32_t m = (uint32_t)k > kj ? 0u : ((uint32_t)k == kj ? ((j & 3) ? keep : 0u) : 0xFFFFFFFFu);
+                const uint32_t m = (uint32_t)k > kj ? 0u : ((uint32_t)k == kj ? keep : 0xFFFFFFFFu);
                 out[k] = (out[k] & m) | (v & ~m);
             }
         }
