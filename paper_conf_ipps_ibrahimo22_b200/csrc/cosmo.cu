@@ -85,6 +85,12 @@ constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 #ifndef SPP_KC_PREFETCH_TAIL
 #define SPP_KC_PREFETCH_TAIL 1
 #endif
+// key tiles are read once: their TMA loads carry an L2 evict_first hint so they do
+// not displace the LUT tails (evict_last) and cold rows (r2: C2 0.817 -> 0.834,
+// dense C5 rows +1-3 points; profiles/r02a3_*, r02a5_*)
+#ifndef SPP_KC_KEY_EF
+#define SPP_KC_KEY_EF 1
+#endif
 constexpr int kTileVox = kConsumers * 8;  // voxels per CTA iteration (8 per consumer thread)
 constexpr int kStageBytes = kTileVox * 2;
 #ifndef SPP_KC_LA
@@ -719,6 +725,9 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
                                            KeyRing ring, uint64_t i0, uint64_t i1, uint32_t items_per_sample,
                                            uint64_t chunk, uint64_t N, uint64_t plane) {
     uint32_t gt = 0;  // CTA-global tile index, same sequence as the consumers' ring.count
+#if SPP_KC_KEY_EF
+    const uint64_t key_pol = l2_policy_evict_first();
+#endif
 #pragma unroll 1
     for (uint64_t it = i0; it < i1; it++) {
         const int s = (int)(it / items_per_sample);
@@ -752,7 +761,11 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
                 if (!escd) {
                     fence_proxy_async_smem();
                     mbar_arrive_expect_tx(&ring.full[stg], bytes);
+#if SPP_KC_KEY_EF
+                    bulk_g2s_hint(stage, sv.keys + st * kwb, bytes, &ring.full[stg], key_pol);
+#else
                     bulk_g2s(stage, sv.keys + st * kwb, bytes, &ring.full[stg]);
+#endif
                     continue;
                 }
                 // FORMAT.md 1.5 tile: low bytes, the eidx entries of its blocks (from an

@@ -320,6 +320,40 @@ def test_cosmo_corruption_detected(dev):
         assert st & 0xFF == 3 and st >> 8 == 1, (i, st)
 
 
+def test_cosmo_raw_slabs_full_size(dev, orc):
+    """RAW-escape slabs (FORMAT.md 1.1, kw = 8) at the paper's 4x128^3 size,
+    in a batch that mixes them with key slabs of the same and other samples
+    (the per-sample shared output table and the hot prefix share one region):
+    an all-RAW dense sample (lambda = 64) in both policies, a sparse sample with
+    a dense RAW band, and the paper preset; fp16, fp32 and int16 bit-exact, and
+    an index >= |U| in a RAW plane is reported as corrupt on its sample."""
+    from synth import gen_cosmo
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(77)
+    dense = gen_cosmo(3101, lam=64.0, rho_c=0.0)
+    band = gen_cosmo(3102, "sparse")
+    band[:, 40:72] = rng.integers(0, 3000, size=(4, 32, 128, 128))
+    paper = gen_cosmo(3103)
+    xs = [dense, band, paper, dense]
+    bufs = [spp.spp_encode_cosmo(dense), spp.spp_encode_cosmo(band), spp.spp_encode_cosmo(paper),
+            spp.spp_encode_cosmo(dense, localize=True)]
+    kws = [{s["kw"] for s in fmt.cosmo_header(b)["slabs"]} for b in bufs]
+    assert kws[0] == {8} and 8 in kws[1] and kws[1] - {8} and kws[3] == {8}
+    for out, tr in (("f16", 1), ("f32", 1), ("i16", 0)):
+        got, st = _decode("cosmo", bufs, dense.shape, out=out, transform=tr)
+        assert st == 0
+        for g, x in zip(got, xs):
+            _same_bits(g, orc.cosmo_direct(x, tr, out))
+    h = fmt.cosmo_header(bufs[1])
+    rs = [s for s in h["slabs"] if s["kw"] == 8][0]
+    bad = bufs[1].copy()
+    nvox = (rs["z1"] - rs["z0"]) * 128 * 128
+    o = rs["keys_off"] + 2 * (2 * nvox + 12345)  # plane 2 of the slab
+    bad[o:o + 2] = 0xFF
+    _, st = _decode("cosmo", [bufs[0], bufs[2], bad], dense.shape, out="f16")
+    assert st & 0xFF == 3 and st >> 8 == 2, st
+
+
 # ------------------------------------------------------------------ DeepCAM
 def _dc_ref(orc, b, shape, shift, scale, out):
     return orc.deepcam_decode(b, shape, shift, scale, out)
