@@ -778,7 +778,11 @@ __device__ __forceinline__ void kc_produce(const void *const *__restrict__ src, 
                                             ? esc_copy_bytes(e0, e1) : 0u;
                 fence_proxy_async_smem();
                 mbar_arrive_expect_tx(&ring.full[stg], bytes + (i_hi - i_lo) + ebytes);
+#if SPP_KC_KEY_EF
+                bulk_g2s_hint(stage, ev.low + st, bytes, &ring.full[stg], key_pol);
+#else
                 bulk_g2s(stage, ev.low + st, bytes, &ring.full[stg]);
+#endif
                 bulk_g2s(stage + kIdxOff, reinterpret_cast<const uint8_t *>(ev.eidx) + i_lo, i_hi - i_lo, &ring.full[stg]);
                 if (ebytes)
                     bulk_g2s(stage + kEscOff, reinterpret_cast<const uint8_t *>(ev.esc) + ((2u * e0) & ~15u), ebytes,
