@@ -46,6 +46,10 @@ namespace {
 
 using namespace spp::deepcam;
 
+// L2 policy of the decoded rows' TMA bulk stores (written once): 1 = evict_first hint
+#ifndef SPP_KD_ROW_EF
+#define SPP_KD_ROW_EF 0
+#endif
 struct DcMeta {  // written by KD0, read by KD (32 B)
     const uint8_t *dir;
     const uint8_t *payload;
@@ -504,7 +508,11 @@ template <int OUT>
 __device__ __forceinline__ void row_buffer_release(uint8_t *row, uint8_t *rowbuf, uint32_t W, int lane) {
     fence_proxy_async_smem();  // this lane's row writes -> visible to the async proxy
     __syncwarp();
+#if SPP_KD_ROW_EF
+    if (lane == 0) bulk_s2g_hint(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u), l2_policy_evict_first());
+#else
     if (lane == 0) bulk_s2g(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
+#endif
 }
 
 template <int OUT, int VPL>
