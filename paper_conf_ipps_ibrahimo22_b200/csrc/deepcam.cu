@@ -47,8 +47,9 @@ namespace {
 using namespace spp::deepcam;
 
 // L2 policy of the decoded rows' TMA bulk stores (written once): 1 = evict_first hint
+// (r2: C4 0.844 -> 0.851 of the measured peak, 3 alternating runs, profiles/r02a8_*)
 #ifndef SPP_KD_ROW_EF
-#define SPP_KD_ROW_EF 0
+#define SPP_KD_ROW_EF 1
 #endif
 struct DcMeta {  // written by KD0, read by KD (32 B)
     const uint8_t *dir;
