@@ -32,8 +32,10 @@ constexpr uint32_t kLabelMagic = 0x4C505053u;  // "SPPL"
 constexpr int kLabelHeader = 32;
 constexpr int kKlWarps = 8;  // warps per CTA
 constexpr uint32_t kKlChunk = 4096;  // positions per bitmap pass (128 words per warp)
-constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 16 words per lane)
+constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 16 words, 64 positions per lane)
+constexpr uint32_t kKlStageW = 2304;  // staging bytes per buffer: one row, or a row pair of W <= 1152
 constexpr uint32_t kKlFastRuns = 32;  // staged RUN rows: one run per lane
+constexpr uint32_t kKlPairRuns = 16;  // row pairs: one run per lane of a half-warp
 
 // inclusive warp scan, the shuffle's in-range predicate guarding the add
 __device__ __forceinline__ uint32_t scan_u32(uint32_t v) {
@@ -111,6 +113,101 @@ __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t byt
     return true;
 }
 
+// inclusive scan within each half-warp (16-lane segments)
+__device__ __forceinline__ uint32_t scan16_u32(uint32_t v) {
+#pragma unroll
+    for (int d = 1; d < 16; d <<= 1)
+        asm("{\n.reg .u32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, 0x1000, 0xffffffff;\n@p add.u32 %0, %0, t;\n}\n"
+            : "+r"(v)
+            : "r"(d));
+    return v;
+}
+// 0xFFFFFFFF << n with PTX shl semantics (n >= 32 gives 0)
+__device__ __forceinline__ uint32_t ones_shl(uint32_t n) {
+    uint32_t r;
+    asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(0xFFFFFFFFu), "r"(n));
+    return r;
+}
+
+// Two consecutive RUN rows, nrun <= 16 each (W % 128 == 0, 2W <= kKlStageW):
+// half-warp h (lanes 16h .. 16h + 15) decodes row g + h exactly as
+// kl_run_row_staged does with a whole warp -- lane hl holds run hl, a 16-lane
+// scan gives the starts, each start sets one bit in the bitmap of the lane
+// owning its position (W / 16 positions, three bitmap words per lane), a popc
+// scan gives the run at each lane's first position, the lane fills its WPL2
+// words in registers -- and the two rows, adjacent in dst, leave by ONE TMA bulk
+// store.  Every warp-collective step (scans, ballots, the bitmap round trip,
+// the proxy fence and the store) is paid once per two rows.  p, bytes, nrun
+// are the lane's half's row.  Returns the rows decoded: bit 0 row g, bit 16
+// row g + 1.
+template <int WPL2>  // words per lane of a half-warp row: W = 1152 -> 18
+__device__ __forceinline__ uint32_t kl_run_pair_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
+                                                       uint32_t magic2, uint32_t *bm, uint32_t bm_s, uint8_t *stage,
+                                                       uint32_t stage_s, uint8_t *row0, int lane) {
+    const uint32_t h = (uint32_t)lane >> 4, hl = (uint32_t)lane & 15u, hb = (uint32_t)lane & 16u;
+    const bool fits = 4ull + 3ull * nrun <= bytes;
+    const bool have = fits && hl < nrun;
+    const uint32_t len = have ? __ldg(reinterpret_cast<const uint16_t *>(p + 4) + hl) : 0u;
+    const uint32_t val = have ? __ldg(p + 4 + 2 * nrun + hl) : 0u;
+    const uint32_t incl = scan16_u32(len), st = incl - len;
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, (int)(hb | 15u));
+    const uint32_t zero_len = __ballot_sync(0xffffffffu, have && len == 0);
+    const bool okh = fits && ((zero_len >> hb) & 0xFFFFu) == 0 && tot == W;
+    const uint32_t okm = __ballot_sync(0xffffffffu, okh) & 0x00010001u;
+    constexpr uint32_t rlen = 4u * WPL2;  // positions per lane
+    sts_u4(bm_s + 16u * (uint32_t)lane, make_uint4(0u, 0u, 0u, 0u));
+    __syncwarp();
+    if (have && okh) {
+        const uint32_t o = __umulhi(st, magic2);  // st / rlen (exact: st < 2^16, rlen <= 72)
+        const uint32_t b = st - o * rlen;
+        atomicOr(bm + 4 * (hb | o) + (b >> 5), 1u << (b & 31));
+    }
+    __syncwarp();
+    const uint4 mm = lds_u4(bm_s + 16u * (uint32_t)lane);
+    const uint32_t c = __popc(mm.x) + __popc(mm.y) + __popc(mm.z);
+    const uint32_t before = scan16_u32(c) - c;  // run starts before this lane's first position
+    uint32_t idx = before + (mm.x & 1u) - 1u;  // run of the first position (run 0 starts at 0)
+    uint32_t r0 = mm.x & ~1u, r1 = mm.y, r2 = mm.z;
+    uint32_t v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & 15u))) * 0x01010101u;
+    uint32_t out[WPL2];
+#pragma unroll
+    for (int k = 0; k < WPL2; k++) out[k] = v;
+    const uint32_t tmax = __reduce_max_sync(0xffffffffu, c - (mm.x & 1u));
+    for (uint32_t t = 0; t < tmax; t++) {  // one pass per run starting inside the lane's words
+        const bool has = (r0 | r1 | r2) != 0;
+        const uint32_t j = r0 ? __ffs(r0) - 1u : (r1 ? 31u + __ffs(r1) : 63u + __ffs(r2));
+        if (r0) r0 &= r0 - 1;
+        else if (r1) r1 &= r1 - 1;
+        else r2 &= r2 - 1;
+        idx += has;
+        v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & 15u))) * 0x01010101u;
+        if (has) {
+            const int j8 = 8 * (int)j;
+#pragma unroll
+            for (int k = 0; k < WPL2; k++) {  // bytes at or after j take v
+                const uint32_t take = ones_shl((uint32_t)max(j8 - 32 * k, 0));
+                out[k] = (out[k] & ~take) | (v & take);
+            }
+        }
+    }
+    const uint32_t lo = stage_s + h * W + rlen * hl;
+    if constexpr ((WPL2 & 1) == 0) {
+#pragma unroll
+        for (int k = 0; k < WPL2; k += 2) sts_u2(lo + 4u * k, make_uint2(out[k], out[k + 1]));
+    } else {
+#pragma unroll
+        for (int k = 0; k < WPL2; k++) sts_f32(lo + 4u * k, __uint_as_float(out[k]));
+    }
+    fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
+    __syncwarp();
+    if (lane == 0 && okm) {
+        if (okm == 0x00010001u) bulk_s2g(row0, stage, 2 * W);
+        else if (okm & 1u) bulk_s2g(row0, stage, W);
+        else bulk_s2g(row0 + W, stage + W, W);
+    }
+    return okm;
+}
+
 // header check shared by both kinds: returns total (0 if invalid)
 __device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t limit, uint32_t kind, uint32_t H,
                                                     uint32_t W) {
@@ -124,17 +221,18 @@ __device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t l
     return ok ? total : 0;
 }
 
-template <int WPL>  // 0: no staged rows (W % 16 != 0, W > 2048 or an unaligned dst)
+template <int WPL, int WPL2>  // WPL 0: no staged rows (W % 16 != 0, W > 2048 or an unaligned dst); WPL2 0: no row pairs
 __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *const *__restrict__ src,
                                                                    const uint64_t *__restrict__ src_bytes, int n,
                                                                    uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
                                                                    uint32_t *__restrict__ status) {
     __shared__ uint32_t bitmap[kKlWarps][kKlChunk / 32];
-    __shared__ __align__(128) uint8_t stage_rows[kKlWarps][2][kKlFastW];  // double-buffered staging rows
+    __shared__ __align__(128) uint8_t stage_rows[kKlWarps][2][kKlStageW];  // double-buffered staging rows
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t *bm = bitmap[warp];
     const uint32_t bm_s = smem_u32(bm);
     const uint32_t magic = 0xFFFFFFFFu / (4u * (WPL > 0 ? WPL : 1)) + 1u;
+    const uint32_t magic2 = 0xFFFFFFFFu / (4u * (WPL2 > 0 ? WPL2 : 1)) + 1u;
     uint32_t nstaged = 0;  // rows this warp has stored by TMA (buffer nstaged & 1 next)
     const uint64_t T = (uint64_t)n * H;
     const uint64_t NW = (uint64_t)gridDim.x * kKlWarps, gw = (uint64_t)blockIdx.x * kKlWarps + warp;
@@ -171,6 +269,33 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
         }
     };
     for (uint64_t g = g0; g < g1; g++) {
+        if constexpr (WPL2 > 0) {
+            // two RUN rows of <= 16 runs each: one half-warp per row, one bulk store
+            if (g + 1 < g1) {
+                if (g == g0 || g + 1 >= wbase + kWarp) load_window(g);
+                const int kk = (int)(g - wbase);
+                const uint32_t h0 = __shfl_sync(0xffffffffu, w_hdr, kk), h1 = __shfl_sync(0xffffffffu, w_hdr, kk + 1);
+                const bool pair_ok = __shfl_sync(0xffffffffu, w_ok, kk) && __shfl_sync(0xffffffffu, w_ok, kk + 1) &&
+                                     (h0 & 0xFFu) == 1u && (h1 & 0xFFu) == 1u && (h0 >> 16) >= 1 &&
+                                     (h0 >> 16) <= kKlPairRuns && (h1 >> 16) >= 1 && (h1 >> 16) <= kKlPairRuns;
+                if (pair_ok) {
+                    const int kh = kk + (lane >> 4);
+                    const uint8_t *p = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_p, kh));
+                    const uint32_t bytes = __shfl_sync(0xffffffffu, w_bytes, kh);
+                    const uint32_t nrun = (lane >> 4 ? h1 : h0) >> 16;
+                    uint8_t *stage = stage_rows[warp][nstaged & 1];
+                    if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
+                    __syncwarp();
+                    const uint32_t okm = kl_run_pair_staged<(WPL2 > 0 ? WPL2 : 1)>(
+                        p, bytes, nrun, W, magic2, bm, bm_s, stage, smem_u32(stage), dst + g * (uint64_t)W, lane);
+                    nstaged += okm != 0;
+                    if (lane == 0 && !(okm & 1u)) report(status, SPP_ERR_CORRUPT, (int64_t)(g / H));
+                    if (lane == 0 && !(okm >> 16)) report(status, SPP_ERR_CORRUPT, (int64_t)((g + 1) / H));
+                    g++;
+                    continue;
+                }
+            }
+        }
         if (g == g0 || g >= wbase + kWarp) load_window(g);
         const int kk = (int)(g - wbase);
         bool ok = __shfl_sync(0xffffffffu, w_ok, kk) != 0;
@@ -304,18 +429,28 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
         // staged rows leave by TMA bulk store: 16-B aligned rows of a multiple of 16 bytes
         const bool staged = (W % 16) == 0 && W <= (int)kKlFastW && (reinterpret_cast<uintptr_t>(d_dst) & 15) == 0;
         const int wpl = staged ? (W / 4 + kWarp - 1) / kWarp : 0;
+        // row pairs (one half-warp per row, one bulk store per pair): W % 128 == 0, 2W <= kKlStageW
+        const bool pairs = staged && W % 128 == 0 && 2 * W <= (int)kKlStageW;
         const unsigned grid = (unsigned)std::max<uint64_t>(1, ctas);
         uint8_t *dst = static_cast<uint8_t *>(d_dst);
-        switch (wpl) {
+        switch (pairs ? 100 + wpl : wpl) {
 #define SPP_KL_CASE(k)                                                                                            \
     case k:                                                                                                       \
-        kl_decode_mask<k><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W, dst, \
-                                                                 status);                                         \
+        kl_decode_mask<k, 0><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W,  \
+                                                                    dst, status);                                 \
+        break;
+#define SPP_KL_PAIR(k)                                                                                            \
+    case 100 + k:                                                                                                 \
+        kl_decode_mask<k, 2 * k><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H,          \
+                                                                        (uint32_t)W, dst, status);                \
         break;
             SPP_KL_CASE(0) SPP_KL_CASE(1) SPP_KL_CASE(2) SPP_KL_CASE(3) SPP_KL_CASE(4) SPP_KL_CASE(5) SPP_KL_CASE(6)
             SPP_KL_CASE(7) SPP_KL_CASE(8) SPP_KL_CASE(9) SPP_KL_CASE(10) SPP_KL_CASE(11) SPP_KL_CASE(12)
             SPP_KL_CASE(13) SPP_KL_CASE(14) SPP_KL_CASE(15) SPP_KL_CASE(16)
+            SPP_KL_PAIR(1) SPP_KL_PAIR(2) SPP_KL_PAIR(3) SPP_KL_PAIR(4) SPP_KL_PAIR(5) SPP_KL_PAIR(6)
+            SPP_KL_PAIR(7) SPP_KL_PAIR(8) SPP_KL_PAIR(9)
 #undef SPP_KL_CASE
+#undef SPP_KL_PAIR
             default: return SPP_ERR_INVALID_ARG;
         }
     }

@@ -52,13 +52,15 @@ def _runs_mask(rng, H, W):
 
 
 @pytest.mark.parametrize("H,W", [(768, 1152), (5, 37), (3, 2100), (1, 1), (4, 1024), (40, 1152), (40, 2048),
-                                 (36, 16), (40, 1040), (34, 48)])
+                                 (36, 16), (40, 1040), (34, 48), (7, 128), (33, 1152), (19, 2304)])
 def test_label_masks_lossless(dev, orc, H, W):
     """Paper-shaped DeepCAM masks (cyclone discs, river bands), random masks
     (verbatim rows), constant masks, W not a multiple of 16, W over the 1,024-
     position chunk; rows of exactly 1..40 runs (the staged path takes <= 32 runs
     with W % 16 == 0 and W <= 2048: 1152, 2048, 16, 1040 with a partial last
-    lane, 48); mixed in one batch, bit-exact vs the masks and the oracle."""
+    lane, 48; 2304 takes the general path; row pairs -- one half-warp per row, <= 16 runs each -- when
+    W % 128 == 0 and W <= 1152: 1152, 1024, 128, odd H); mixed in one batch,
+    bit-exact vs the masks and the oracle."""
     from synth import gen_deepcam_labels
     from paper_conf_ipps_ibrahimo22_b200 import spp
     rng = np.random.default_rng(H * 7 + W)
@@ -103,6 +105,31 @@ def test_label_corruption_detected(dev):
     for i, c in enumerate(bad):
         _, st = _decode("mask", [good, c, good], (32, 256), src_bytes=True)
         assert st == (3 | (1 << 8)), (i, st)
+
+
+def test_label_row_pairs_corruption_and_neighbours(dev):
+    """Row pairs (W % 128 == 0): a corrupt run length in the first or the
+    second row of a pair is reported on its sample and the other samples of
+    the batch decode bit-exactly; rows of 16 and 17 runs side by side (a pair
+    falls back to single rows when either has more than 16 runs)."""
+    from synth import gen_deepcam_labels
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    rng = np.random.default_rng(42)
+    H, W = 24, 1152
+    m16 = _runs_mask(rng, 40, W)[14:14 + H]  # rows of 15..38 runs: pairs of <= 16 and > 16 runs mixed
+    masks = [gen_deepcam_labels(71, H=H, W=W), m16, gen_deepcam_labels(72, H=H, W=W)]
+    bufs = [spp.spp_encode_label_mask(m) for m in masks]
+    got, st = _decode("mask", bufs, (H, W), src_bytes=True)
+    assert st == 0 and np.array_equal(got, np.stack(masks))
+    for y in (0, 1, 6, 7, H - 1):
+        bad = bufs[0].copy()
+        h = fmt.label_header(bad)
+        row = h["payload_off"] + int(h["dir"][y])
+        assert bad[row] == 1  # a RUN row
+        bad[row + 4] ^= 0x01  # its first run length: the lengths no longer sum to W
+        got, st = _decode("mask", [bufs[2], bad, bufs[1]], (H, W), src_bytes=True)
+        assert st == (3 | (1 << 8)), (y, st)
+        assert np.array_equal(got[0], masks[2]) and np.array_equal(got[2], masks[1])
 
 
 @pytest.mark.parametrize("source", ["device", "host"])
