@@ -36,6 +36,16 @@ constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 
 constexpr uint32_t kKlStageW = 2304;  // staging bytes per buffer: one row, or a row pair of W <= 1152
 constexpr uint32_t kKlFastRuns = 32;  // staged RUN rows: one run per lane
 constexpr uint32_t kKlPairRuns = 16;  // row pairs: one run per lane of a half-warp
+#ifndef SPP_KL_ROW_EF  // 1: the staged rows' TMA bulk stores carry an L2 evict_first hint (+4%, r02b2)
+#define SPP_KL_ROW_EF 1
+#endif
+__device__ __forceinline__ void kl_store(void *dst, const void *src, uint32_t bytes) {
+#if SPP_KL_ROW_EF
+    bulk_s2g_hint(dst, src, bytes, l2_policy_evict_first());
+#else
+    bulk_s2g(dst, src, bytes);
+#endif
+}
 
 // inclusive warp scan, the shuffle's in-range predicate guarding the add
 __device__ __forceinline__ uint32_t scan_u32(uint32_t v) {
@@ -109,7 +119,7 @@ __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t byt
         if ((uint32_t)k < nw) sts_f32(stage_s + lo + 4u * k, __uint_as_float(out[k]));
     fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
     __syncwarp();
-    if (lane == 0) bulk_s2g(row, stage, W);
+    if (lane == 0) kl_store(row, stage, W);
     return true;
 }
 
@@ -201,9 +211,9 @@ __device__ __forceinline__ uint32_t kl_run_pair_staged(const uint8_t *p, uint32_
     fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
     __syncwarp();
     if (lane == 0 && okm) {
-        if (okm == 0x00010001u) bulk_s2g(row0, stage, 2 * W);
-        else if (okm & 1u) bulk_s2g(row0, stage, W);
-        else bulk_s2g(row0 + W, stage + W, W);
+        if (okm == 0x00010001u) kl_store(row0, stage, 2 * W);
+        else if (okm & 1u) kl_store(row0, stage, W);
+        else kl_store(row0 + W, stage + W, W);
     }
     return okm;
 }
@@ -425,25 +435,17 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
                                                                            static_cast<float *>(d_dst), status);
     } else {
         const uint64_t rows = (uint64_t)n * H;
-        const uint64_t ctas = std::min<uint64_t>((uint64_t)dp.sms * 8, (rows + kKlWarps - 1) / kKlWarps);
         // staged rows leave by TMA bulk store: 16-B aligned rows of a multiple of 16 bytes
         const bool staged = (W % 16) == 0 && W <= (int)kKlFastW && (reinterpret_cast<uintptr_t>(d_dst) & 15) == 0;
         const int wpl = staged ? (W / 4 + kWarp - 1) / kWarp : 0;
         // row pairs (one half-warp per row, one bulk store per pair): W % 128 == 0, 2W <= kKlStageW
         const bool pairs = staged && W % 128 == 0 && 2 * W <= (int)kKlStageW;
-        const unsigned grid = (unsigned)std::max<uint64_t>(1, ctas);
-        uint8_t *dst = static_cast<uint8_t *>(d_dst);
+        void (*kern)(const void *const *, const uint64_t *, int, uint32_t, uint32_t, uint8_t *, uint32_t *) = nullptr;
         switch (pairs ? 100 + wpl : wpl) {
-#define SPP_KL_CASE(k)                                                                                            \
-    case k:                                                                                                       \
-        kl_decode_mask<k, 0><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W,  \
-                                                                    dst, status);                                 \
-        break;
-#define SPP_KL_PAIR(k)                                                                                            \
-    case 100 + k:                                                                                                 \
-        kl_decode_mask<k, 2 * k><<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H,          \
-                                                                        (uint32_t)W, dst, status);                \
-        break;
+#define SPP_KL_CASE(k) \
+    case k: kern = kl_decode_mask<k, 0>; break;
+#define SPP_KL_PAIR(k) \
+    case 100 + k: kern = kl_decode_mask<k, 2 * k>; break;
             SPP_KL_CASE(0) SPP_KL_CASE(1) SPP_KL_CASE(2) SPP_KL_CASE(3) SPP_KL_CASE(4) SPP_KL_CASE(5) SPP_KL_CASE(6)
             SPP_KL_CASE(7) SPP_KL_CASE(8) SPP_KL_CASE(9) SPP_KL_CASE(10) SPP_KL_CASE(11) SPP_KL_CASE(12)
             SPP_KL_CASE(13) SPP_KL_CASE(14) SPP_KL_CASE(15) SPP_KL_CASE(16)
@@ -453,6 +455,13 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
 #undef SPP_KL_PAIR
             default: return SPP_ERR_INVALID_ARG;
         }
+        // 8 CTAs per SM: about two waves of the pair instance (4 resident per SM); measured
+        // 3% faster than one resident wave (profiles/r02b2_*): later CTAs fill SMs whose
+        // first CTAs finished early
+        const uint64_t ctas = std::min<uint64_t>((uint64_t)dp.sms * 8, (rows + kKlWarps - 1) / kKlWarps);
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, ctas);
+        kern<<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W,
+                                                    static_cast<uint8_t *>(d_dst), status);
     }
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }
