@@ -51,6 +51,7 @@ using namespace spp::deepcam;
 #ifndef SPP_KD_ROW_EF
 #define SPP_KD_ROW_EF 1
 #endif
+constexpr uint64_t kRowEfBytes = 64ull << 20;  // launches writing more than this (half of L2) use evict_first
 struct DcMeta {  // written by KD0, read by KD (32 B)
     const uint8_t *dir;
     const uint8_t *payload;
@@ -506,20 +507,16 @@ __device__ __forceinline__ void row_buffer_acquire(int lane) {
     __syncwarp();
 }
 template <int OUT>
-__device__ __forceinline__ void row_buffer_release(uint8_t *row, uint8_t *rowbuf, uint32_t W, int lane) {
+__device__ __forceinline__ void row_buffer_release(uint8_t *row, uint8_t *rowbuf, uint32_t W, int lane, uint64_t rpol) {
     fence_proxy_async_smem();  // this lane's row writes -> visible to the async proxy
     __syncwarp();
-#if SPP_KD_ROW_EF
-    if (lane == 0) bulk_s2g_hint(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u), l2_policy_evict_first());
-#else
-    if (lane == 0) bulk_s2g(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u));
-#endif
+    if (lane == 0) bulk_s2g_hint(row, rowbuf, W * (OUT == SPP_OUT_F32 ? 4u : 2u), rpol);
 }
 
 template <int OUT, int VPL>
 __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes, uint32_t W, uint32_t *bbits,
                                                     uint32_t nbw, float shv, float scv, uint8_t *row, uint8_t *rowbuf,
-                                                    int lane) {
+                                                    int lane, uint64_t rpol) {
     constexpr bool STAGED = VPL == 36;  // one pass per line (W = 32 * VPL): row staged in rowbuf, one TMA bulk store
     const uint32_t hdr = *reinterpret_cast<const uint32_t *>(buf);
     const uint32_t nseg = hdr >> 16;
@@ -650,7 +647,7 @@ __device__ __forceinline__ bool decode_line_aligned(uint8_t *buf, uint32_t bytes
             emit_vpl<OUT, VPL>(row, p0, y);
         }
     }
-    if constexpr (STAGED) row_buffer_release<OUT>(row, rowbuf, W, lane);
+    if constexpr (STAGED) row_buffer_release<OUT>(row, rowbuf, W, lane, rpol);
     return true;
 }
 
@@ -662,14 +659,14 @@ template <int OUT, bool RAWSEG>  // RAWSEG: a mode-3 line (FORMAT.md 2.7); mode-
 __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t buf_s, uint32_t hdr, uint32_t bytes,
                                                     uint32_t W, uint32_t *bbits, uint32_t nbw, float shv, float scv,
                                                     uint8_t *row, uint8_t *rowbuf, uint32_t rowbuf_s, uint32_t rep_s,
-                                                    int lane) {
+                                                    int lane, uint64_t rpol) {
     constexpr int VPL = 36;
     const uint32_t nseg = hdr >> 16;
     // mode 3 (FORMAT.md 2.7) also allows RAW segments; with A = 36 and W = 1152
     // it never has more than 32 segments, so the fallback sees only mode 1
     constexpr uint32_t max_kind = RAWSEG ? kRawSeg : kDiff;
     if (nseg > (uint32_t)kWarp)
-        return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, rowbuf, lane);
+        return decode_line_aligned<OUT, VPL>(buf, bytes, W, bbits, nbw, shv, scv, row, rowbuf, lane, rpol);
     if (nseg < 1 || 4u + 8u * nseg > bytes) return false;
     const uint32_t dl_s = buf_s + 4 + 8 * nseg;
     const bool have = (uint32_t)lane < nseg;
@@ -759,7 +756,7 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t buf_s
     }
     row_buffer_acquire(lane);
     stage_vpl<OUT, VPL>(rowbuf_s + p0 * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
-    row_buffer_release<OUT>(row, rowbuf, W, lane);
+    row_buffer_release<OUT>(row, rowbuf, W, lane, rpol);
     return true;
 }
 
@@ -770,7 +767,8 @@ __device__ __forceinline__ bool decode_line_onepass(uint8_t *buf, uint32_t buf_s
 // leaves like a one-pass SEG row (staged in the slot, one TMA bulk store).
 template <int OUT>
 __device__ __forceinline__ bool decode_line_raw16_onepass(uint8_t *buf, uint32_t bytes, uint32_t W, float shv,
-                                                          float scv, uint8_t *row, uint8_t *rowbuf, int lane) {
+                                                          float scv, uint8_t *row, uint8_t *rowbuf, int lane,
+                                                          uint64_t rpol) {
     constexpr int VPL = 36;
     if (16u + 2u * W > bytes) return false;
     const uint32_t src = smem_u32(buf + 16) + 2u * VPL * (uint32_t)lane;
@@ -789,7 +787,7 @@ __device__ __forceinline__ bool decode_line_raw16_onepass(uint8_t *buf, uint32_t
     }
     row_buffer_acquire(lane);
     stage_vpl<OUT, VPL>(smem_u32(rowbuf) + VPL * (uint32_t)lane * (uint32_t)(OUT == SPP_OUT_F32 ? 4 : 2), y);
-    row_buffer_release<OUT>(row, rowbuf, W, lane);
+    row_buffer_release<OUT>(row, rowbuf, W, lane, rpol);
     return true;
 }
 
@@ -945,7 +943,7 @@ template <int OUT, bool VEC, int VPL, bool RAWSEG>  // RAWSEG: opts.raw_segments
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SPP_KD_WS_MINB) kd_decode_ws(
     const DcMeta *__restrict__ meta, int n, uint32_t L, uint32_t H, uint32_t W, const float *__restrict__ shift,
     const float *__restrict__ scale, uint8_t *__restrict__ dst, uint32_t cap, uint32_t rowb, uint32_t nwords,
-    uint32_t warp_bytes, uint32_t *__restrict__ status) {
+    uint32_t warp_bytes, uint32_t *__restrict__ status, uint32_t row_ef) {
     extern __shared__ __align__(16) uint8_t smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int wpc = (int)(blockDim.x >> 5) - 1;  // consumer warps; warp wpc produces
@@ -1121,6 +1119,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
     const uint32_t nsb = nwords / 2;  // words of the start bitmap (and of its prefix counts)
     const uint32_t rep_s = smem_u32(smem_raw + (size_t)wpc * warp_bytes);  // 48 B of 0x80 (producer-filled)
     const uint32_t base_s = smem_u32(base), rowbuf_s = smem_u32(rowbuf);      // shared addresses, hoisted
+    // L2 policy of the row stores: evict_first when the launch writes far more than
+    // L2 holds (batches: C4 +0.8%, profiles/r02a8_*), normal otherwise (a single
+    // sample's output stays L2-resident for its consumer)
+    uint64_t rpol;
+    if (row_ef) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(rpol));
+    else asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(rpol));
     uint32_t fph = 0;  // bit s: parity of slot s's next full phase
     uint32_t s = 0;
     const uint32_t nlines = (uint32_t)(g_end - g_begin);  // < 2^32: lines of one warp
@@ -1152,17 +1156,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kWsWarps * kWarp, SP
             bool ok;
             if (RAWSEG && mode == kModeRaw16) {
                 if constexpr (RAWSEG && VPL == 36)
-                    ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, rowbuf, lane);
+                    ok = decode_line_raw16_onepass<OUT>(buf, bytes, W, shv, scv, row, rowbuf, lane, rpol);
             } else if (VEC && al == (uint32_t)VPL && (mode == kModeSeg || (RAWSEG && mode == kModeSegRaw))) {
                 if constexpr (VPL == 36) {
                     if (!RAWSEG || mode == kModeSeg)
                         ok = decode_line_onepass<OUT, false>(buf, buf_s, hdr, bytes, W, sbits, nbw, shv, scv, row,
-                                                             rowbuf, rowbuf_s, rep_s, lane);
+                                                             rowbuf, rowbuf_s, rep_s, lane, rpol);
                     else
                         ok = decode_line_onepass<OUT, true>(buf, buf_s, hdr, bytes, W, sbits, nbw, shv, scv, row,
-                                                            rowbuf, rowbuf_s, rep_s, lane);
+                                                            rowbuf, rowbuf_s, rep_s, lane, rpol);
                 }
-                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane);
+                else ok = decode_line_aligned<OUT, VPL>(buf, bytes, W, sbits, nbw, shv, scv, row, rowbuf, lane, rpol);
             } else {
                 ok = decode_line<OUT, VEC>(buf, bytes, W, al, sbits, wpre, nsb, shv, scv, row, lane);
             }
@@ -1221,10 +1225,12 @@ spp_status launch_kd_ws(const DcMeta *meta, int n, void *d_dst, const spp_decode
     const uint64_t max_ctas = (uint64_t)dp.sms * occ;
     // st.async needs a cluster of at least 2 CTAs (they never touch each other's memory): even grid
     int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(max_ctas, (lines + wpc - 1) / wpc));
+    // row stores evict_first when the launch's output far exceeds L2 (SPP_KD_ROW_EF)
+    const uint32_t row_ef = SPP_KD_ROW_EF && lines * W * (OUT == SPP_OUT_F32 ? 4u : 2u) > kRowEfBytes;
     grid += grid & 1;
     kern<<<grid, (wpc + 1) * kWarp, smem, stream>>>(meta, n, (uint32_t)(o.C * o.H), (uint32_t)o.H, W, o.shift,
                                                      o.scale, static_cast<uint8_t *>(d_dst), cap, rowb, nwords,
-                                                     warp_bytes, o.status);
+                                                     warp_bytes, o.status, row_ef);
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }
 
