@@ -36,15 +36,15 @@ constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 
 constexpr uint32_t kKlStageW = 2304;  // staging bytes per buffer: one row, or a row pair of W <= 1152
 constexpr uint32_t kKlFastRuns = 32;  // staged RUN rows: one run per lane
 constexpr uint32_t kKlPairRuns = 16;  // row pairs: one run per lane of a half-warp
-#ifndef SPP_KL_ROW_EF  // 1: the staged rows' TMA bulk stores carry an L2 evict_first hint (+4%, r02b2)
+// L2 policy of the staged rows' TMA bulk stores: evict_first when the launch writes
+// more than kRowEfBytes (+4% on 2048 masks, profiles/r02b2_*, r02b3_*), normal below
+// (a loader batch's labels stay L2-resident for their consumer)
+#ifndef SPP_KL_ROW_EF
 #define SPP_KL_ROW_EF 1
 #endif
-__device__ __forceinline__ void kl_store(void *dst, const void *src, uint32_t bytes) {
-#if SPP_KL_ROW_EF
-    bulk_s2g_hint(dst, src, bytes, l2_policy_evict_first());
-#else
-    bulk_s2g(dst, src, bytes);
-#endif
+constexpr uint64_t kRowEfBytes = 64ull << 20;
+__device__ __forceinline__ void kl_store(void *dst, const void *src, uint32_t bytes, uint64_t pol) {
+    bulk_s2g_hint(dst, src, bytes, pol);
 }
 
 // inclusive warp scan, the shuffle's in-range predicate guarding the add
@@ -69,7 +69,8 @@ __device__ __forceinline__ void bulk_wait_read_1() { asm volatile("cp.async.bulk
 template <int WPL>  // words (4 positions) per lane: W = 1152 -> 9
 __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
                                                   uint32_t magic, uint32_t *bm, uint32_t bm_s,
-                                                  uint8_t *stage, uint32_t stage_s, uint8_t *row, int lane) {
+                                                  uint8_t *stage, uint32_t stage_s, uint8_t *row, int lane,
+                                                  uint64_t pol) {
     if (4ull + 3ull * nrun > bytes) return false;
     const bool have = (uint32_t)lane < nrun;
     const uint32_t len = have ? __ldg(reinterpret_cast<const uint16_t *>(p + 4) + lane) : 0u;
@@ -119,7 +120,7 @@ __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t byt
         if ((uint32_t)k < nw) sts_f32(stage_s + lo + 4u * k, __uint_as_float(out[k]));
     fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
     __syncwarp();
-    if (lane == 0) kl_store(row, stage, W);
+    if (lane == 0) kl_store(row, stage, W, pol);
     return true;
 }
 
@@ -153,7 +154,7 @@ __device__ __forceinline__ uint32_t ones_shl(uint32_t n) {
 template <int WPL2>  // words per lane of a half-warp row: W = 1152 -> 18
 __device__ __forceinline__ uint32_t kl_run_pair_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
                                                        uint32_t magic2, uint32_t *bm, uint32_t bm_s, uint8_t *stage,
-                                                       uint32_t stage_s, uint8_t *row0, int lane) {
+                                                       uint32_t stage_s, uint8_t *row0, int lane, uint64_t pol) {
     const uint32_t h = (uint32_t)lane >> 4, hl = (uint32_t)lane & 15u, hb = (uint32_t)lane & 16u;
     const bool fits = 4ull + 3ull * nrun <= bytes;
     const bool have = fits && hl < nrun;
@@ -211,9 +212,9 @@ __device__ __forceinline__ uint32_t kl_run_pair_staged(const uint8_t *p, uint32_
     fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
     __syncwarp();
     if (lane == 0 && okm) {
-        if (okm == 0x00010001u) kl_store(row0, stage, 2 * W);
-        else if (okm & 1u) kl_store(row0, stage, W);
-        else kl_store(row0 + W, stage + W, W);
+        if (okm == 0x00010001u) kl_store(row0, stage, 2 * W, pol);
+        else if (okm & 1u) kl_store(row0, stage, W, pol);
+        else kl_store(row0 + W, stage + W, W, pol);
     }
     return okm;
 }
@@ -235,7 +236,7 @@ template <int WPL, int WPL2>  // WPL 0: no staged rows (W % 16 != 0, W > 2048 or
 __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *const *__restrict__ src,
                                                                    const uint64_t *__restrict__ src_bytes, int n,
                                                                    uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
-                                                                   uint32_t *__restrict__ status) {
+                                                                   uint32_t *__restrict__ status, uint32_t row_ef) {
     __shared__ uint32_t bitmap[kKlWarps][kKlChunk / 32];
     __shared__ __align__(128) uint8_t stage_rows[kKlWarps][2][kKlStageW];  // double-buffered staging rows
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -244,6 +245,9 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
     const uint32_t magic = 0xFFFFFFFFu / (4u * (WPL > 0 ? WPL : 1)) + 1u;
     const uint32_t magic2 = 0xFFFFFFFFu / (4u * (WPL2 > 0 ? WPL2 : 1)) + 1u;
     uint32_t nstaged = 0;  // rows this warp has stored by TMA (buffer nstaged & 1 next)
+    uint64_t pol;
+    if (row_ef) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    else asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
     const uint64_t T = (uint64_t)n * H;
     const uint64_t NW = (uint64_t)gridDim.x * kKlWarps, gw = (uint64_t)blockIdx.x * kKlWarps + warp;
     const uint64_t g0 = gw * T / NW, g1 = (gw + 1) * T / NW;
@@ -297,7 +301,7 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                     if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
                     __syncwarp();
                     const uint32_t okm = kl_run_pair_staged<(WPL2 > 0 ? WPL2 : 1)>(
-                        p, bytes, nrun, W, magic2, bm, bm_s, stage, smem_u32(stage), dst + g * (uint64_t)W, lane);
+                        p, bytes, nrun, W, magic2, bm, bm_s, stage, smem_u32(stage), dst + g * (uint64_t)W, lane, pol);
                     nstaged += okm != 0;
                     if (lane == 0 && !(okm & 1u)) report(status, SPP_ERR_CORRUPT, (int64_t)(g / H));
                     if (lane == 0 && !(okm >> 16)) report(status, SPP_ERR_CORRUPT, (int64_t)((g + 1) / H));
@@ -330,7 +334,7 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
             if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
             __syncwarp();
             ok = kl_run_row_staged<(WPL > 0 ? WPL : 1)>(p, (uint32_t)bytes, hdr >> 16, W, magic, bm, bm_s, stage, smem_u32(stage),
-                                        row, lane);
+                                        row, lane, pol);
             nstaged += ok;
         } else if (ok && mode == 1) {  // maximal runs
             const uint32_t nrun = hdr >> 16;
@@ -440,7 +444,8 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
         const int wpl = staged ? (W / 4 + kWarp - 1) / kWarp : 0;
         // row pairs (one half-warp per row, one bulk store per pair): W % 128 == 0, 2W <= kKlStageW
         const bool pairs = staged && W % 128 == 0 && 2 * W <= (int)kKlStageW;
-        void (*kern)(const void *const *, const uint64_t *, int, uint32_t, uint32_t, uint8_t *, uint32_t *) = nullptr;
+        void (*kern)(const void *const *, const uint64_t *, int, uint32_t, uint32_t, uint8_t *, uint32_t *,
+                     uint32_t) = nullptr;
         switch (pairs ? 100 + wpl : wpl) {
 #define SPP_KL_CASE(k) \
     case k: kern = kl_decode_mask<k, 0>; break;
@@ -460,8 +465,9 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
         // first CTAs finished early
         const uint64_t ctas = std::min<uint64_t>((uint64_t)dp.sms * 8, (rows + kKlWarps - 1) / kKlWarps);
         const unsigned grid = (unsigned)std::max<uint64_t>(1, ctas);
+        const uint32_t row_ef = SPP_KL_ROW_EF && rows * (uint64_t)W > kRowEfBytes;
         kern<<<grid, kKlWarps * kWarp, 0, stream>>>(d_src, src_bytes, n, (uint32_t)H, (uint32_t)W,
-                                                    static_cast<uint8_t *>(d_dst), status);
+                                                    static_cast<uint8_t *>(d_dst), status, row_ef);
     }
     return cudaGetLastError() == cudaSuccess ? SPP_OK : SPP_ERR_CUDA;
 }
