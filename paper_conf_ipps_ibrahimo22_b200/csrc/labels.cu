@@ -20,6 +20,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <type_traits>
 
 #include "common.cuh"
 #include "spp_format.h"
@@ -36,6 +37,12 @@ constexpr uint32_t kKlFastW = 2048;  // staged rows: W % 16 == 0, W <= 2048 (<= 
 constexpr uint32_t kKlStageW = 2304;  // staging bytes per buffer: one row, or a row pair of W <= 1152
 constexpr uint32_t kKlFastRuns = 32;  // staged RUN rows: one run per lane
 constexpr uint32_t kKlPairRuns = 16;  // row pairs: one run per lane of a half-warp
+#ifndef SPP_KL_GROUP_MINB  // CTAs per SM the row-group instances' registers target
+#define SPP_KL_GROUP_MINB 4
+#endif
+#ifndef SPP_KL_QUADS  // 1: try 4-row groups (<= 8 runs per row) before pairs (measured 2.4% slower: r02b9)
+#define SPP_KL_QUADS 0
+#endif
 // L2 policy of the staged rows' TMA bulk stores: evict_first when the launch writes
 // more than kRowEfBytes (+4% on 2048 masks, profiles/r02b2_*, r02b3_*), normal below
 // (a loader batch's labels stay L2-resident for their consumer)
@@ -124,13 +131,14 @@ __device__ __forceinline__ bool kl_run_row_staged(const uint8_t *p, uint32_t byt
     return true;
 }
 
-// inclusive scan within each half-warp (16-lane segments)
-__device__ __forceinline__ uint32_t scan16_u32(uint32_t v) {
+// inclusive scan within each LPR-lane segment of the warp (LPR = 16: half-warps, 8: quarters)
+template <int LPR>
+__device__ __forceinline__ uint32_t scan_seg_u32(uint32_t v) {
 #pragma unroll
-    for (int d = 1; d < 16; d <<= 1)
-        asm("{\n.reg .u32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, 0x1000, 0xffffffff;\n@p add.u32 %0, %0, t;\n}\n"
+    for (int d = 1; d < LPR; d <<= 1)
+        asm("{\n.reg .u32 t;\n.reg .pred p;\nshfl.sync.up.b32 t|p, %0, %1, %2, 0xffffffff;\n@p add.u32 %0, %0, t;\n}\n"
             : "+r"(v)
-            : "r"(d));
+            : "r"(d), "n"((32 - LPR) << 8));
     return v;
 }
 // 0xFFFFFFFF << n with PTX shl semantics (n >= 32 gives 0)
@@ -140,81 +148,98 @@ __device__ __forceinline__ uint32_t ones_shl(uint32_t n) {
     return r;
 }
 
-// Two consecutive RUN rows, nrun <= 16 each (W % 128 == 0, 2W <= kKlStageW):
-// half-warp h (lanes 16h .. 16h + 15) decodes row g + h exactly as
-// kl_run_row_staged does with a whole warp -- lane hl holds run hl, a 16-lane
-// scan gives the starts, each start sets one bit in the bitmap of the lane
-// owning its position (W / 16 positions, three bitmap words per lane), a popc
-// scan gives the run at each lane's first position, the lane fills its WPL2
-// words in registers -- and the two rows, adjacent in dst, leave by ONE TMA bulk
-// store.  Every warp-collective step (scans, ballots, the bitmap round trip,
-// the proxy fence and the store) is paid once per two rows.  p, bytes, nrun
-// are the lane's half's row.  Returns the rows decoded: bit 0 row g, bit 16
-// row g + 1.
-template <int WPL2>  // words per lane of a half-warp row: W = 1152 -> 18
-__device__ __forceinline__ uint32_t kl_run_pair_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
-                                                       uint32_t magic2, uint32_t *bm, uint32_t bm_s, uint8_t *stage,
-                                                       uint32_t stage_s, uint8_t *row0, int lane, uint64_t pol) {
-    const uint32_t h = (uint32_t)lane >> 4, hl = (uint32_t)lane & 15u, hb = (uint32_t)lane & 16u;
+// G consecutive RUN rows (G = 2 or 4), at most 32/G runs each (W % 128 == 0,
+// G W <= 2 kKlStageW): each LPR = 32/G-lane segment of the warp decodes one
+// row exactly as kl_run_row_staged does with a whole warp -- lane hl holds run
+// hl, a segment scan gives the starts, each start sets one bit in the bitmap
+// of the lane owning its position (W / LPR positions per lane), a popc scan
+// gives the run at each lane's first position, the lane fills its WPLG words
+// in registers -- and the G rows, adjacent in dst, leave by ONE TMA bulk store.
+// Every warp-collective step (scans, ballots, the bitmap round trip, the proxy
+// fence and the store) is paid once per G rows.  p, bytes, nrun are the lane's
+// segment's row.  Returns the rows decoded: bit LPR r set = row g + r.
+template <int G, int WPLG>  // W = 1152: G = 2 -> 18 words per lane, G = 4 -> 36
+__device__ __forceinline__ uint32_t kl_run_group_staged(const uint8_t *p, uint32_t bytes, uint32_t nrun, uint32_t W,
+                                                        uint32_t magicg, uint32_t *bm, uint32_t bm_s, uint8_t *stage,
+                                                        uint32_t stage_s, uint8_t *row0, int lane, uint64_t pol) {
+    constexpr uint32_t LPR = 32 / G;                    // lanes per row
+    constexpr uint32_t rlen = 4u * WPLG;                // positions per lane
+    constexpr int NB = (int)((rlen + 31) / 32);         // bitmap words per lane
+    constexpr int BMS = NB <= 4 ? 4 : 8;                // ... allocated in 16-B units
+    constexpr uint32_t leaders = G == 2 ? 0x00010001u : 0x01010101u;
+    const uint32_t hl = (uint32_t)lane & (LPR - 1), hb = (uint32_t)lane & ~(LPR - 1), h = (uint32_t)lane / LPR;
     const bool fits = 4ull + 3ull * nrun <= bytes;
     const bool have = fits && hl < nrun;
     const uint32_t len = have ? __ldg(reinterpret_cast<const uint16_t *>(p + 4) + hl) : 0u;
     const uint32_t val = have ? __ldg(p + 4 + 2 * nrun + hl) : 0u;
-    const uint32_t incl = scan16_u32(len), st = incl - len;
-    const uint32_t tot = __shfl_sync(0xffffffffu, incl, (int)(hb | 15u));
+    const uint32_t incl = scan_seg_u32<LPR>(len), st = incl - len;
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, (int)(hb | (LPR - 1)));
     const uint32_t zero_len = __ballot_sync(0xffffffffu, have && len == 0);
-    const bool okh = fits && ((zero_len >> hb) & 0xFFFFu) == 0 && tot == W;
-    const uint32_t okm = __ballot_sync(0xffffffffu, okh) & 0x00010001u;
-    constexpr uint32_t rlen = 4u * WPL2;  // positions per lane
-    sts_u4(bm_s + 16u * (uint32_t)lane, make_uint4(0u, 0u, 0u, 0u));
+    const bool okh = fits && ((zero_len >> hb) & ((1u << LPR) - 1u)) == 0 && tot == W;
+    const uint32_t okm = __ballot_sync(0xffffffffu, okh) & leaders;
+#pragma unroll
+    for (int w = 0; w < BMS; w += 4) sts_u4(bm_s + 4u * (BMS * (uint32_t)lane + w), make_uint4(0u, 0u, 0u, 0u));
     __syncwarp();
     if (have && okh) {
-        const uint32_t o = __umulhi(st, magic2);  // st / rlen (exact: st < 2^16, rlen <= 72)
+        const uint32_t o = __umulhi(st, magicg);  // st / rlen (exact: st < 2^16, rlen <= 144)
         const uint32_t b = st - o * rlen;
-        atomicOr(bm + 4 * (hb | o) + (b >> 5), 1u << (b & 31));
+        atomicOr(bm + BMS * (hb | o) + (b >> 5), 1u << (b & 31));
     }
     __syncwarp();
-    const uint4 mm = lds_u4(bm_s + 16u * (uint32_t)lane);
-    const uint32_t c = __popc(mm.x) + __popc(mm.y) + __popc(mm.z);
-    const uint32_t before = scan16_u32(c) - c;  // run starts before this lane's first position
-    uint32_t idx = before + (mm.x & 1u) - 1u;  // run of the first position (run 0 starts at 0)
-    uint32_t r0 = mm.x & ~1u, r1 = mm.y, r2 = mm.z;
-    uint32_t v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & 15u))) * 0x01010101u;
-    uint32_t out[WPL2];
+    uint32_t mw[BMS];
 #pragma unroll
-    for (int k = 0; k < WPL2; k++) out[k] = v;
-    const uint32_t tmax = __reduce_max_sync(0xffffffffu, c - (mm.x & 1u));
+    for (int w = 0; w < BMS; w += 4) {
+        const uint4 q = lds_u4(bm_s + 4u * (BMS * (uint32_t)lane + w));
+        mw[w] = q.x, mw[w + 1] = q.y, mw[w + 2] = q.z, mw[w + 3] = q.w;
+    }
+    uint32_t c = 0;
+#pragma unroll
+    for (int w = 0; w < NB; w++) c += __popc(mw[w]);
+    const uint32_t first = mw[0] & 1u;
+    const uint32_t before = scan_seg_u32<LPR>(c) - c;  // run starts before this lane's first position
+    uint32_t idx = before + first - 1u;                 // run of the first position (run 0 starts at 0)
+    mw[0] &= ~1u;
+    uint32_t v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & (LPR - 1)))) * 0x01010101u;
+    uint32_t out[WPLG];
+#pragma unroll
+    for (int k = 0; k < WPLG; k++) out[k] = v;
+    const uint32_t tmax = __reduce_max_sync(0xffffffffu, c - first);
     for (uint32_t t = 0; t < tmax; t++) {  // one pass per run starting inside the lane's words
-        const bool has = (r0 | r1 | r2) != 0;
-        const uint32_t j = r0 ? __ffs(r0) - 1u : (r1 ? 31u + __ffs(r1) : 63u + __ffs(r2));
-        if (r0) r0 &= r0 - 1;
-        else if (r1) r1 &= r1 - 1;
-        else r2 &= r2 - 1;
+        bool has = false;
+        uint32_t j = 0;
+#pragma unroll
+        for (int w = 0; w < NB; w++) {  // the lowest remaining start
+            if (!has && mw[w]) {
+                j = 32u * w + __ffs(mw[w]) - 1u;
+                mw[w] &= mw[w] - 1;
+                has = true;
+            }
+        }
         idx += has;
-        v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & 15u))) * 0x01010101u;
+        v = __shfl_sync(0xffffffffu, val, (int)(hb | (idx & (LPR - 1)))) * 0x01010101u;
         if (has) {
             const int j8 = 8 * (int)j;
 #pragma unroll
-            for (int k = 0; k < WPL2; k++) {  // bytes at or after j take v
+            for (int k = 0; k < WPLG; k++) {  // bytes at or after j take v
                 const uint32_t take = ones_shl((uint32_t)max(j8 - 32 * k, 0));
                 out[k] = (out[k] & ~take) | (v & take);
             }
         }
     }
     const uint32_t lo = stage_s + h * W + rlen * hl;
-    if constexpr ((WPL2 & 1) == 0) {
+    static_assert((WPLG & 1) == 0, "row groups stage 8-byte pairs of words");
 #pragma unroll
-        for (int k = 0; k < WPL2; k += 2) sts_u2(lo + 4u * k, make_uint2(out[k], out[k + 1]));
-    } else {
-#pragma unroll
-        for (int k = 0; k < WPL2; k++) sts_f32(lo + 4u * k, __uint_as_float(out[k]));
-    }
+    for (int k = 0; k < WPLG; k += 2) sts_u2(lo + 4u * k, make_uint2(out[k], out[k + 1]));
     fence_proxy_async_smem();  // this lane's staged words -> visible to the bulk store
     __syncwarp();
     if (lane == 0 && okm) {
-        if (okm == 0x00010001u) kl_store(row0, stage, 2 * W, pol);
-        else if (okm & 1u) kl_store(row0, stage, W, pol);
-        else kl_store(row0 + W, stage + W, W, pol);
+        if (okm == leaders) {
+            kl_store(row0, stage, G * W, pol);
+        } else {
+#pragma unroll
+            for (int r = 0; r < G; r++)
+                if ((okm >> (LPR * r)) & 1u) kl_store(row0 + r * W, stage + r * W, W, pol);
+        }
     }
     return okm;
 }
@@ -232,18 +257,21 @@ __device__ __forceinline__ uint64_t label_header_ok(const uint8_t *b, uint64_t l
     return ok ? total : 0;
 }
 
-template <int WPL, int WPL2>  // WPL 0: no staged rows (W % 16 != 0, W > 2048 or an unaligned dst); WPL2 0: no row pairs
-__global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *const *__restrict__ src,
+template <int WPL, int WPLQ>  // WPL 0: no staged rows (W % 16 != 0, W > 2048 or an unaligned dst);
+                              // WPLQ: words per lane of a 4-row group (W / 32), 0: no row groups
+__global__ void __launch_bounds__(kKlWarps * kWarp, WPLQ > 0 ? SPP_KL_GROUP_MINB : 4) kl_decode_mask(const void *const *__restrict__ src,
                                                                    const uint64_t *__restrict__ src_bytes, int n,
                                                                    uint32_t H, uint32_t W, uint8_t *__restrict__ dst,
                                                                    uint32_t *__restrict__ status, uint32_t row_ef) {
-    __shared__ uint32_t bitmap[kKlWarps][kKlChunk / 32];
+    __shared__ uint32_t bitmap[kKlWarps][WPLQ > 0 ? 256 : kKlChunk / 32];  // 4-row groups: 8 words per lane
     __shared__ __align__(128) uint8_t stage_rows[kKlWarps][2][kKlStageW];  // double-buffered staging rows
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t *bm = bitmap[warp];
     const uint32_t bm_s = smem_u32(bm);
     const uint32_t magic = 0xFFFFFFFFu / (4u * (WPL > 0 ? WPL : 1)) + 1u;
+    constexpr int WPL2 = WPLQ / 2;  // words per lane of a row pair
     const uint32_t magic2 = 0xFFFFFFFFu / (4u * (WPL2 > 0 ? WPL2 : 1)) + 1u;
+    const uint32_t magic4 = 0xFFFFFFFFu / (4u * (WPLQ > 0 ? WPLQ : 1)) + 1u;
     uint32_t nstaged = 0;  // rows this warp has stored by TMA (buffer nstaged & 1 next)
     uint64_t pol;
     if (row_ef) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
@@ -283,29 +311,51 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
         }
     };
     for (uint64_t g = g0; g < g1; g++) {
-        if constexpr (WPL2 > 0) {
-            // two RUN rows of <= 16 runs each: one half-warp per row, one bulk store
+        if constexpr (WPLQ > 0) {
+            // G consecutive RUN rows of <= 32/G runs each (4, else 2): one 32/G-lane segment
+            // per row, one bulk store per group.  The group's staging buffer is the warp's
+            // whole staging area, so every staged store first waits for the previous one
+            // to have read shared memory (bulk_wait_read_all below).
+            auto group_ok = [&](int G, uint32_t maxruns, int kk) {
+                const int src = kk + min(lane, G - 1);  // lanes >= G repeat row G - 1
+                const uint32_t hr = __shfl_sync(0xffffffffu, w_hdr, src);
+                const bool good = __shfl_sync(0xffffffffu, w_ok, src) && (hr & 0xFFu) == 1u && (hr >> 16) >= 1 &&
+                                  (hr >> 16) <= maxruns;
+                return __all_sync(0xffffffffu, good) != 0;
+            };
+            auto run_group = [&](auto gtag, int kk) {
+                constexpr int G = decltype(gtag)::value;
+                constexpr uint32_t LPR = 32 / G;
+                const int kh = kk + lane / (int)LPR;
+                const uint8_t *p = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_p, kh));
+                const uint32_t bytes = __shfl_sync(0xffffffffu, w_bytes, kh);
+                const uint32_t nrun = __shfl_sync(0xffffffffu, w_hdr, kh) >> 16;
+                uint8_t *stage = &stage_rows[warp][0][0];
+                if (lane == 0) bulk_wait_read_all();  // the previous store has read the staging area
+                __syncwarp();
+                constexpr int WG = G == 4 ? (WPLQ > 0 ? WPLQ : 2) : (WPL2 > 0 ? WPL2 : 2);
+                const uint32_t okm = kl_run_group_staged<G, WG>(p, bytes, nrun, W, G == 4 ? magic4 : magic2, bm,
+                                                                bm_s, stage, smem_u32(stage), dst + g * (uint64_t)W,
+                                                                lane, pol);
+                if (lane == 0)
+                    for (int r = 0; r < G; r++)
+                        if (!((okm >> (LPR * r)) & 1u)) report(status, SPP_ERR_CORRUPT, (int64_t)((g + r) / H));
+            };
+            if (SPP_KL_QUADS && g + 3 < g1) {
+                if (g == g0 || g + 3 >= wbase + kWarp) load_window(g);
+                const int kk = (int)(g - wbase);
+                if (group_ok(4, 8, kk)) {
+                    run_group(std::integral_constant<int, 4>{}, kk);
+                    g += 3;
+                    continue;
+                }
+            }
             if (g + 1 < g1) {
                 if (g == g0 || g + 1 >= wbase + kWarp) load_window(g);
                 const int kk = (int)(g - wbase);
-                const uint32_t h0 = __shfl_sync(0xffffffffu, w_hdr, kk), h1 = __shfl_sync(0xffffffffu, w_hdr, kk + 1);
-                const bool pair_ok = __shfl_sync(0xffffffffu, w_ok, kk) && __shfl_sync(0xffffffffu, w_ok, kk + 1) &&
-                                     (h0 & 0xFFu) == 1u && (h1 & 0xFFu) == 1u && (h0 >> 16) >= 1 &&
-                                     (h0 >> 16) <= kKlPairRuns && (h1 >> 16) >= 1 && (h1 >> 16) <= kKlPairRuns;
-                if (pair_ok) {
-                    const int kh = kk + (lane >> 4);
-                    const uint8_t *p = reinterpret_cast<const uint8_t *>(__shfl_sync(0xffffffffu, w_p, kh));
-                    const uint32_t bytes = __shfl_sync(0xffffffffu, w_bytes, kh);
-                    const uint32_t nrun = (lane >> 4 ? h1 : h0) >> 16;
-                    uint8_t *stage = stage_rows[warp][nstaged & 1];
-                    if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
-                    __syncwarp();
-                    const uint32_t okm = kl_run_pair_staged<(WPL2 > 0 ? WPL2 : 1)>(
-                        p, bytes, nrun, W, magic2, bm, bm_s, stage, smem_u32(stage), dst + g * (uint64_t)W, lane, pol);
-                    nstaged += okm != 0;
-                    if (lane == 0 && !(okm & 1u)) report(status, SPP_ERR_CORRUPT, (int64_t)(g / H));
-                    if (lane == 0 && !(okm >> 16)) report(status, SPP_ERR_CORRUPT, (int64_t)((g + 1) / H));
-                    g++;
+                if (group_ok(2, kKlPairRuns, kk)) {
+                    run_group(std::integral_constant<int, 2>{}, kk);
+                    g += 1;
                     continue;
                 }
             }
@@ -330,8 +380,11 @@ __global__ void __launch_bounds__(kKlWarps * kWarp) kl_decode_mask(const void *c
                 }
             }
         } else if (WPL > 0 && ok && mode == 1 && (hdr >> 16) >= 1 && (hdr >> 16) <= kKlFastRuns) {
-            uint8_t *stage = stage_rows[warp][nstaged & 1];
-            if (lane == 0) bulk_wait_read_1();  // the store that last used this buffer has read it
+            uint8_t *stage = stage_rows[warp][WPLQ > 0 ? 0 : nstaged & 1];
+            if (lane == 0) {  // the store that last used this buffer has read it
+                if constexpr (WPLQ > 0) bulk_wait_read_all();  // (a group store may cover both buffers)
+                else bulk_wait_read_1();
+            }
             __syncwarp();
             ok = kl_run_row_staged<(WPL > 0 ? WPL : 1)>(p, (uint32_t)bytes, hdr >> 16, W, magic, bm, bm_s, stage, smem_u32(stage),
                                         row, lane, pol);
@@ -442,22 +495,22 @@ spp_status labels_decode(int kind, const void *const *d_src, const uint64_t *src
         // staged rows leave by TMA bulk store: 16-B aligned rows of a multiple of 16 bytes
         const bool staged = (W % 16) == 0 && W <= (int)kKlFastW && (reinterpret_cast<uintptr_t>(d_dst) & 15) == 0;
         const int wpl = staged ? (W / 4 + kWarp - 1) / kWarp : 0;
-        // row pairs (one half-warp per row, one bulk store per pair): W % 128 == 0, 2W <= kKlStageW
-        const bool pairs = staged && W % 128 == 0 && 2 * W <= (int)kKlStageW;
+        // row groups (4 or 2 rows per warp, one bulk store per group): W % 128 == 0, 4W <= 2 kKlStageW
+        const bool groups = staged && W % 128 == 0 && 4 * W <= 2 * (int)kKlStageW;
         void (*kern)(const void *const *, const uint64_t *, int, uint32_t, uint32_t, uint8_t *, uint32_t *,
                      uint32_t) = nullptr;
-        switch (pairs ? 100 + wpl : wpl) {
+        switch (groups ? 100 + wpl : wpl) {
 #define SPP_KL_CASE(k) \
     case k: kern = kl_decode_mask<k, 0>; break;
-#define SPP_KL_PAIR(k) \
-    case 100 + k: kern = kl_decode_mask<k, 2 * k>; break;
+#define SPP_KL_GROUP(k) \
+    case 100 + k: kern = kl_decode_mask<k, 4 * k>; break;
             SPP_KL_CASE(0) SPP_KL_CASE(1) SPP_KL_CASE(2) SPP_KL_CASE(3) SPP_KL_CASE(4) SPP_KL_CASE(5) SPP_KL_CASE(6)
             SPP_KL_CASE(7) SPP_KL_CASE(8) SPP_KL_CASE(9) SPP_KL_CASE(10) SPP_KL_CASE(11) SPP_KL_CASE(12)
             SPP_KL_CASE(13) SPP_KL_CASE(14) SPP_KL_CASE(15) SPP_KL_CASE(16)
-            SPP_KL_PAIR(1) SPP_KL_PAIR(2) SPP_KL_PAIR(3) SPP_KL_PAIR(4) SPP_KL_PAIR(5) SPP_KL_PAIR(6)
-            SPP_KL_PAIR(7) SPP_KL_PAIR(8) SPP_KL_PAIR(9)
+            SPP_KL_GROUP(1) SPP_KL_GROUP(2) SPP_KL_GROUP(3) SPP_KL_GROUP(4) SPP_KL_GROUP(5) SPP_KL_GROUP(6)
+            SPP_KL_GROUP(7) SPP_KL_GROUP(8) SPP_KL_GROUP(9)
 #undef SPP_KL_CASE
-#undef SPP_KL_PAIR
+#undef SPP_KL_GROUP
             default: return SPP_ERR_INVALID_ARG;
         }
         // 8 CTAs per SM: about two waves of the pair instance (4 resident per SM); measured

@@ -58,7 +58,8 @@ def test_label_masks_lossless(dev, orc, H, W):
     (verbatim rows), constant masks, W not a multiple of 16, W over the 1,024-
     position chunk; rows of exactly 1..40 runs (the staged path takes <= 32 runs
     with W % 16 == 0 and W <= 2048: 1152, 2048, 16, 1040 with a partial last
-    lane, 48; 2304 takes the general path; row pairs -- one half-warp per row, <= 16 runs each -- when
+    lane, 48; 2304 takes the general path; row pairs -- 2 rows of <= 16 runs,
+    one half-warp per row (4-row groups of <= 8 runs with SPP_KL_QUADS) -- when
     W % 128 == 0 and W <= 1152: 1152, 1024, 128, odd H); mixed in one batch,
     bit-exact vs the masks and the oracle."""
     from synth import gen_deepcam_labels
@@ -108,20 +109,22 @@ def test_label_corruption_detected(dev):
 
 
 def test_label_row_pairs_corruption_and_neighbours(dev):
-    """Row pairs (W % 128 == 0): a corrupt run length in the first or the
-    second row of a pair is reported on its sample and the other samples of
-    the batch decode bit-exactly; rows of 16 and 17 runs side by side (a pair
-    falls back to single rows when either has more than 16 runs)."""
+    """Row pairs (W % 128 == 0: 2 rows of <= 16 runs, else one row per warp;
+    4-row groups of <= 8 runs first with SPP_KL_QUADS): a corrupt run length
+    in any row of a group is reported on its sample and the other samples of
+    the batch decode bit-exactly; rows of 8/9 and 16/17 runs side by side (a
+    group falls back to a smaller one when a row has too many runs)."""
     from synth import gen_deepcam_labels
     from paper_conf_ipps_ibrahimo22_b200 import spp
     rng = np.random.default_rng(42)
     H, W = 24, 1152
     m16 = _runs_mask(rng, 40, W)[14:14 + H]  # rows of 15..38 runs: pairs of <= 16 and > 16 runs mixed
-    masks = [gen_deepcam_labels(71, H=H, W=W), m16, gen_deepcam_labels(72, H=H, W=W)]
+    m8 = _runs_mask(rng, 40, W)[np.r_[0:8, 8:12, 4:12, 0:4]]  # rows of 1..12 runs: quads, pairs around 8/9
+    masks = [gen_deepcam_labels(71, H=H, W=W), m16, gen_deepcam_labels(72, H=H, W=W), m8]
     bufs = [spp.spp_encode_label_mask(m) for m in masks]
     got, st = _decode("mask", bufs, (H, W), src_bytes=True)
     assert st == 0 and np.array_equal(got, np.stack(masks))
-    for y in (0, 1, 6, 7, H - 1):
+    for y in (0, 1, 2, 3, 6, 7, H - 1):
         bad = bufs[0].copy()
         h = fmt.label_header(bad)
         row = h["payload_off"] + int(h["dir"][y])
