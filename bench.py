@@ -584,9 +584,9 @@ def main():
         line["secondary"] = sec
     if variant:
         line["variant_escape_keys"] = variant
-    print(json.dumps(line), flush=True)
-    if dist:
+    if dist:  # NCCL's teardown log lines (NCCL_DEBUG=INFO, stdout) come before the JSON line
         dist.destroy_process_group()
+    print(json.dumps(line), flush=True)
 
 
 def run_reference(args, W):
