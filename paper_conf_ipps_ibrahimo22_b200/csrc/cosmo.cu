@@ -88,6 +88,9 @@ constexpr int kKeyStages = SPP_KC_STAGES;  // TMA ring of key tiles
 // key tiles are read once: their TMA loads carry an L2 evict_first hint so they do
 // not displace the LUT tails (evict_last) and cold rows (r2: C2 0.817 -> 0.834,
 // dense C5 rows +1-3 points; profiles/r02a3_*, r02a5_*)
+#ifndef SPP_KC_BAD_MAX
+#define SPP_KC_BAD_MAX 1
+#endif
 #ifndef SPP_KC_KEY_EF
 #define SPP_KC_KEY_EF 1
 #endif
@@ -251,9 +254,14 @@ template <int OUT, bool SMEM>
 __device__ __forceinline__ typename Entry<OUT>::T make_entry(uint2 e, const FuView &fu, uint32_t &bad) {
     uint32_t idx[4] = {e.x & 0xFFFFu, e.x >> 16, e.y & 0xFFFFu, e.y >> 16};
     float f[4];
+#if SPP_KC_BAD_MAX  // one compare of the largest index instead of four
+    bad |= max(max(idx[0], idx[1]), max(idx[2], idx[3])) >= fu.nU;
+#endif
 #pragma unroll
     for (int c = 0; c < 4; c++) {
+#if !SPP_KC_BAD_MAX
         bad |= idx[c] >= fu.nU;
+#endif
         const uint32_t i = min(idx[c], fu.nU - 1);
         if constexpr (SMEM) f[c] = lds_f32(fu.smem + 4 * i);
         else f[c] = ld_ro_f32(fu.global + i);
