@@ -212,7 +212,12 @@ size_t spp_decoded_sample_bytes(spp_format fmt, const spp_decode_opts *opts);
  *           16-B aligned
  * Launches the sm_100a kernels (CosmoFlow: transform of the unique values then
  * the fused LUT expansion; DeepCAM: header/directory parse then the warp-per-line
- * differential decode) on `stream`.  Returns after enqueueing. */
+ * differential decode) on `stream`.  Returns after enqueueing.
+ * L2 residency of the output: CosmoFlow stores it as streaming (evict-first)
+ * data; DeepCAM rows are stored with an L2 evict_first hint when the launch
+ * writes more than 64 MB (batches) and with normal priority below that, so a
+ * small batch's output can still be in L2 for its consumer.  Compressed inputs
+ * are read once (CosmoFlow key tiles carry an evict_first hint). */
 spp_status spp_decode_batch(spp_format fmt, const void *const *d_src, int n, void *d_dst,
                             const spp_decode_opts *opts, spp_stream_t stream);
 
@@ -282,7 +287,8 @@ spp_status spp_encode_label_vector(const float *v, int n, void *dst, size_t dst_
  *   src_bytes : optional device u64[n] bounding each stream's reads (NULL = trust the header)
  *   status    : optional device word, as spp_decode_opts.status (a stream whose header does not match
  *               kind/H/W, or a malformed row, sets SPP_ERR_CORRUPT | sample << 8)
- * Host-checkable errors (n < 0, null pointers, bad kind/dims) return SPP_ERR_INVALID_ARG. */
+ * Host-checkable errors (n < 0, null pointers, bad kind/dims) return SPP_ERR_INVALID_ARG.
+ * Masks are stored with an L2 evict_first hint when the launch writes more than 64 MB. */
 spp_status spp_decode_labels(int kind, const void *const *d_src, const uint64_t *src_bytes, int n, void *d_dst,
                              int H, int W, uint32_t *status, spp_stream_t stream);
 
