@@ -135,6 +135,22 @@ def test_label_row_pairs_corruption_and_neighbours(dev):
         assert np.array_equal(got[0], masks[2]) and np.array_equal(got[2], masks[1])
 
 
+def test_label_masks_large_launch(dev):
+    """A launch writing more than 64 MB of masks (96 paper-shaped 768 x 1152
+    masks: the row stores take the L2 evict_first policy) decodes
+    bit-exactly, like the small launches above."""
+    from synth import gen_deepcam_labels
+    from paper_conf_ipps_ibrahimo22_b200 import spp
+    masks = [gen_deepcam_labels(6100 + i) for i in range(4)]
+    bufs = [spp.spp_encode_label_mask(m) for m in masks]
+    n = 96
+    assert n * 768 * 1152 > 64 << 20
+    got, st = _decode("mask", [bufs[i % 4] for i in range(n)], (768, 1152), src_bytes=True)
+    assert st == 0
+    for i in range(n):
+        assert np.array_equal(got[i], masks[i % 4]), i
+
+
 @pytest.mark.parametrize("source", ["device", "host"])
 def test_loader_delivers_labels(dev, orc, source):
     """DecodeLoader with labels: every batch's decoded samples AND labels match
